@@ -1,0 +1,133 @@
+/*
+ * spinfer.h — C ABI of the B200 (sm_100a) TCA-BME SpMM library (libspinfer.so).
+ *
+ * The operation (§2.1, §2.3): Y = W x X with
+ *   W in R^{M x K}  — an fp16 weight matrix, unstructured-sparse (30-70% zeros,
+ *                     P:13), stored in TCA-BME (§4.2);
+ *   X in R^{K x N}  — fp16 activations, N = decode tokens;
+ *   Y in R^{M x N}  — fp16 output, fp32 accumulation (Listing 1).
+ *
+ * TCA-BME: 8x8 BitmapTiles (one uint64 bitmap each) grouped
+ * 2x2 column-major into 16x16 TCTiles, TCTiles column-major inside
+ * 64x64 GroupTiles, GroupTiles row-major. Three arrays:
+ *   gtile_offset int32[NGT+1], NGT = (M/64)(K/64): start (in fp16 elements) of
+ *                each GroupTile's values, gtile_offset[0] = 0,
+ *                gtile_offset[NGT] = n_values;
+ *   bitmap       uint64[NBT], NBT = M*K/64, in GroupTile -> TCTile -> BitmapTile
+ *                order; bit b <-> (row b/8, col b%8) of the BitmapTile;
+ *   values       fp16[n_values], non-zeros in the same nested order, ascending
+ *                bit order inside a BitmapTile; each GroupTile's
+ *                segment is padded with +0.0 to a multiple of 8 halves (16 B,
+ *                P:266). Storage = eq. (9) + padding (<= 7 halves/GT).
+ * "Non-zero" means (bits & 0x7FFF) != 0: -0.0 is dropped, NaN/Inf are kept.
+ * All readings of silent/garbled points are listed in DESIGN.md.
+ *
+ * Conventions for every call:
+ *  - Pointers are DEVICE pointers unless marked (host). fp16 is passed as
+ *    uint16_t bit patterns. Matrices are row-major and contiguous.
+ *  - Device pointers must be 16-byte aligned (cp.async.bulk requirement).
+ *  - All buffers are owned and allocated by the CALLER; the library keeps no
+ *    state and allocates no persistent memory (encode_count uses one 64-byte
+ *    stream-ordered temporary). Calls are stream-ordered and asynchronous
+ *    except spinfer_encode_count, which synchronizes `stream`.
+ *  - Every function returns a spinfer_status; nothing aborts, no exception
+ *    crosses the ABI. Asynchronous device faults surface at the caller's next
+ *    synchronization (as a CUDA error there).
+ *  - `stream` is a cudaStream_t passed as void* (0 = legacy default stream).
+ *  - Requires an sm_100 device (SPINFER_ENODEV otherwise).
+ */
+#ifndef SPINFER_H_
+#define SPINFER_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    SPINFER_OK = 0,
+    SPINFER_EINVAL = -1,     /* null pointer, bad shape (M or K not a positive multiple of 64,
+                                N not in {8,16,24,32}), misaligned pointer, struct/call mismatch */
+    SPINFER_ENOSPC = -2,     /* workspace too small */
+    SPINFER_EOVERFLOW = -3,  /* n_values would reach 2^31 (gtile_offset is int32) */
+    SPINFER_ECUDA = -4,      /* CUDA launch/runtime error */
+    SPINFER_ENODEV = -5      /* current device is not sm_100 */
+} spinfer_status;
+
+#if defined(__GNUC__)
+#define SPINFER_API __attribute__((visibility("default")))
+#else
+#define SPINFER_API
+#endif
+
+#define SPINFER_GT 64        /* GroupTile edge GT_H = GT_W (paper silent; reading A1) */
+
+/* Host-side descriptor of one TCA-BME matrix. The three device arrays are
+ * caller-owned (e.g. torch tensors). */
+typedef struct {
+    int32_t M, K;             /* M % 64 == 0, K % 64 == 0 */
+    int32_t gt_h, gt_w;       /* must be 64, 64 */
+    int64_t nnz;              /* true non-zeros (informational) */
+    int64_t n_values;         /* == gtile_offset[NGT] (padded count), < 2^31 */
+    int32_t max_gt_values;    /* max_g (gtile_offset[g+1]-gtile_offset[g]) — sizes the SpMM
+                                 pipeline stages; <= 0 means unknown (assume 4096, dense) */
+    int32_t reserved;
+    int32_t *gtile_offset;    /* device [NGT+1] */
+    uint64_t *bitmap;         /* device [NBT] */
+    uint16_t *values;         /* device [max(n_values,8)] fp16 bits */
+} spinfer_tca;
+
+/* Encode, phase 1 (P:196 sizes; GPU encoder, not described by the paper).
+ * W: device fp16 [M][K]. Writes gtile_offset[0..NGT] (device, caller-allocated
+ * NGT+1 int32) and returns to the HOST n_values (padded), nnz and max_gt_values.
+ * Synchronizes `stream`. SPINFER_EOVERFLOW if n_values >= 2^31. */
+SPINFER_API int spinfer_encode_count(const uint16_t *W, int M, int K, int32_t *gtile_offset,
+                         int64_t *n_values /* host */, int64_t *nnz /* host */,
+                         int32_t *max_gt_values /* host, may be NULL */, void *stream);
+
+/* Encode, phase 2: fills T->bitmap (NBT uint64) and T->values (n_values fp16,
+ * padding written as +0.0) from W, using T->gtile_offset from phase 1.
+ * T (host struct) must carry M, K, gt_h = gt_w = 64 and the three device pointers. */
+SPINFER_API int spinfer_encode_fill(const uint16_t *W, const spinfer_tca *T, void *stream);
+
+/* Decode TCA-BME -> dense fp16 W_out [M][K] (device); unset bits give +0.0. */
+SPINFER_API int spinfer_decode(const spinfer_tca *T, uint16_t *W_out, void *stream);
+
+/* Bytes of device workspace spinfer_spmm needs for this shape (split-K partials
+ * and fix-up counters). The workspace must be ZERO-FILLED before its first use;
+ * every spinfer_spmm call leaves the counter region zero again, so one zeroed
+ * workspace can be reused by successive calls on ONE stream (not concurrently). */
+SPINFER_API size_t spinfer_spmm_workspace_bytes(int M, int K, int N);
+
+/* Y = W x X with fp32 accumulation and one round-to-nearest-even to
+ * fp16 per output. X: device fp16 [K][N] row-major; Y: device fp16
+ * [M][N] row-major (fully overwritten). N in {8, 16, 24, 32} (decode batch,
+ * P:329). One persistent kernel launch (stream-K over GroupTiles with an
+ * in-kernel split-K fix-up, P:216 / Alg. 1). */
+SPINFER_API int spinfer_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N,
+                 void *workspace, size_t ws_bytes, void *stream);
+
+/* Tensor-parallel row partition: rank `rank` of `world` owns rows
+ * [*row_begin, *row_begin + *row_count) — contiguous, multiples of 64, sizes
+ * differ by at most 64 (host only). */
+SPINFER_API int spinfer_tp_rows(int M, int world, int rank, int *row_begin /* host */, int *row_count /* host */);
+
+/* Row-partitioned SpMM: T_shard encodes W[row_begin : row_begin+row_count, :]
+ * (as returned by spinfer_tp_rows(M_full, world, rank)); writes ONLY those rows
+ * of Y_full [M_full][N]. Performs no communication: the caller gathers Y_full
+ * (e.g. NCCL all-gather) when the next layer needs it. */
+SPINFER_API int spinfer_spmm_tp(const spinfer_tca *T_shard, const uint16_t *X, uint16_t *Y_full, int M_full,
+                    int K, int N, int world, int rank, void *workspace, size_t ws_bytes, void *stream);
+
+/* Static string for a status code. */
+SPINFER_API const char *spinfer_status_str(int status);
+
+/* Library build/version info (host string). */
+SPINFER_API const char *spinfer_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPINFER_H_ */

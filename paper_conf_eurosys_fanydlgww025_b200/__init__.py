@@ -1,0 +1,236 @@
+"""spinfer-b200: TCA-BME SpMM (SpInfer, EuroSys '25) for B200 / sm_100a.
+
+Thin Python binding over the C ABI in include/spinfer.h (libspinfer.so, built
+in-tree by build.py). This module only marshals arguments: every step of the
+path (encode, decode, SpMM, split-K fix-up) runs in the library's CUDA kernels.
+PyTorch supplies device memory, streams and (in tp.py) process groups. There is
+no CPU fallback: if the library or a CUDA device is missing, calls raise.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import torch
+
+__all__ = ["TCA", "SpinferError", "encode", "decode", "spmm", "spmm_tp", "tp_rows", "workspace",
+           "workspace_bytes", "storage_bytes", "algorithmic_bytes", "lib", "LIB_PATH"]
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libspinfer.so")
+GT = 64
+
+_STATUS = {0: "SPINFER_OK", -1: "SPINFER_EINVAL", -2: "SPINFER_ENOSPC", -3: "SPINFER_EOVERFLOW",
+           -4: "SPINFER_ECUDA", -5: "SPINFER_ENODEV"}
+
+
+class SpinferError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        self.status = status
+        super().__init__(f"{what}: {_STATUS.get(status, status)} ({status})")
+
+
+class _Tca(ctypes.Structure):
+    _fields_ = [("M", ctypes.c_int32), ("K", ctypes.c_int32), ("gt_h", ctypes.c_int32), ("gt_w", ctypes.c_int32),
+                ("nnz", ctypes.c_int64), ("n_values", ctypes.c_int64), ("max_gt_values", ctypes.c_int32),
+                ("reserved", ctypes.c_int32), ("gtile_offset", ctypes.c_void_p), ("bitmap", ctypes.c_void_p),
+                ("values", ctypes.c_void_p)]
+
+
+_lib = None
+
+# Exported symbols (must match include/spinfer.h; checked by tests/test_abi.py).
+SYMBOLS = ["spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spinfer_spmm_workspace_bytes",
+           "spinfer_spmm", "spinfer_tp_rows", "spinfer_spmm_tp", "spinfer_status_str", "spinfer_version"]
+
+
+def lib() -> ctypes.CDLL:
+    """Load libspinfer.so (raises if it was not built: no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise RuntimeError(f"{LIB_PATH} is missing: run `python -c 'import __graft_entry__ as g; g.build()'` "
+                           "(nvcc, sm_100a). There is no CPU fallback.")
+    L = ctypes.CDLL(LIB_PATH)
+    vp, i32, i64, sz = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_size_t
+    P = ctypes.POINTER
+    L.spinfer_encode_count.argtypes = [vp, i32, i32, vp, P(ctypes.c_int64), P(ctypes.c_int64), P(ctypes.c_int32), vp]
+    L.spinfer_encode_fill.argtypes = [vp, P(_Tca), vp]
+    L.spinfer_decode.argtypes = [P(_Tca), vp, vp]
+    L.spinfer_spmm_workspace_bytes.argtypes = [i32, i32, i32]
+    L.spinfer_spmm_workspace_bytes.restype = sz
+    L.spinfer_spmm.argtypes = [P(_Tca), vp, vp, i32, i32, i32, vp, sz, vp]
+    L.spinfer_tp_rows.argtypes = [i32, i32, i32, P(ctypes.c_int), P(ctypes.c_int)]
+    L.spinfer_spmm_tp.argtypes = [P(_Tca), vp, vp, i32, i32, i32, i32, i32, vp, sz, vp]
+    L.spinfer_status_str.argtypes = [i32]
+    L.spinfer_status_str.restype = ctypes.c_char_p
+    L.spinfer_version.restype = ctypes.c_char_p
+    for f in ("spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spinfer_spmm", "spinfer_tp_rows",
+              "spinfer_spmm_tp"):
+        getattr(L, f).restype = ctypes.c_int
+    _lib = L
+    return L
+
+
+def _check(rc: int, what: str):
+    if rc != 0:
+        raise SpinferError(rc, what)
+
+
+def _stream(stream=None) -> int:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return int(s.cuda_stream)
+
+
+def _dev_u16(t: torch.Tensor, name: str) -> torch.Tensor:
+    if not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA tensor")
+    if t.dtype == torch.float16:
+        t = t.view(torch.int16)
+    if t.dtype not in (torch.int16, torch.uint16):
+        raise ValueError(f"{name} must be float16 (got {t.dtype})")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    return t
+
+
+@dataclass
+class TCA:
+    """A TCA-BME matrix: three device tensors + sizes."""
+    M: int
+    K: int
+    gtile_offset: torch.Tensor   # int32 [NGT+1]
+    bitmap: torch.Tensor         # int64 (uint64 bits) [NBT]
+    values: torch.Tensor         # float16 [max(n_values, 8)]
+    n_values: int
+    nnz: int
+    max_gt_values: int
+
+    def c_struct(self) -> _Tca:
+        return _Tca(self.M, self.K, GT, GT, self.nnz, self.n_values, self.max_gt_values, 0,
+                    self.gtile_offset.data_ptr(), self.bitmap.data_ptr(), self.values.data_ptr())
+
+    def storage_bytes(self) -> int:
+        return storage_bytes(self.M, self.K, self.n_values)
+
+    def shard(self, row_begin: int, row_count: int) -> "TCA":
+        """Zero-copy row shard: GT rows [a, b) are a contiguous slice of all three
+        arrays; GTileOffset is rebased (on device) by the shard's first offset."""
+        if row_begin % GT or row_count % GT:
+            raise ValueError("shard rows must be multiples of 64")
+        KG = self.K // GT
+        a, b = row_begin // GT, (row_begin + row_count) // GT
+        off = self.gtile_offset[a * KG: b * KG + 1]
+        base = int(off[0].item())
+        end = int(off[-1].item())
+        new_off = (off - base).contiguous()
+        vals = self.values[base:max(end, base + 8)]
+        if base % 8:
+            raise AssertionError("GT value segments are 16-byte aligned by construction")
+        return TCA(row_count, self.K, new_off, self.bitmap[a * KG * 64: b * KG * 64], vals, end - base, -1,
+                   self.max_gt_values)
+
+
+def storage_bytes(M: int, K: int, n_values: int) -> int:
+    """Buffer bytes of a TCA-BME matrix: eq. (9) with the padded value count."""
+    return 4 * ((M // GT) * (K // GT) + 1) + 8 * (M * K // 64) + 2 * n_values
+
+
+def algorithmic_bytes(T: TCA, N: int) -> int:
+    """Bytes the SpMM must move: the whole TCA-BME matrix,
+    X [K][N] and Y [M][N] in fp16."""
+    return T.storage_bytes() + 2 * T.K * N + 2 * T.M * N
+
+
+def encode(W: torch.Tensor, stream=None) -> TCA:
+    """Dense fp16 W [M][K] (CUDA) -> TCA-BME on the same device (GPU encoder, bit-exact
+    with the oracle). One host synchronization (the value count readback)."""
+    W = _dev_u16(W, "W")
+    if W.dim() != 2:
+        raise ValueError("W must be 2-D")
+    M, K = W.shape
+    L = lib()
+    st = _stream(stream)
+    with torch.cuda.device(W.device):
+        off = torch.empty((M // GT) * (K // GT) + 1 if M % GT == 0 and K % GT == 0 else 1, dtype=torch.int32,
+                          device=W.device)
+        nv, nz, mx = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int32()
+        _check(L.spinfer_encode_count(W.data_ptr(), M, K, off.data_ptr(), ctypes.byref(nv), ctypes.byref(nz),
+                                      ctypes.byref(mx), st), "spinfer_encode_count")
+        bm = torch.empty(M * K // 64, dtype=torch.int64, device=W.device)
+        vals = torch.empty(max(nv.value, 8), dtype=torch.float16, device=W.device)
+        T = TCA(M, K, off, bm, vals, int(nv.value), int(nz.value), int(mx.value))
+        cs = T.c_struct()
+        _check(L.spinfer_encode_fill(W.data_ptr(), ctypes.byref(cs), st), "spinfer_encode_fill")
+    return T
+
+
+def decode(T: TCA, stream=None) -> torch.Tensor:
+    """TCA-BME -> dense fp16 [M][K] (unset bits -> +0.0)."""
+    out = torch.empty((T.M, T.K), dtype=torch.float16, device=T.bitmap.device)
+    cs = T.c_struct()
+    with torch.cuda.device(out.device):
+        _check(lib().spinfer_decode(ctypes.byref(cs), out.data_ptr(), _stream(stream)), "spinfer_decode")
+    return out
+
+
+def workspace_bytes(M: int, K: int, N: int) -> int:
+    with torch.cuda.device(torch.cuda.current_device()):
+        return int(lib().spinfer_spmm_workspace_bytes(M, K, N))
+
+
+_ws_cache: dict = {}
+
+
+def workspace(M: int, K: int, N: int, device=None) -> torch.Tensor:
+    """A zero-filled workspace for spinfer_spmm (cached per device; one stream at a time)."""
+    dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+    with torch.cuda.device(dev):
+        need = max(int(lib().spinfer_spmm_workspace_bytes(M, K, N)), 256)
+    ws = _ws_cache.get(dev)
+    if ws is None or ws.numel() < need:
+        ws = torch.zeros(need, dtype=torch.uint8, device=dev)
+        _ws_cache[dev] = ws
+    return ws
+
+
+def spmm(T: TCA, X: torch.Tensor, Y: torch.Tensor | None = None, ws: torch.Tensor | None = None,
+         stream=None) -> torch.Tensor:
+    """Y = W X: X fp16 [K][N] (CUDA), N in {8,16,24,32}; returns fp16 [M][N]."""
+    X = _dev_u16(X, "X")
+    K, N = X.shape
+    if K != T.K:
+        raise ValueError(f"X has K={K}, W has K={T.K}")
+    if Y is None:
+        Y = torch.empty((T.M, N), dtype=torch.float16, device=X.device)
+    Yv = _dev_u16(Y, "Y")
+    if ws is None:
+        ws = workspace(T.M, T.K, N, X.device)
+    cs = T.c_struct()
+    with torch.cuda.device(X.device):
+        _check(lib().spinfer_spmm(ctypes.byref(cs), X.data_ptr(), Yv.data_ptr(), T.M, T.K, N, ws.data_ptr(),
+                                  ws.numel(), _stream(stream)), "spinfer_spmm")
+    return Y
+
+
+def tp_rows(M: int, world: int, rank: int):
+    b, c = ctypes.c_int(), ctypes.c_int()
+    _check(lib().spinfer_tp_rows(M, world, rank, ctypes.byref(b), ctypes.byref(c)), "spinfer_tp_rows")
+    return int(b.value), int(c.value)
+
+
+def spmm_tp(T_shard: TCA, X: torch.Tensor, Y_full: torch.Tensor, M_full: int, world: int, rank: int,
+            ws: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """Row-partitioned SpMM: writes rows tp_rows(M_full, world, rank) of Y_full [M_full][N]. No communication."""
+    X = _dev_u16(X, "X")
+    K, N = X.shape
+    Yv = _dev_u16(Y_full, "Y_full")
+    if ws is None:
+        ws = workspace(max(T_shard.M, GT), K, N, X.device)
+    cs = T_shard.c_struct()
+    with torch.cuda.device(X.device):
+        _check(lib().spinfer_spmm_tp(ctypes.byref(cs), X.data_ptr(), Yv.data_ptr(), M_full, K, N, world, rank,
+                                     ws.data_ptr(), ws.numel(), _stream(stream)), "spinfer_spmm_tp")
+    return Y_full

@@ -1,0 +1,129 @@
+// abi.cu — the extern "C" boundary declared in include/spinfer.h: argument
+// validation, status codes, and dispatch to the sm_100a kernels.
+#include <cstring>
+#include "internal.cuh"
+
+namespace spinfer {
+
+int check_device() {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return SPINFER_ENODEV; }
+    int major = 0, minor = 0;
+    if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev) != cudaSuccess ||
+        cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev) != cudaSuccess) {
+        cudaGetLastError();
+        return SPINFER_ENODEV;
+    }
+    return (major == 10 && minor == 0) ? SPINFER_OK : SPINFER_ENODEV;   // built for sm_100a only
+}
+
+static bool shape_ok(int M, int K) { return M > 0 && K > 0 && M % kGT == 0 && K % kGT == 0; }
+
+int validate_tca(const spinfer_tca *T, int M, int K) {
+    if (!T || !T->gtile_offset || !T->bitmap || !T->values) return SPINFER_EINVAL;
+    if (T->M != M || T->K != K || T->gt_h != kGT || T->gt_w != kGT || !shape_ok(M, K)) return SPINFER_EINVAL;
+    if (T->n_values < 0) return SPINFER_EINVAL;
+    if (T->n_values >= (1LL << 31)) return SPINFER_EOVERFLOW;
+    if (!aligned16(T->gtile_offset) || !aligned16(T->bitmap) || !aligned16(T->values)) return SPINFER_EINVAL;
+    return SPINFER_OK;
+}
+
+}  // namespace spinfer
+
+using namespace spinfer;
+
+extern "C" {
+
+int spinfer_encode_count(const uint16_t *W, int M, int K, int32_t *gtile_offset, int64_t *n_values, int64_t *nnz,
+                         int32_t *max_gt_values, void *stream) {
+    if (!W || !gtile_offset || !n_values || !nnz || !shape_ok(M, K) || !aligned16(W)) return SPINFER_EINVAL;
+    int rc = check_device();
+    if (rc) return rc;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    void *tmp = nullptr;
+    if (cudaMallocAsync(&tmp, 64, st) != cudaSuccess) { cudaGetLastError(); return SPINFER_ECUDA; }
+    int64_t stats[8] = {0};
+    rc = SPINFER_ECUDA;
+    if (cudaMemsetAsync(tmp, 0, 64, st) == cudaSuccess) {
+        rc = launch_encode_count(W, M, K, gtile_offset, reinterpret_cast<int64_t *>(tmp), st);
+        if (rc == SPINFER_OK) {
+            if (cudaMemcpyAsync(stats, tmp, 64, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+                cudaStreamSynchronize(st) != cudaSuccess)
+                rc = SPINFER_ECUDA;
+        }
+    }
+    cudaFreeAsync(tmp, st);
+    if (rc) { cudaGetLastError(); return rc; }
+    if (stats[2] >= (1LL << 31)) return SPINFER_EOVERFLOW;
+    *nnz = stats[0];
+    *n_values = stats[2];
+    if (max_gt_values) *max_gt_values = (int32_t)stats[1];
+    return SPINFER_OK;
+}
+
+int spinfer_encode_fill(const uint16_t *W, const spinfer_tca *T, void *stream) {
+    if (!W || !aligned16(W) || !T) return SPINFER_EINVAL;
+    int rc = validate_tca(T, T->M, T->K);
+    if (rc) return rc;
+    if ((rc = check_device())) return rc;
+    return launch_encode_fill(W, T, reinterpret_cast<cudaStream_t>(stream));
+}
+
+int spinfer_decode(const spinfer_tca *T, uint16_t *W_out, void *stream) {
+    if (!T || !W_out || !aligned16(W_out)) return SPINFER_EINVAL;
+    int rc = validate_tca(T, T->M, T->K);
+    if (rc) return rc;
+    if ((rc = check_device())) return rc;
+    return launch_decode(T, W_out, reinterpret_cast<cudaStream_t>(stream));
+}
+
+size_t spinfer_spmm_workspace_bytes(int M, int K, int N) {
+    if (!shape_ok(M, K) || (N != 8 && N != 16 && N != 24 && N != 32)) return 0;
+    return spmm_workspace_bytes(M, K, N);
+}
+
+int spinfer_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *workspace,
+                 size_t ws_bytes, void *stream) {
+    if (!X || !Y || (N != 8 && N != 16 && N != 24 && N != 32)) return SPINFER_EINVAL;
+    if (!aligned16(X) || !aligned16(Y) || (workspace && !aligned16(workspace))) return SPINFER_EINVAL;
+    int rc = validate_tca(T, M, K);
+    if (rc) return rc;
+    if ((rc = check_device())) return rc;
+    return launch_spmm(T, X, Y, M, K, N, workspace, ws_bytes, reinterpret_cast<cudaStream_t>(stream));
+}
+
+int spinfer_tp_rows(int M, int world, int rank, int *row_begin, int *row_count) {
+    if (!row_begin || !row_count || M <= 0 || M % kGT || world <= 0 || rank < 0 || rank >= world)
+        return SPINFER_EINVAL;
+    const int MG = M / kGT, q = MG / world, rem = MG % world;
+    *row_begin = (rank * q + (rank < rem ? rank : rem)) * kGT;
+    *row_count = (q + (rank < rem ? 1 : 0)) * kGT;
+    return SPINFER_OK;
+}
+
+int spinfer_spmm_tp(const spinfer_tca *T_shard, const uint16_t *X, uint16_t *Y_full, int M_full, int K, int N,
+                    int world, int rank, void *workspace, size_t ws_bytes, void *stream) {
+    int b = 0, c = 0;
+    int rc = spinfer_tp_rows(M_full, world, rank, &b, &c);
+    if (rc) return rc;
+    if (!T_shard || !Y_full) return SPINFER_EINVAL;
+    if (T_shard->M != c) return SPINFER_EINVAL;
+    if (c == 0) return SPINFER_OK;   // rank owns no rows (more ranks than GT rows)
+    return spinfer_spmm(T_shard, X, Y_full + (size_t)b * N, c, K, N, workspace, ws_bytes, stream);
+}
+
+const char *spinfer_status_str(int status) {
+    switch (status) {
+        case SPINFER_OK: return "SPINFER_OK";
+        case SPINFER_EINVAL: return "SPINFER_EINVAL: invalid argument";
+        case SPINFER_ENOSPC: return "SPINFER_ENOSPC: workspace too small";
+        case SPINFER_EOVERFLOW: return "SPINFER_EOVERFLOW: n_values >= 2^31";
+        case SPINFER_ECUDA: return "SPINFER_ECUDA: CUDA error";
+        case SPINFER_ENODEV: return "SPINFER_ENODEV: device is not sm_100";
+        default: return "SPINFER: unknown status";
+    }
+}
+
+const char *spinfer_version(void) { return "spinfer-b200 0.1 (sm_100a; TCA-BME GT=64; mma.sync SMBD)"; }
+
+}  // extern "C"

@@ -1,0 +1,27 @@
+// internal.cuh — declarations shared by the library's translation units.
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+#include "spinfer.h"
+
+namespace spinfer {
+
+constexpr int kGT = 64;    // GroupTile edge (reading A1)
+constexpr int kNumSMsDefault = 148;
+
+int check_device();        // SPINFER_OK or SPINFER_ENODEV / SPINFER_ECUDA
+inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+int validate_tca(const spinfer_tca *T, int M, int K);
+
+// encode.cu
+int launch_encode_count(const uint16_t *W, int M, int K, int32_t *gtile_offset, int64_t *stats_dev,
+                        cudaStream_t st);
+int launch_encode_fill(const uint16_t *W, const spinfer_tca *T, cudaStream_t st);
+int launch_decode(const spinfer_tca *T, uint16_t *W_out, cudaStream_t st);
+
+// spmm.cu
+size_t spmm_workspace_bytes(int M, int K, int N);
+int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *ws,
+                size_t ws_bytes, cudaStream_t st);
+
+}  // namespace spinfer

@@ -1,0 +1,477 @@
+// spmm.cu — TCA-BME SpMM Y = W x X for sm_100a (§4.3).
+//
+// One persistent kernel, one CTA per SM. Work = "units": a unit is the column
+// of R = 2 GroupTiles (one per GT row of a 128-row "rowblock") at GT column gc,
+// linearised u = rb * KG + gc. CTA p owns units [floor(pU/P), floor((p+1)U/P))
+// (stream-K: perfect balance in GroupTiles, each CTA reads one contiguous byte
+// range per GT row). This replaces the paper's split-K grid mapping (Alg. 1
+// lines 1-3); rowblocks split across CTAs are combined by an
+// in-kernel "last arriver sums" fix-up (the paper's ReductionWorkspace).
+//
+// Warp roles (10 warps):
+//   warp 0    producer: one lane issues cp.async.bulk (TMA 1-D) copies of the
+//             stage's bitmaps, values and X slab into an S-stage smem ring,
+//             signalled on a full mbarrier with the byte count (replaces the
+//             paper's LDGSTS.128 double buffer).
+//   warp 1    scan: for each staged GroupTile computes every BitmapTile's base
+//             (PopCount prefix over earlier BTs) and writes a table of
+//             {bitmap half-word, smem address of that half's first value}.
+//   warps 2-9 consumers (GT row r = w/4, TCTile column c = w%4): SMBD decode
+//             (MaskedPopCount, Alg. 2, two-phase a0/a1 P:287) into
+//             mma.m16n8k16 A fragments, X via ldmatrix.trans, mma.sync with
+//             fp32 accumulators (Listing 1).
+#include <cstdio>
+#include <algorithm>
+#include "internal.cuh"
+#include "ptx.cuh"
+
+namespace spinfer {
+namespace {
+
+constexpr int kR = 2;               // GT rows per rowblock (128 output rows)
+constexpr int kCW = 8;              // consumer warps = kR rows x 4 TCTile columns
+constexpr int kThreads = 32 * (2 + kCW);
+constexpr int kTblSlots = 2;
+constexpr int kMaxStages = 8;
+
+struct Params {
+    const int32_t *off;
+    const uint64_t *bm;
+    const uint16_t *vals;
+    const uint16_t *X;
+    uint16_t *Y;
+    float *ws_part;
+    int32_t *ws_cnt;
+    int KG, MG;
+    long long U;
+    int P;
+    int G, S;
+    uint32_t stage_bytes, st_x, st_v0, st_v1;   // stage slot size; offsets in a slot (bitmaps at 0)
+    uint32_t tbl_bytes;
+    uint32_t o_pre, o_tbl, o_scr, o_stage;      // region offsets from the smem base
+};
+
+__device__ __forceinline__ long long unit_start(long long p, long long U, int P) { return p * U / P; }
+__device__ __forceinline__ int unit_owner(long long u, long long U, int P) {
+    return (int)(((u + 1) * (long long)P - 1) / U);
+}
+
+// SMBD for one BitmapTile and this lane. `e` = table entry
+// {bitmap half-word w, smem byte address of that half's first value}. With
+// sh = 2*(lane%16) and lm = (1<<sh)-1:
+//   count = PopCount(w & lm)                       (MaskedPopCount, Alg. 2)
+//   t0 = V[count], t1 = V[count+1]                 (zero-extended u16 loads)
+//   a0 = bit(sh)   ? t0 : 0
+//   a1 = bit(sh+1) ? (bit(sh) ? t1 : t0) : 0       (Phase II reuses count)
+// The four cases are one PRMT whose selector is looked up (by a second PRMT)
+// from y = (w >> sh) & 3; the zero bytes come from the u16 loads' upper bytes.
+__device__ __forceinline__ uint32_t smbd(uint32_t entry, uint32_t lm, uint32_t sh) {
+    uint2 e = lds_v2(entry);
+    uint32_t cnt = __popc(e.x & lm);
+    uint32_t a = e.y + 2u * cnt;
+    uint32_t t0 = lds_u16(a), t1 = lds_u16(a + 2u);
+    uint32_t y = (e.x >> sh) & 3u;
+    uint32_t sel = prmt(0x10321032u, 0x54103232u, y * 0x11u + 0x40u);
+    return prmt(t0, t1, sel);
+}
+
+template <int NT>
+__device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const float (&acc)[4][NT][4], int lane) {
+#pragma unroll
+    for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt) {
+            int r0 = row_base + tr * 16 + (lane >> 2);
+            int col = nt * 8 + 2 * (lane & 3);
+            __half2 lo = __floats2half2_rn(acc[tr][nt][0], acc[tr][nt][1]);   // one RNE per output (A11)
+            __half2 hi = __floats2half2_rn(acc[tr][nt][2], acc[tr][nt][3]);
+            *reinterpret_cast<__half2 *>(Y + (size_t)r0 * N + col) = lo;
+            *reinterpret_cast<__half2 *>(Y + (size_t)(r0 + 8) * N + col) = hi;
+        }
+}
+
+template <int NT>
+__global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
+    constexpr int N = NT * 8;
+    extern __shared__ __align__(128) uint8_t smem[];
+    const uint32_t sbase = smem_u32(smem);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int p = blockIdx.x;
+    const long long U = prm.U;
+    const int KG = prm.KG, G = prm.G, S = prm.S;
+    const long long u0 = unit_start(p, U, prm.P), u1 = unit_start(p + 1, U, prm.P);
+
+    // barriers: full[S], empty[S], scanned[2], tbl_empty[2]
+    const uint32_t bar_full = sbase, bar_empty = sbase + 8 * kMaxStages;
+    const uint32_t bar_scan = sbase + 16 * kMaxStages, bar_tble = bar_scan + 8 * kTblSlots;
+    int4 *pre = reinterpret_cast<int4 *>(smem + prm.o_pre);
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(bar_full + 8 * s, 1);
+            mbar_init(bar_empty + 8 * s, kCW);
+        }
+        for (int t = 0; t < kTblSlots; ++t) {
+            mbar_init(bar_scan + 8 * t, 32);
+            mbar_init(bar_tble + 8 * t, kCW);
+        }
+        fence_barrier_init();
+    }
+    // Preload this CTA's GTileOffset entries: pre[u-u0] = {start_r0, end_r0, start_r1, end_r1}.
+    for (long long i = threadIdx.x; i < u1 - u0; i += kThreads) {
+        long long u = u0 + i;
+        int rb = (int)(u / KG), gc = (int)(u % KG);
+        int4 v = make_int4(0, 0, 0, 0);
+        long long g0 = (long long)(kR * rb) * KG + gc;
+        v.x = __ldg(prm.off + g0);
+        v.y = __ldg(prm.off + g0 + 1);
+        if (kR * rb + 1 < prm.MG) {
+            v.z = __ldg(prm.off + g0 + KG);
+            v.w = __ldg(prm.off + g0 + KG + 1);
+        }
+        pre[i] = v;
+    }
+    __syncthreads();
+
+    if (warp == 0) {
+        // ------------------------------------------------------------ producer
+        if (lane != 0) return;
+        const uint64_t pol_w = policy_evict_first(), pol_x = policy_evict_last();
+        int i = 0;
+        for (long long u = u0; u < u1; ++i) {
+            int rb = (int)(u / KG), gc = (int)(u % KG);
+            int g = (int)min((long long)min(G, KG - gc), u1 - u);
+            int rows = min(kR, prm.MG - kR * rb);
+            int slot = i % S;
+            if (i >= S) mbar_wait(bar_empty + 8 * slot, ((i / S) - 1) & 1);
+            const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
+            const int4 ps = pre[u - u0], pe = pre[u - u0 + g - 1];
+            uint32_t vb0 = 2u * (uint32_t)(pe.y - ps.x);
+            uint32_t vb1 = rows > 1 ? 2u * (uint32_t)(pe.w - ps.z) : 0u;
+            uint32_t xb = (uint32_t)g * 64u * N * 2u;
+            uint32_t total = (uint32_t)rows * g * 512u + vb0 + vb1 + xb;
+            const uint32_t fb = bar_full + 8 * slot;
+            mbar_arrive_expect_tx(fb, total);
+            for (int r = 0; r < rows; ++r) {
+                long long gA = (long long)(kR * rb + r) * KG + gc;
+                bulk_g2s(st + (uint32_t)(r * G) * 512u, prm.bm + gA * 64, (uint32_t)g * 512u, fb, pol_w);
+            }
+            if (vb0) bulk_g2s(st + prm.st_v0, prm.vals + ps.x, vb0, fb, pol_w);
+            if (vb1) bulk_g2s(st + prm.st_v1, prm.vals + ps.z, vb1, fb, pol_w);
+            bulk_g2s(st + prm.st_x, prm.X + (size_t)gc * 64 * N, xb, fb, pol_x);
+            u += g;
+        }
+        return;
+    }
+
+    if (warp == 1) {
+        // ------------------------------------------------------------ scan
+        int i = 0;
+        for (long long u = u0; u < u1; ++i) {
+            int rb = (int)(u / KG), gc = (int)(u % KG);
+            int g = (int)min((long long)min(G, KG - gc), u1 - u);
+            int rows = min(kR, prm.MG - kR * rb);
+            int slot = i % S, t = i & 1;
+            mbar_wait(bar_full + 8 * slot, (i / S) & 1);
+            if (i >= kTblSlots) mbar_wait(bar_tble + 8 * t, ((i / kTblSlots) - 1) & 1);
+            const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
+            const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes;
+            for (int r = 0; r < rows; ++r) {
+                const int base_r = r ? pre[u - u0].z : pre[u - u0].x;
+                const uint32_t vsm = st + (r ? prm.st_v1 : prm.st_v0);
+                for (int j = 0; j < g; ++j) {
+                    const int4 pj = pre[u - u0 + j];
+                    const int rel = (r ? pj.z : pj.x) - base_r;          // GT j's values in the chunk
+                    const uint32_t bmsm = st + (uint32_t)(r * G + j) * 512u;
+                    // lane handles BTs `lane` and `lane + 32` of the GT (storage order)
+                    uint2 ba = lds_v2(bmsm + 8u * lane);
+                    uint2 bb = lds_v2(bmsm + 256u + 8u * lane);
+                    uint32_t pal = __popc(ba.x), pah = __popc(ba.y);
+                    uint32_t pbl = __popc(bb.x), pbh = __popc(bb.y);
+                    uint32_t packed = (pal + pah) | ((pbl + pbh) << 16);
+                    uint32_t incl = packed;
+#pragma unroll
+                    for (int o = 1; o < 32; o <<= 1) {
+                        uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                        if (lane >= o) incl += y;
+                    }
+                    uint32_t tot_a = __shfl_sync(0xffffffffu, incl, 31) & 0xFFFFu;
+                    uint32_t excl = incl - packed;
+                    uint32_t ea = excl & 0xFFFFu, eb = tot_a + (excl >> 16);   // PopCount prefix
+                    uint32_t Aa = vsm + 2u * (uint32_t)(rel + (int)ea);
+                    uint32_t Ab = vsm + 2u * (uint32_t)(rel + (int)eb);
+                    const uint32_t te = tb + (uint32_t)((r * G + j) * 64) * 16u;
+                    sts_v4(te + 16u * lane, make_uint4(ba.x, Aa, ba.y, Aa + 2u * pal));
+                    sts_v4(te + 16u * (lane + 32), make_uint4(bb.x, Ab, bb.y, Ab + 2u * pbl));
+                }
+            }
+            mbar_arrive(bar_scan + 8 * t);
+            u += g;
+        }
+        return;
+    }
+
+    // ---------------------------------------------------------------- consumers
+    const int cw = warp - 2, r = cw >> 2, c = cw & 3;
+    const uint32_t sh = 2u * (lane & 15);
+    const uint32_t lm = (1u << sh) - 1u;
+    const uint32_t hioff = (uint32_t)(lane >> 4) * 8u;
+    // ldmatrix.trans row addresses: matrix m = lane/8 -> (k half m&1, n half m>>1)
+    const uint32_t xlane = (uint32_t)((((lane >> 3) & 1) * 8 + (lane & 7)) * N + ((lane >> 4) & 1) * 8) * 2u;
+    float acc[4][NT][4];
+    const uint32_t scr = sbase + prm.o_scr + (uint32_t)r * (2u * 64u * N * 4u);
+
+    int i = 0;
+    long long seg_u0 = u0;
+    for (long long u = u0; u < u1; ++i) {
+        const int rb = (int)(u / KG), gc = (int)(u % KG);
+        const int g = (int)min((long long)min(G, KG - gc), u1 - u);
+        const int rows = min(kR, prm.MG - kR * rb);
+        const int slot = i % S, t = i & 1;
+        if (gc == 0 || u == u0) {
+            seg_u0 = u;
+#pragma unroll
+            for (int a = 0; a < 4; ++a)
+#pragma unroll
+                for (int b = 0; b < NT; ++b)
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) acc[a][b][q] = 0.f;
+        }
+        mbar_wait(bar_full + 8 * slot, (i / S) & 1);
+        mbar_wait(bar_scan + 8 * t, (i / kTblSlots) & 1);
+        if (r < rows) {
+            const uint32_t xs = sbase + prm.o_stage + slot * prm.stage_bytes + prm.st_x + xlane;
+            const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes + (uint32_t)(r * G * 64 + c * 16) * 16u + hioff;
+            for (int j = 0; j < g; ++j) {
+                uint32_t bfr[NT][2];
+                const uint32_t xk = xs + (uint32_t)(64 * j + 16 * c) * N * 2u;
+                if constexpr (NT == 1) {
+                    ldsm_x2_trans(xk, bfr[0][0], bfr[0][1]);
+                } else {
+#pragma unroll
+                    for (int nt = 0; nt + 1 < NT; nt += 2)
+                        ldsm_x4_trans(xk + nt * 16u, bfr[nt][0], bfr[nt][1], bfr[nt + 1][0], bfr[nt + 1][1]);
+                    if constexpr (NT % 2 == 1) ldsm_x2_trans(xk + (NT - 1) * 16u, bfr[NT - 1][0], bfr[NT - 1][1]);
+                }
+                const uint32_t tj = tb + (uint32_t)j * 64u * 16u;
+#pragma unroll
+                for (int tr = 0; tr < 4; ++tr) {
+                    uint32_t a[4];
+#pragma unroll
+                    for (int b = 0; b < 4; ++b) a[b] = smbd(tj + (uint32_t)(tr * 4 + b) * 16u, lm, sh);
+#pragma unroll
+                    for (int nt = 0; nt < NT; ++nt) mma_16816(acc[tr][nt], a, bfr[nt][0], bfr[nt][1]);
+                }
+            }
+        }
+        __syncwarp();
+        if (lane == 0) {
+            mbar_arrive(bar_empty + 8 * slot);
+            mbar_arrive(bar_tble + 8 * t);
+        }
+        u += g;
+        const bool seg_end = (gc + g == KG) || (u == u1);
+        if (seg_end && r < rows) {
+            // -------------------------------------------------------- epilogue
+            // (1) reduce the 4 TCTile-column partials of GT row r (tree via smem)
+            const uint32_t bid = 1u + (uint32_t)r;
+            if (c >= 2) {
+#pragma unroll
+                for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                    for (int nt = 0; nt < NT; ++nt)
+                        sts_f4(scr + (uint32_t)(c - 2) * (64u * N * 4u) + (uint32_t)((tr * NT + nt) * 32 + lane) * 16u,
+                               make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]));
+            }
+            named_bar_sync(bid, 128);
+            if (c < 2) {
+#pragma unroll
+                for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                    for (int nt = 0; nt < NT; ++nt) {
+                        float4 v = lds_f4(scr + (uint32_t)c * (64u * N * 4u) + (uint32_t)((tr * NT + nt) * 32 + lane) * 16u);
+                        acc[tr][nt][0] += v.x; acc[tr][nt][1] += v.y; acc[tr][nt][2] += v.z; acc[tr][nt][3] += v.w;
+                    }
+            }
+            named_bar_sync(bid, 128);
+            if (c == 1) {
+#pragma unroll
+                for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                    for (int nt = 0; nt < NT; ++nt)
+                        sts_f4(scr + (uint32_t)((tr * NT + nt) * 32 + lane) * 16u,
+                               make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]));
+            }
+            named_bar_sync(bid, 128);
+            if (c == 0) {
+#pragma unroll
+                for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                    for (int nt = 0; nt < NT; ++nt) {
+                        float4 v = lds_f4(scr + (uint32_t)((tr * NT + nt) * 32 + lane) * 16u);
+                        acc[tr][nt][0] += v.x; acc[tr][nt][1] += v.y; acc[tr][nt][2] += v.z; acc[tr][nt][3] += v.w;
+                    }
+            }
+            named_bar_sync(bid, 128);
+            // (2) write Y, or combine split rowblocks across CTAs (split-K fix-up)
+            if (c == 0) {
+                const int grow = kR * rb + r;
+                const int row_base = grow * 64;
+                const bool complete = (seg_u0 == (long long)rb * KG) && (u == (long long)(rb + 1) * KG);
+                if (complete) {
+                    store_y<NT>(prm.Y, N, row_base, acc, lane);
+                } else {
+                    const int pf = unit_owner((long long)rb * KG, U, prm.P);
+                    const int pl = unit_owner((long long)(rb + 1) * KG - 1, U, prm.P);
+                    const int myslot = (rb == (int)(u0 / KG)) ? 0 : 1;
+                    float4 *part = reinterpret_cast<float4 *>(prm.ws_part) + (((size_t)p * 2 + myslot) * kR + r) * (64 * N / 4);
+#pragma unroll
+                    for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                        for (int nt = 0; nt < NT; ++nt)
+                            part[(tr * NT + nt) * 32 + lane] =
+                                make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]);
+                    __threadfence();
+                    __syncwarp();
+                    int old = 0;
+                    if (lane == 0) old = atomicAdd(prm.ws_cnt + grow, 1);
+                    old = __shfl_sync(0xffffffffu, old, 0);
+                    if (old == pl - pf) {   // last contributor: sum all partials in CTA order
+                        __threadfence();
+#pragma unroll
+                        for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+                                for (int q = 0; q < 4; ++q) acc[tr][nt][q] = 0.f;
+                        for (int q = pf; q <= pl; ++q) {
+                            const int sl = (rb == (int)(unit_start(q, U, prm.P) / KG)) ? 0 : 1;
+                            const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part) + (((size_t)q * 2 + sl) * kR + r) * (64 * N / 4);
+#pragma unroll
+                            for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                                for (int nt = 0; nt < NT; ++nt) {
+                                    float4 v = ldg_cg_f4(pp + (tr * NT + nt) * 32 + lane);
+                                    acc[tr][nt][0] += v.x; acc[tr][nt][1] += v.y; acc[tr][nt][2] += v.z; acc[tr][nt][3] += v.w;
+                                }
+                        }
+                        store_y<NT>(prm.Y, N, row_base, acc, lane);
+                        if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed
+                    }
+                }
+            }
+        }
+    }
+}
+
+struct Plan {
+    int P, G, S;
+    long long U;
+    size_t smem;
+    Params prm;
+};
+
+int num_sms() {
+    int dev = 0, n = kNumSMsDefault;
+    if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    return n > 0 ? n : kNumSMsDefault;
+}
+
+int choose_P(long long U) {
+    long long P = min((long long)num_sms(), U);
+    // keep the preloaded offsets (16 B per unit) within 16 KiB of shared memory
+    while ((U + P - 1) / P > 1024) P += num_sms();
+    return (int)max(1LL, P);
+}
+
+inline uint32_t align_up(uint32_t x, uint32_t a) { return (x + a - 1) / a * a; }
+
+bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
+    const int MG = M / kGT, KG = K / kGT;
+    const int nRB = (MG + kR - 1) / kR;
+    pl->U = (long long)nRB * KG;
+    pl->P = choose_P(pl->U);
+    const long long upc = (pl->U + pl->P - 1) / pl->P;
+    int dev = 0, smem_max = 232448;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    int maxv = max_gt_values > 0 ? max_gt_values : 4096;
+    maxv = min(4096, (maxv + 7) & ~7);
+    const uint32_t o_pre = 256;
+    const uint32_t pre_bytes = align_up((uint32_t)(16 * upc), 128);
+    for (int G = 4; G >= 1; --G) {
+        uint32_t tbl = (uint32_t)kR * G * 64 * 16;
+        uint32_t scr = (uint32_t)kR * 2 * 64 * N * 4;
+        uint32_t st_x = (uint32_t)kR * G * 512;
+        uint32_t st_v0 = st_x + (uint32_t)G * 64 * N * 2;
+        uint32_t vcap = align_up((uint32_t)G * maxv * 2, 16);
+        uint32_t st_v1 = st_v0 + vcap;
+        uint32_t stage = align_up(st_v1 + vcap, 128);
+        uint32_t fixed = o_pre + pre_bytes + kTblSlots * tbl + scr + 128;   // +slack for the t1 over-read
+        if ((long long)fixed + 2LL * stage > smem_max) continue;
+        int S = (int)std::min<long long>(kMaxStages, ((long long)smem_max - fixed) / stage);
+        if (S < 3 && G > 1) continue;
+        pl->G = G;
+        pl->S = S;
+        Params &q = pl->prm;
+        q.KG = KG; q.MG = MG; q.U = pl->U; q.P = pl->P; q.G = G; q.S = S;
+        q.stage_bytes = stage; q.st_x = st_x; q.st_v0 = st_v0; q.st_v1 = st_v1;
+        q.tbl_bytes = tbl;
+        q.o_pre = o_pre;
+        q.o_tbl = o_pre + pre_bytes;
+        q.o_scr = q.o_tbl + kTblSlots * tbl;
+        q.o_stage = q.o_scr + scr;
+        pl->smem = (size_t)q.o_stage + (size_t)S * stage + 128;
+        return true;
+    }
+    return false;
+}
+
+template <int NT>
+int launch_nt(const Plan &pl, cudaStream_t st) {
+    static int configured_smem = 0;   // per-instantiation max dynamic smem already set
+    if ((int)pl.smem > configured_smem) {
+        if (cudaFuncSetAttribute(k_spmm<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem) != cudaSuccess)
+            return SPINFER_ECUDA;
+        configured_smem = (int)pl.smem;
+    }
+    k_spmm<NT><<<pl.P, kThreads, pl.smem, st>>>(pl.prm);
+    return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
+}
+
+}  // namespace
+
+size_t spmm_workspace_bytes(int M, int K, int N) {
+    if (M <= 0 || K <= 0 || M % kGT || K % kGT || N <= 0 || N > 32) return 0;
+    const int MG = M / kGT, KG = K / kGT;
+    const long long U = (long long)((MG + kR - 1) / kR) * KG;
+    const int P = choose_P(U);
+    size_t cnt = ((size_t)MG * 4 + 255) / 256 * 256;
+    size_t part = (size_t)P * 2 * kR * 64 * N * 4;
+    return cnt + part;
+}
+
+int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *ws, size_t ws_bytes,
+                cudaStream_t st) {
+    Plan pl;
+    if (!make_plan(M, K, N, T->max_gt_values, &pl)) return SPINFER_EINVAL;
+    const size_t need = spmm_workspace_bytes(M, K, N);
+    if (ws_bytes < need || ws == nullptr) return SPINFER_ENOSPC;
+    Params &q = pl.prm;
+    q.off = T->gtile_offset;
+    q.bm = T->bitmap;
+    q.vals = T->values;
+    q.X = X;
+    q.Y = Y;
+    q.ws_cnt = reinterpret_cast<int32_t *>(ws);
+    q.ws_part = reinterpret_cast<float *>(reinterpret_cast<uint8_t *>(ws) + ((size_t)(M / kGT) * 4 + 255) / 256 * 256);
+    switch (N) {
+        case 8: return launch_nt<1>(pl, st);
+        case 16: return launch_nt<2>(pl, st);
+        case 24: return launch_nt<3>(pl, st);
+        case 32: return launch_nt<4>(pl, st);
+        default: return SPINFER_EINVAL;
+    }
+}
+
+}  // namespace spinfer

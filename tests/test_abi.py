@@ -1,0 +1,73 @@
+"""The C-ABI library loads and exports every symbol include/spinfer.h declares
+(-m "not gpu": no compute calls), plus host-only logic (tp_rows, status strings)."""
+import os
+import re
+import subprocess
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _header_functions():
+    src = open(os.path.join(ROOT, "include", "spinfer.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(spinfer_[a-z_]+)\s*\(", src)))
+
+
+@pytest.fixture(scope="module")
+def sp():
+    from paper_conf_eurosys_fanydlgww025_b200 import build
+    build.build()
+    import paper_conf_eurosys_fanydlgww025_b200 as sp
+    return sp
+
+
+def test_header_symbols_exported(sp):
+    names = _header_functions()
+    assert set(names) == set(sp.SYMBOLS), names
+    out = subprocess.run(["nm", "-D", "--defined-only", sp.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT (spinfer_\w+)", out))
+    assert set(names) <= exported
+    # nothing else leaks from the library (hidden visibility)
+    assert exported == set(names), exported - set(names)
+    L = sp.lib()
+    for n in names:
+        assert getattr(L, n) is not None
+
+
+def test_built_for_sm100a(sp):
+    out = subprocess.run(["cuobjdump", "--list-elf", sp.LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    sass = subprocess.run(["cuobjdump", "-sass", sp.LIB_PATH], capture_output=True, text=True).stdout
+    assert "HMMA.16816.F32" in sass          # tensor-core mma in the SpMM kernel
+    assert "UBLKCP" in sass                  # cp.async.bulk (TMA) staging
+    assert "SYNCS" in sass                   # mbarrier pipeline
+
+
+def test_status_strings_and_version(sp):
+    L = sp.lib()
+    assert L.spinfer_status_str(0) == b"SPINFER_OK"
+    assert b"EINVAL" in L.spinfer_status_str(-1)
+    assert b"ENOSPC" in L.spinfer_status_str(-2)
+    assert b"sm_100a" in L.spinfer_version()
+
+
+def test_tp_rows_host_logic(sp):
+    import oracle
+    for M in (64, 1152, 9216, 28672, 36864):
+        for world in (1, 2, 4, 8):
+            for r in range(world):
+                assert sp.tp_rows(M, world, r) == oracle.tp_rows(M, world, r)
+    with pytest.raises(sp.SpinferError):
+        sp.tp_rows(100, 2, 0)
+    with pytest.raises(sp.SpinferError):
+        sp.tp_rows(128, 2, 2)
+
+
+def test_no_cpu_fallback_without_device(sp):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("has a GPU")
+    with pytest.raises((ValueError, RuntimeError)):
+        sp.encode(torch.zeros((64, 64), dtype=torch.float16))
