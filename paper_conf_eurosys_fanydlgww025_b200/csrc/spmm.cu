@@ -21,6 +21,7 @@
 //             mma.m16n8k16 A fragments, X via ldmatrix.trans, mma.sync with
 //             fp32 accumulators (Listing 1).
 #include <cstdio>
+#include <cstdlib>
 #include <algorithm>
 #include "internal.cuh"
 #include "ptx.cuh"
@@ -378,7 +379,10 @@ int num_sms() {
 }
 
 int choose_P(long long U) {
-    long long P = min((long long)num_sms(), U);
+    long long cap = num_sms();
+    // SPINFER_MAX_CTAS caps the persistent grid (tests use it to force many stages per CTA)
+    if (const char *e = getenv("SPINFER_MAX_CTAS")) { long long v = atoll(e); if (v > 0 && v < cap) cap = v; }
+    long long P = min(cap, U);
     // keep the preloaded offsets (16 B per unit) within 16 KiB of shared memory
     while ((U + P - 1) / P > 1024) P += num_sms();
     return (int)max(1LL, P);
