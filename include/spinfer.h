@@ -95,10 +95,13 @@ SPINFER_API int spinfer_encode_fill(const uint16_t *W, const spinfer_tca *T, voi
 /* Decode TCA-BME -> dense fp16 W_out [M][K] (device); unset bits give +0.0. */
 SPINFER_API int spinfer_decode(const spinfer_tca *T, uint16_t *W_out, void *stream);
 
-/* Bytes of device workspace spinfer_spmm needs for this shape (split-K partials
- * and fix-up counters). The workspace must be ZERO-FILLED before its first use;
- * every spinfer_spmm call leaves the counter region zero again, so one zeroed
- * workspace can be reused by successive calls on ONE stream (not concurrently). */
+/* Bytes of device workspace spinfer_spmm needs for this shape: a fixed 64 KiB
+ * region of split-K fix-up counters (one int32 per GT row; M <= 1,048,576)
+ * followed by fp32 split-K partials. 0 for an invalid shape. The workspace must
+ * be ZERO-FILLED before its first use; every spinfer_spmm call leaves the
+ * counter region zero again, so one zeroed workspace (sized for the largest
+ * shape) can be reused by successive calls of any shape on ONE stream — never
+ * by two calls that may run concurrently. */
 SPINFER_API size_t spinfer_spmm_workspace_bytes(int M, int K, int N);
 
 /* Y = W x X with fp32 accumulation and one round-to-nearest-even to

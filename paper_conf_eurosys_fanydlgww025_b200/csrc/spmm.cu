@@ -34,6 +34,12 @@ constexpr int kCW = 8;              // consumer warps = kR rows x 4 TCTile colum
 constexpr int kThreads = 32 * (2 + kCW);
 constexpr int kTblSlots = 2;
 constexpr int kMaxStages = 8;
+constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector table constant
+// Workspace = [fix-up counters: one int32 per GT row, fixed-size region][split-K partials].
+// The counter region has the same size for every shape so that one zeroed
+// workspace can serve calls of different shapes (partials never overlap counters).
+constexpr int kMaxCounters = 16384;                 // M <= 1,048,576 rows
+constexpr size_t kCounterBytes = (size_t)kMaxCounters * 4;
 
 struct Params {
     const int32_t *off;
@@ -57,24 +63,23 @@ __device__ __forceinline__ int unit_owner(long long u, long long U, int P) {
     return (int)(((u + 1) * (long long)P - 1) / U);
 }
 
-// SMBD for one BitmapTile and this lane. `e` = table entry
-// {bitmap half-word w, smem byte address of that half's first value}. With
-// sh = 2*(lane%16) and lm = (1<<sh)-1:
+// SMBD for one BitmapTile and one lane, split into phases so
+// a warp keeps many shared-memory loads in flight. The scan warp's table entry
+// for (BT, lane-half h) is {w, A}: w = bitmap word h (bits 32h..32h+31), A = smem
+// byte address of the first value of that half. With sh = 2*(lane%16), lm = (1<<sh)-1:
 //   count = PopCount(w & lm)                       (MaskedPopCount, Alg. 2)
 //   t0 = V[count], t1 = V[count+1]                 (zero-extended u16 loads)
-//   a0 = bit(sh)   ? t0 : 0
+//   a0 = bit(sh)   ? t0 : 0                        (Phase I)
 //   a1 = bit(sh+1) ? (bit(sh) ? t1 : t0) : 0       (Phase II reuses count)
-// The four cases are one PRMT whose selector is looked up (by a second PRMT)
-// from y = (w >> sh) & 3; the zero bytes come from the u16 loads' upper bytes.
-__device__ __forceinline__ uint32_t smbd(uint32_t entry, uint32_t lm, uint32_t sh) {
-    uint2 e = lds_v2(entry);
-    uint32_t cnt = __popc(e.x & lm);
-    uint32_t a = e.y + 2u * cnt;
-    uint32_t t0 = lds_u16(a), t1 = lds_u16(a + 2u);
-    uint32_t y = (e.x >> sh) & 3u;
-    uint32_t sel = prmt(0x10321032u, 0x54103232u, y * 0x11u + 0x40u);
-    return prmt(t0, t1, sel);
-}
+// The four (bit(sh), bit(sh+1)) cases are one PRMT of {t0, t1} whose selector is
+// looked up by a second PRMT from y = (w >> sh) & 3; zero halves select the u16
+// loads' zero upper bytes. Selector table (nibbles = source bytes, low half first):
+//   y=0 -> 0x3232 (0,0)   y=1 -> 0x3210 (t0,0)   y=2 -> 0x1032 (0,t0)   y=3 -> 0x5410 (t0,t1)
+// low selector byte  = byte y of 0x10321032, high byte = byte y of 0x54103232,
+// so sel = prmt(0x10321032, 0x54103232, y*0x11 + 0x40).
+struct SmbdConst {
+    uint32_t lm, sh, ca, c40;
+};
 
 template <int NT>
 __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const float (&acc)[4][NT][4], int lane) {
@@ -117,6 +122,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             mbar_init(bar_tble + 8 * t, kCW);
         }
         fence_barrier_init();
+        // SMBD selector-table word, read back into a register by every consumer thread so
+        // ptxas keeps it live in a register instead of re-materialising it per PRMT.
+        reinterpret_cast<uint32_t *>(smem)[kConstWord] = 0x10321032u;
+        reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = 0x40u;
     }
     // Preload this CTA's GTileOffset entries: pre[u-u0] = {start_r0, end_r0, start_r1, end_r1}.
     for (long long i = threadIdx.x; i < u1 - u0; i += kThreads) {
@@ -167,6 +176,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
 
     if (warp == 1) {
         // ------------------------------------------------------------ scan
+        // Table per staged GT (r, j), 1024 B: [lane-half h][BT in GT storage order] {w, A},
+        // so a consumer lane fetches the entries of 2 consecutive BTs with one 16-B load.
         int i = 0;
         for (long long u = u0; u < u1; ++i) {
             int rb = (int)(u / KG), gc = (int)(u % KG);
@@ -201,9 +212,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
                     uint32_t ea = excl & 0xFFFFu, eb = tot_a + (excl >> 16);   // PopCount prefix
                     uint32_t Aa = vsm + 2u * (uint32_t)(rel + (int)ea);
                     uint32_t Ab = vsm + 2u * (uint32_t)(rel + (int)eb);
-                    const uint32_t te = tb + (uint32_t)((r * G + j) * 64) * 16u;
-                    sts_v4(te + 16u * lane, make_uint4(ba.x, Aa, ba.y, Aa + 2u * pal));
-                    sts_v4(te + 16u * (lane + 32), make_uint4(bb.x, Ab, bb.y, Ab + 2u * pbl));
+                    const uint32_t te = tb + (uint32_t)(r * G + j) * 1024u + 8u * lane;
+                    sts_v2(te, ba.x, Aa);
+                    sts_v2(te + 512u, ba.y, Aa + 2u * pal);
+                    sts_v2(te + 256u, bb.x, Ab);
+                    sts_v2(te + 768u, bb.y, Ab + 2u * pbl);
                 }
             }
             mbar_arrive(bar_scan + 8 * t);
@@ -216,7 +229,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
     const int cw = warp - 2, r = cw >> 2, c = cw & 3;
     const uint32_t sh = 2u * (lane & 15);
     const uint32_t lm = (1u << sh) - 1u;
-    const uint32_t hioff = (uint32_t)(lane >> 4) * 8u;
+    const uint32_t ca = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];   // 0x10321032
+    const uint32_t c40 = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];   // 0x40
+    const uint32_t hioff = (uint32_t)(lane >> 4) * 512u;
     // ldmatrix.trans row addresses: matrix m = lane/8 -> (k half m&1, n half m>>1)
     const uint32_t xlane = (uint32_t)((((lane >> 3) & 1) * 8 + (lane & 7)) * N + ((lane >> 4) & 1) * 8) * 2u;
     float acc[4][NT][4];
@@ -242,8 +257,33 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
         mbar_wait(bar_scan + 8 * t, (i / kTblSlots) & 1);
         if (r < rows) {
             const uint32_t xs = sbase + prm.o_stage + slot * prm.stage_bytes + prm.st_x + xlane;
-            const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes + (uint32_t)(r * G * 64 + c * 16) * 16u + hioff;
+            // this warp's 16 entries of GT j (TCTiles c*4 .. c*4+3, all 4 BTs): 128 contiguous bytes
+            const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes + (uint32_t)(r * G) * 1024u + hioff +
+                                (uint32_t)c * 128u;
+            uint4 E[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) E[q] = lds_v4(tb + 16u * q);
             for (int j = 0; j < g; ++j) {
+                // phase 1: value addresses and selectors of the 16 BTs
+                uint32_t addr[16], s1[16];
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {
+                    const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
+                    const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;
+                    addr[k] = A + 2u * __popc(w & lm);
+                    s1[k] = ((w >> sh) & 3u) * 0x11u + c40;
+                }
+                // phase 2: 32 value loads in flight
+                uint32_t t0[16], t1[16];
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {
+                    t0[k] = lds_u16(addr[k]);
+                    t1[k] = lds_u16(addr[k] + 2u);
+                }
+                // phase 3: prefetch the next GT's table entries (unconditionally: past the last
+                // GT this reads other, in-bounds table/scratch bytes that are never used), X fragments
+#pragma unroll
+                for (int q = 0; q < 8; ++q) E[q] = lds_v4(tb + (uint32_t)(j + 1) * 1024u + 16u * q);
                 uint32_t bfr[NT][2];
                 const uint32_t xk = xs + (uint32_t)(64 * j + 16 * c) * N * 2u;
                 if constexpr (NT == 1) {
@@ -254,14 +294,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
                         ldsm_x4_trans(xk + nt * 16u, bfr[nt][0], bfr[nt][1], bfr[nt + 1][0], bfr[nt + 1][1]);
                     if constexpr (NT % 2 == 1) ldsm_x2_trans(xk + (NT - 1) * 16u, bfr[NT - 1][0], bfr[NT - 1][1]);
                 }
-                const uint32_t tj = tb + (uint32_t)j * 64u * 16u;
+                // phase 4: assemble the A fragments (Ra0..Ra3 = BTs TL,BL,TR,BR) and mma
 #pragma unroll
                 for (int tr = 0; tr < 4; ++tr) {
-                    uint32_t a[4];
+                    uint32_t afr[4];
 #pragma unroll
-                    for (int b = 0; b < 4; ++b) a[b] = smbd(tj + (uint32_t)(tr * 4 + b) * 16u, lm, sh);
+                    for (int b = 0; b < 4; ++b) {
+                        const int k = tr * 4 + b;
+                        afr[b] = prmt(t0[k], t1[k], prmt(ca, 0x54103232u, s1[k]));
+                    }
 #pragma unroll
-                    for (int nt = 0; nt < NT; ++nt) mma_16816(acc[tr][nt], a, bfr[nt][0], bfr[nt][1]);
+                    for (int nt = 0; nt < NT; ++nt) mma_16816(acc[tr][nt], afr, bfr[nt][0], bfr[nt][1]);
                 }
             }
         }
@@ -446,13 +489,12 @@ int launch_nt(const Plan &pl, cudaStream_t st) {
 }  // namespace
 
 size_t spmm_workspace_bytes(int M, int K, int N) {
-    if (M <= 0 || K <= 0 || M % kGT || K % kGT || N <= 0 || N > 32) return 0;
+    if (M <= 0 || K <= 0 || M % kGT || K % kGT || N <= 0 || N > 32 || M / kGT > kMaxCounters) return 0;
     const int MG = M / kGT, KG = K / kGT;
     const long long U = (long long)((MG + kR - 1) / kR) * KG;
     const int P = choose_P(U);
-    size_t cnt = ((size_t)MG * 4 + 255) / 256 * 256;
     size_t part = (size_t)P * 2 * kR * 64 * N * 4;
-    return cnt + part;
+    return kCounterBytes + part;
 }
 
 int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *ws, size_t ws_bytes,
@@ -460,6 +502,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     Plan pl;
     if (!make_plan(M, K, N, T->max_gt_values, &pl)) return SPINFER_EINVAL;
     const size_t need = spmm_workspace_bytes(M, K, N);
+    if (need == 0) return SPINFER_EINVAL;
     if (ws_bytes < need || ws == nullptr) return SPINFER_ENOSPC;
     Params &q = pl.prm;
     q.off = T->gtile_offset;
@@ -468,7 +511,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     q.X = X;
     q.Y = Y;
     q.ws_cnt = reinterpret_cast<int32_t *>(ws);
-    q.ws_part = reinterpret_cast<float *>(reinterpret_cast<uint8_t *>(ws) + ((size_t)(M / kGT) * 4 + 255) / 256 * 256);
+    q.ws_part = reinterpret_cast<float *>(reinterpret_cast<uint8_t *>(ws) + kCounterBytes);
     switch (N) {
         case 8: return launch_nt<1>(pl, st);
         case 16: return launch_nt<2>(pl, st);

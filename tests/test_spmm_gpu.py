@@ -93,7 +93,7 @@ def test_spmm_deterministic_and_workspace_reusable():
     c = f16_bits(sp.spmm(T, X1))
     assert np.array_equal(a, c) and not np.array_equal(a, b)
     ws = sp.workspace(2048, 2048, 16)
-    cnt = ws[: (2048 // 64) * 4].view(dtype=__import__("torch").int32)
+    cnt = ws[: 65536].view(dtype=__import__("torch").int32)
     assert int(cnt.abs().sum()) == 0
 
 
