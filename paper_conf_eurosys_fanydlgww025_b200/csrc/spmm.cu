@@ -34,6 +34,8 @@ constexpr int kCW = 8;              // consumer warps = kR rows x 4 TCTile colum
 constexpr int kThreads = 32 * (2 + kCW);
 constexpr int kTblSlots = 2;
 constexpr int kMaxStages = 8;
+constexpr int kMaxG = 4;
+constexpr int kTraceCTAs = 4, kTraceStages = 64;            // max GroupTile columns per stage
 constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector table constant
 // Workspace = [fix-up counters: one int32 per GT row, fixed-size region][split-K partials].
 // The counter region has the same size for every shape so that one zeroed
@@ -56,7 +58,13 @@ struct Params {
     uint32_t stage_bytes, st_x, st_v0, st_v1;   // stage slot size; offsets in a slot (bitmaps at 0)
     uint32_t tbl_bytes;
     uint32_t o_pre, o_tbl, o_scr, o_stage;      // region offsets from the smem base
+    long long *trace;   // experiments only (SPINFER_TRACE): [kTraceCTAs][kTraceStages][8] clock64 stamps
+    int dbg;   // experiments only (SPINFER_DEBUG_MODE): bit0 = consumers skip decode/MMA, bit1 = scan warp skips work
 };
+
+__device__ __forceinline__ void trace_ev(const Params &prm, int p, int i, int ev) {
+    if (prm.trace && p < kTraceCTAs && i < kTraceStages) prm.trace[((size_t)p * kTraceStages + i) * 8 + ev] = clock64();
+}
 
 __device__ __forceinline__ long long unit_start(long long p, long long U, int P) { return p * U / P; }
 __device__ __forceinline__ int unit_owner(long long u, long long U, int P) {
@@ -154,6 +162,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             int rows = min(kR, prm.MG - kR * rb);
             int slot = i % S;
             if (i >= S) mbar_wait(bar_empty + 8 * slot, ((i / S) - 1) & 1);
+            trace_ev(prm, p, i, 0);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const int4 ps = pre[u - u0], pe = pre[u - u0 + g - 1];
             uint32_t vb0 = 2u * (uint32_t)(pe.y - ps.x);
@@ -185,41 +194,67 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             int rows = min(kR, prm.MG - kR * rb);
             int slot = i % S, t = i & 1;
             mbar_wait(bar_full + 8 * slot, (i / S) & 1);
+            if (lane == 0) trace_ev(prm, p, i, 1);
             if (i >= kTblSlots) mbar_wait(bar_tble + 8 * t, ((i / kTblSlots) - 1) & 1);
+            if (lane == 0) trace_ev(prm, p, i, 2);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes;
-            for (int r = 0; r < rows; ++r) {
-                const int base_r = r ? pre[u - u0].z : pre[u - u0].x;
-                const uint32_t vsm = st + (r ? prm.st_v1 : prm.st_v0);
-                for (int j = 0; j < g; ++j) {
-                    const int4 pj = pre[u - u0 + j];
-                    const int rel = (r ? pj.z : pj.x) - base_r;          // GT j's values in the chunk
-                    const uint32_t bmsm = st + (uint32_t)(r * G + j) * 512u;
-                    // lane handles BTs `lane` and `lane + 32` of the GT (storage order)
-                    uint2 ba = lds_v2(bmsm + 8u * lane);
-                    uint2 bb = lds_v2(bmsm + 256u + 8u * lane);
-                    uint32_t pal = __popc(ba.x), pah = __popc(ba.y);
-                    uint32_t pbl = __popc(bb.x), pbh = __popc(bb.y);
-                    uint32_t packed = (pal + pah) | ((pbl + pbh) << 16);
-                    uint32_t incl = packed;
+            // all rows x g GroupTiles of the stage are scanned together: slot q = r*kMaxG + j,
+            // static bounds, unconditional full-warp shuffles (absent GTs scan zeros), so the
+            // kR*kMaxG independent shuffle chains interleave (ILP) with no divergence handling.
+            const bool work = !(prm.dbg & 2);
+            uint2 ba[kR * kMaxG], bb[kR * kMaxG];
+            uint32_t packed[kR * kMaxG], incl[kR * kMaxG];
 #pragma unroll
-                    for (int o = 1; o < 32; o <<= 1) {
-                        uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
-                        if (lane >= o) incl += y;
-                    }
-                    uint32_t tot_a = __shfl_sync(0xffffffffu, incl, 31) & 0xFFFFu;
-                    uint32_t excl = incl - packed;
-                    uint32_t ea = excl & 0xFFFFu, eb = tot_a + (excl >> 16);   // PopCount prefix
-                    uint32_t Aa = vsm + 2u * (uint32_t)(rel + (int)ea);
-                    uint32_t Ab = vsm + 2u * (uint32_t)(rel + (int)eb);
+            for (int q = 0; q < kR * kMaxG; ++q) {
+                const int r = q / kMaxG, j = q % kMaxG;
+                const uint32_t bmsm = st + (uint32_t)(r * G + j) * 512u;
+                if (work && r < rows && j < g) {
+                    // lane handles BTs `lane` and `lane + 32` of the GT (storage order)
+                    ba[q] = lds_v2(bmsm + 8u * lane);
+                    bb[q] = lds_v2(bmsm + 256u + 8u * lane);
+                } else {
+                    ba[q] = make_uint2(0u, 0u);
+                    bb[q] = make_uint2(0u, 0u);
+                }
+            }
+#pragma unroll
+            for (int q = 0; q < kR * kMaxG; ++q) {
+                packed[q] = (__popc(ba[q].x) + __popc(ba[q].y)) | ((__popc(bb[q].x) + __popc(bb[q].y)) << 16);
+                incl[q] = packed[q];
+            }
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                uint32_t y[kR * kMaxG];
+#pragma unroll
+                for (int q = 0; q < kR * kMaxG; ++q) y[q] = __shfl_up_sync(0xffffffffu, incl[q], o);
+#pragma unroll
+                for (int q = 0; q < kR * kMaxG; ++q) incl[q] += (lane >= o) ? y[q] : 0u;
+            }
+            uint32_t tot_a[kR * kMaxG];
+#pragma unroll
+            for (int q = 0; q < kR * kMaxG; ++q) tot_a[q] = __shfl_sync(0xffffffffu, incl[q], 31) & 0xFFFFu;
+            const int4 p0 = pre[u - u0];
+#pragma unroll
+            for (int q = 0; q < kR * kMaxG; ++q) {
+                const int r = q / kMaxG, j = q % kMaxG;
+                if (work && r < rows && j < g) {
+                    const int4 pj = pre[u - u0 + j];
+                    const int rel = r ? (pj.z - p0.z) : (pj.x - p0.x);          // GT j's values in the chunk
+                    const uint32_t vsm = st + (r ? prm.st_v1 : prm.st_v0);
+                    const uint32_t excl = incl[q] - packed[q];
+                    const uint32_t ea = excl & 0xFFFFu, eb = tot_a[q] + (excl >> 16);   // PopCount prefix
+                    const uint32_t Aa = vsm + 2u * (uint32_t)(rel + (int)ea);
+                    const uint32_t Ab = vsm + 2u * (uint32_t)(rel + (int)eb);
                     const uint32_t te = tb + (uint32_t)(r * G + j) * 1024u + 8u * lane;
-                    sts_v2(te, ba.x, Aa);
-                    sts_v2(te + 512u, ba.y, Aa + 2u * pal);
-                    sts_v2(te + 256u, bb.x, Ab);
-                    sts_v2(te + 768u, bb.y, Ab + 2u * pbl);
+                    sts_v2(te, ba[q].x, Aa);
+                    sts_v2(te + 512u, ba[q].y, Aa + 2u * __popc(ba[q].x));
+                    sts_v2(te + 256u, bb[q].x, Ab);
+                    sts_v2(te + 768u, bb[q].y, Ab + 2u * __popc(bb[q].x));
                 }
             }
             mbar_arrive(bar_scan + 8 * t);
+            if (lane == 0) trace_ev(prm, p, i, 3);
             u += g;
         }
         return;
@@ -254,8 +289,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
                     for (int q = 0; q < 4; ++q) acc[a][b][q] = 0.f;
         }
         mbar_wait(bar_full + 8 * slot, (i / S) & 1);
+        if (cw == 0 && lane == 0) trace_ev(prm, p, i, 4);
         mbar_wait(bar_scan + 8 * t, (i / kTblSlots) & 1);
-        if (r < rows) {
+        if (cw == 0 && lane == 0) trace_ev(prm, p, i, 5);
+        if (r < rows && !(prm.dbg & 1)) {
             const uint32_t xs = sbase + prm.o_stage + slot * prm.stage_bytes + prm.st_x + xlane;
             // this warp's 16 entries of GT j (TCTiles c*4 .. c*4+3, all 4 BTs): 128 contiguous bytes
             const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes + (uint32_t)(r * G) * 1024u + hioff +
@@ -312,6 +349,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
         if (lane == 0) {
             mbar_arrive(bar_empty + 8 * slot);
             mbar_arrive(bar_tble + 8 * t);
+            if (cw == 0) trace_ev(prm, p, i, 6);
         }
         u += g;
         const bool seg_end = (gc + g == KG) || (u == u1);
@@ -446,7 +484,10 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
     maxv = min(4096, (maxv + 7) & ~7);
     const uint32_t o_pre = 256;
     const uint32_t pre_bytes = align_up((uint32_t)(16 * upc), 128);
-    for (int G = 4; G >= 1; --G) {
+    int gmax = kMaxG, smax = kMaxStages;
+    if (const char *e = getenv("SPINFER_G")) gmax = std::max(1, std::min(kMaxG, atoi(e)));
+    if (const char *e = getenv("SPINFER_S")) smax = std::max(2, std::min(kMaxStages, atoi(e)));
+    for (int G = gmax; G >= 1; --G) {
         uint32_t tbl = (uint32_t)kR * G * 64 * 16;
         uint32_t scr = (uint32_t)kR * 2 * 64 * N * 4;
         uint32_t st_x = (uint32_t)kR * G * 512;
@@ -456,7 +497,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         uint32_t stage = align_up(st_v1 + vcap, 128);
         uint32_t fixed = o_pre + pre_bytes + kTblSlots * tbl + scr + 128;   // +slack for the t1 over-read
         if ((long long)fixed + 2LL * stage > smem_max) continue;
-        int S = (int)std::min<long long>(kMaxStages, ((long long)smem_max - fixed) / stage);
+        int S = (int)std::min<long long>(smax, ((long long)smem_max - fixed) / stage);
         if (S < 3 && G > 1) continue;
         pl->G = G;
         pl->S = S;
@@ -512,13 +553,32 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     q.Y = Y;
     q.ws_cnt = reinterpret_cast<int32_t *>(ws);
     q.ws_part = reinterpret_cast<float *>(reinterpret_cast<uint8_t *>(ws) + kCounterBytes);
-    switch (N) {
-        case 8: return launch_nt<1>(pl, st);
-        case 16: return launch_nt<2>(pl, st);
-        case 24: return launch_nt<3>(pl, st);
-        case 32: return launch_nt<4>(pl, st);
-        default: return SPINFER_EINVAL;
+    q.dbg = 0;
+    if (const char *e = getenv("SPINFER_DEBUG_MODE")) q.dbg = atoi(e);
+    q.trace = nullptr;
+    static long long *trace_buf = nullptr;
+    const char *trace_path = getenv("SPINFER_TRACE");
+    const size_t trace_n = (size_t)kTraceCTAs * kTraceStages * 8;
+    if (trace_path) {
+        if (!trace_buf && cudaMalloc(&trace_buf, trace_n * 8) != cudaSuccess) return SPINFER_ECUDA;
+        cudaMemsetAsync(trace_buf, 0, trace_n * 8, st);
+        q.trace = trace_buf;
     }
+    int rc = SPINFER_EINVAL;
+    switch (N) {
+        case 8: rc = launch_nt<1>(pl, st); break;
+        case 16: rc = launch_nt<2>(pl, st); break;
+        case 24: rc = launch_nt<3>(pl, st); break;
+        case 32: rc = launch_nt<4>(pl, st); break;
+        default: break;
+    }
+    if (trace_path && rc == SPINFER_OK) {   // debug only: synchronous dump of the stage timeline
+        static long long host[kTraceCTAs * kTraceStages * 8];
+        cudaMemcpyAsync(host, trace_buf, sizeof(host), cudaMemcpyDeviceToHost, st);
+        cudaStreamSynchronize(st);
+        if (FILE *f = fopen(trace_path, "wb")) { fwrite(host, 1, sizeof(host), f); fclose(f); }
+    }
+    return rc;
 }
 
 }  // namespace spinfer
