@@ -7,22 +7,28 @@
 // range per GT row). This replaces the paper's split-K grid mapping (Alg. 1
 // lines 1-3); rowblocks split across CTAs are combined by an
 // in-kernel "last arriver sums" fix-up (the paper's ReductionWorkspace).
+// A "stage" = up to G consecutive units of one rowblock.
 //
 // Warp roles (10 warps):
-//   warp 0    producer: one lane issues cp.async.bulk (TMA 1-D) copies of the
-//             stage's bitmaps, values and X slab into an S-stage smem ring,
-//             signalled on a full mbarrier with the byte count (replaces the
-//             paper's LDGSTS.128 double buffer).
-//   warp 1    scan: for each staged GroupTile computes every BitmapTile's base
-//             (PopCount prefix over earlier BTs) and writes a table of
-//             {bitmap half-word, smem address of that half's first value}.
+//   warp 0    producer: lane 0 issues one cp.async.bulk (1-D TMA) per GT row for
+//             the stage's packed values (the only large, contiguous stream); the
+//             32 lanes copy the stage's X slab (L2-resident) with 16-byte loads into
+//             a bank-conflict-free swizzled layout. S-stage smem ring, full/empty
+//             mbarriers (replaces the paper's LDGSTS.128 double buffer, P:224,
+//             P:293-301; measured: per-copy TMA overhead makes few, large copies
+//             the right shape on B200).
+//   warp 1    scan: loads each staged GroupTile's 64 bitmaps straight from global
+//             memory (coalesced, prefetched one stage ahead), computes every
+//             BitmapTile's base (PopCount prefix over earlier BTs) and
+//             writes a table {bitmap half-word, smem address of that half's first
+//             value} — bitmaps never pass through shared memory otherwise.
 //   warps 2-9 consumers (GT row r = w/4, TCTile column c = w%4): SMBD decode
 //             (MaskedPopCount, Alg. 2, two-phase a0/a1 P:287) into
 //             mma.m16n8k16 A fragments, X via ldmatrix.trans, mma.sync with
 //             fp32 accumulators (Listing 1).
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
-#include <algorithm>
 #include "internal.cuh"
 #include "ptx.cuh"
 
@@ -34,9 +40,9 @@ constexpr int kCW = 8;              // consumer warps = kR rows x 4 TCTile colum
 constexpr int kThreads = 32 * (2 + kCW);
 constexpr int kTblSlots = 2;
 constexpr int kMaxStages = 8;
-constexpr int kMaxG = 4;
-constexpr int kTraceCTAs = 4, kTraceStages = 64;            // max GroupTile columns per stage
-constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector table constant
+constexpr int kMaxG = 4;            // max GroupTile columns per stage
+constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector-table constants
+constexpr int kTraceCTAs = 4, kTraceStages = 64;
 // Workspace = [fix-up counters: one int32 per GT row, fixed-size region][split-K partials].
 // The counter region has the same size for every shape so that one zeroed
 // workspace can serve calls of different shapes (partials never overlap counters).
@@ -55,11 +61,11 @@ struct Params {
     long long U;
     int P;
     int G, S;
-    uint32_t stage_bytes, st_x, st_v0, st_v1;   // stage slot size; offsets in a slot (bitmaps at 0)
+    uint32_t stage_bytes, st_v0, st_v1;         // stage slot size; value offsets in a slot (X slab at 0)
     uint32_t tbl_bytes;
     uint32_t o_pre, o_tbl, o_scr, o_stage;      // region offsets from the smem base
     long long *trace;   // experiments only (SPINFER_TRACE): [kTraceCTAs][kTraceStages][8] clock64 stamps
-    int dbg;   // experiments only (SPINFER_DEBUG_MODE): bit0 = consumers skip decode/MMA, bit1 = scan warp skips work
+    int dbg;            // experiments only (SPINFER_DEBUG_MODE): bit0 = consumers skip decode/MMA, bit1 = scan skips work
 };
 
 __device__ __forceinline__ void trace_ev(const Params &prm, int p, int i, int ev) {
@@ -69,6 +75,30 @@ __device__ __forceinline__ void trace_ev(const Params &prm, int p, int i, int ev
 __device__ __forceinline__ long long unit_start(long long p, long long U, int P) { return p * U / P; }
 __device__ __forceinline__ int unit_owner(long long u, long long U, int P) {
     return (int)(((u + 1) * (long long)P - 1) / U);
+}
+
+// Stage descriptor: every role walks the same deterministic stage sequence.
+struct Stage {
+    int rb, gc, g, rows;
+};
+__device__ __forceinline__ Stage stage_at(long long u, long long u1, int KG, int G, int MG) {
+    Stage s;
+    s.rb = (int)(u / KG);
+    s.gc = (int)(u - (long long)s.rb * KG);
+    s.g = (int)min((long long)min(G, KG - s.gc), u1 - u);
+    s.rows = min(kR, MG - kR * s.rb);
+    return s;
+}
+
+// X slab swizzle (16-byte chunk granularity): row k of the slab holds N/8 chunks;
+// chunk c of row k is stored at chunk slot c ^ swz(k) so that the 8 row reads of
+// one ldmatrix phase hit 8 distinct bank groups (N = 16: rows are 32 B apart,
+// rows k and k+4 would collide; N = 32: rows k, k+2). N = 8 and 24 are conflict-free.
+template <int NT>
+__device__ __forceinline__ uint32_t x_swz(uint32_t k) {
+    if constexpr (NT == 2) return (k >> 2) & 1u;
+    else if constexpr (NT == 4) return (k >> 1) & 3u;
+    else return 0u;
 }
 
 // SMBD for one BitmapTile and one lane, split into phases so
@@ -85,9 +115,6 @@ __device__ __forceinline__ int unit_owner(long long u, long long U, int P) {
 //   y=0 -> 0x3232 (0,0)   y=1 -> 0x3210 (t0,0)   y=2 -> 0x1032 (0,t0)   y=3 -> 0x5410 (t0,t1)
 // low selector byte  = byte y of 0x10321032, high byte = byte y of 0x54103232,
 // so sel = prmt(0x10321032, 0x54103232, y*0x11 + 0x40).
-struct SmbdConst {
-    uint32_t lm, sh, ca, c40;
-};
 
 template <int NT>
 __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const float (&acc)[4][NT][4], int lane) {
@@ -112,7 +139,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int p = blockIdx.x;
     const long long U = prm.U;
-    const int KG = prm.KG, G = prm.G, S = prm.S;
+    const int KG = prm.KG, G = prm.G, S = prm.S, MG = prm.MG;
     const long long u0 = unit_start(p, U, prm.P), u1 = unit_start(p + 1, U, prm.P);
 
     // barriers: full[S], empty[S], scanned[2], tbl_empty[2]
@@ -122,7 +149,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
-            mbar_init(bar_full + 8 * s, 1);
+            mbar_init(bar_full + 8 * s, 32);      // the 32 producer lanes (+ TMA transaction bytes)
             mbar_init(bar_empty + 8 * s, kCW);
         }
         for (int t = 0; t < kTblSlots; ++t) {
@@ -130,8 +157,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             mbar_init(bar_tble + 8 * t, kCW);
         }
         fence_barrier_init();
-        // SMBD selector-table word, read back into a register by every consumer thread so
-        // ptxas keeps it live in a register instead of re-materialising it per PRMT.
+        // SMBD selector-table constants, read back into registers by every consumer thread so
+        // ptxas keeps them live in registers instead of re-materialising them per PRMT.
         reinterpret_cast<uint32_t *>(smem)[kConstWord] = 0x10321032u;
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = 0x40u;
     }
@@ -143,7 +170,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
         long long g0 = (long long)(kR * rb) * KG + gc;
         v.x = __ldg(prm.off + g0);
         v.y = __ldg(prm.off + g0 + 1);
-        if (kR * rb + 1 < prm.MG) {
+        if (kR * rb + 1 < MG) {
             v.z = __ldg(prm.off + g0 + KG);
             v.w = __ldg(prm.off + g0 + KG + 1);
         }
@@ -153,32 +180,45 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
 
     if (warp == 0) {
         // ------------------------------------------------------------ producer
-        if (lane != 0) return;
-        const uint64_t pol_w = policy_evict_first(), pol_x = policy_evict_last();
+        const uint64_t pol_w = policy_evict_first();
+        constexpr int cpr = N / 8;                     // 16-byte chunks per X row
         int i = 0;
         for (long long u = u0; u < u1; ++i) {
-            int rb = (int)(u / KG), gc = (int)(u % KG);
-            int g = (int)min((long long)min(G, KG - gc), u1 - u);
-            int rows = min(kR, prm.MG - kR * rb);
-            int slot = i % S;
+            const Stage sg = stage_at(u, u1, KG, G, MG);
+            const int slot = i % S;
             if (i >= S) mbar_wait(bar_empty + 8 * slot, ((i / S) - 1) & 1);
-            trace_ev(prm, p, i, 0);
+            if (lane == 0) trace_ev(prm, p, i, 0);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
-            const int4 ps = pre[u - u0], pe = pre[u - u0 + g - 1];
-            uint32_t vb0 = 2u * (uint32_t)(pe.y - ps.x);
-            uint32_t vb1 = rows > 1 ? 2u * (uint32_t)(pe.w - ps.z) : 0u;
-            uint32_t xb = (uint32_t)g * 64u * N * 2u;
-            uint32_t total = (uint32_t)rows * g * 512u + vb0 + vb1 + xb;
             const uint32_t fb = bar_full + 8 * slot;
-            mbar_arrive_expect_tx(fb, total);
-            for (int r = 0; r < rows; ++r) {
-                long long gA = (long long)(kR * rb + r) * KG + gc;
-                bulk_g2s(st + (uint32_t)(r * G) * 512u, prm.bm + gA * 64, (uint32_t)g * 512u, fb, pol_w);
+            if (lane == 0) {
+                const int4 ps = pre[u - u0], pe = pre[u - u0 + sg.g - 1];
+                const uint32_t vb0 = 2u * (uint32_t)(pe.y - ps.x);
+                const uint32_t vb1 = sg.rows > 1 ? 2u * (uint32_t)(pe.w - ps.z) : 0u;
+                mbar_expect_tx(fb, vb0 + vb1);
+                if (vb0) bulk_g2s(st + prm.st_v0, prm.vals + ps.x, vb0, fb, pol_w);
+                if (vb1) bulk_g2s(st + prm.st_v1, prm.vals + ps.z, vb1, fb, pol_w);
             }
-            if (vb0) bulk_g2s(st + prm.st_v0, prm.vals + ps.x, vb0, fb, pol_w);
-            if (vb1) bulk_g2s(st + prm.st_v1, prm.vals + ps.z, vb1, fb, pol_w);
-            bulk_g2s(st + prm.st_x, prm.X + (size_t)gc * 64 * N, xb, fb, pol_x);
-            u += g;
+            // X slab rows [64 gc, 64 (gc + g)) -> smem, 16 B per lane per step, swizzled.
+            const uint4 *xsrc = reinterpret_cast<const uint4 *>(prm.X + (size_t)sg.gc * 64 * N);
+            const int nchunk = sg.g * 64 * cpr;
+            for (int e0 = 0; e0 < nchunk; e0 += 32 * 8) {
+                uint4 v[8];
+#pragma unroll
+                for (int q = 0; q < 8; ++q) {
+                    const int e = e0 + q * 32 + lane;
+                    if (e < nchunk) v[q] = ldg_nc_v4(xsrc + e);
+                }
+#pragma unroll
+                for (int q = 0; q < 8; ++q) {
+                    const int e = e0 + q * 32 + lane;
+                    if (e < nchunk) {
+                        const uint32_t k = (uint32_t)(e / cpr), cch = (uint32_t)(e % cpr);
+                        sts_v4(st + (k * cpr + (cch ^ x_swz<NT>(k))) * 16u, v[q]);
+                    }
+                }
+            }
+            mbar_arrive(fb);   // release: this lane's X stores are visible to the consumers' acquire
+            u += sg.g;
         }
         return;
     }
@@ -187,58 +227,59 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
         // ------------------------------------------------------------ scan
         // Table per staged GT (r, j), 1024 B: [lane-half h][BT in GT storage order] {w, A},
         // so a consumer lane fetches the entries of 2 consecutive BTs with one 16-B load.
+        // Bitmaps come from global memory, prefetched one stage ahead; all rows x g GTs of
+        // a stage are scanned together (static bounds, unconditional full-warp shuffles,
+        // absent GTs scan zeros) so the independent shuffle chains interleave.
+        constexpr int Q = kR * kMaxG;
+        const bool work = !(prm.dbg & 2);
+        uint2 ba[Q], bb[Q], na[Q], nb[Q];
+        auto fetch = [&](long long u, uint2 (&a)[Q], uint2 (&b)[Q]) {
+            const Stage sg = stage_at(u, u1, KG, G, MG);
+#pragma unroll
+            for (int q = 0; q < Q; ++q) {
+                const int r = q / kMaxG, j = q % kMaxG;
+                if (work && u < u1 && r < sg.rows && j < sg.g) {
+                    const uint64_t *src = prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc + j) * 64;
+                    a[q] = ldg_nc_v2(src + lane);          // BT `lane` of the GT (storage order)
+                    b[q] = ldg_nc_v2(src + 32 + lane);     // BT `lane + 32`
+                } else {
+                    a[q] = make_uint2(0u, 0u);
+                    b[q] = make_uint2(0u, 0u);
+                }
+            }
+        };
+        fetch(u0, ba, bb);
         int i = 0;
         for (long long u = u0; u < u1; ++i) {
-            int rb = (int)(u / KG), gc = (int)(u % KG);
-            int g = (int)min((long long)min(G, KG - gc), u1 - u);
-            int rows = min(kR, prm.MG - kR * rb);
-            int slot = i % S, t = i & 1;
-            mbar_wait(bar_full + 8 * slot, (i / S) & 1);
-            if (lane == 0) trace_ev(prm, p, i, 1);
+            const Stage sg = stage_at(u, u1, KG, G, MG);
+            const int slot = i % S, t = i & 1;
+            fetch(u + sg.g, na, nb);                       // next stage's bitmaps in flight
             if (i >= kTblSlots) mbar_wait(bar_tble + 8 * t, ((i / kTblSlots) - 1) & 1);
             if (lane == 0) trace_ev(prm, p, i, 2);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes;
-            // all rows x g GroupTiles of the stage are scanned together: slot q = r*kMaxG + j,
-            // static bounds, unconditional full-warp shuffles (absent GTs scan zeros), so the
-            // kR*kMaxG independent shuffle chains interleave (ILP) with no divergence handling.
-            const bool work = !(prm.dbg & 2);
-            uint2 ba[kR * kMaxG], bb[kR * kMaxG];
-            uint32_t packed[kR * kMaxG], incl[kR * kMaxG];
+            uint32_t packed[Q], incl[Q];
 #pragma unroll
-            for (int q = 0; q < kR * kMaxG; ++q) {
-                const int r = q / kMaxG, j = q % kMaxG;
-                const uint32_t bmsm = st + (uint32_t)(r * G + j) * 512u;
-                if (work && r < rows && j < g) {
-                    // lane handles BTs `lane` and `lane + 32` of the GT (storage order)
-                    ba[q] = lds_v2(bmsm + 8u * lane);
-                    bb[q] = lds_v2(bmsm + 256u + 8u * lane);
-                } else {
-                    ba[q] = make_uint2(0u, 0u);
-                    bb[q] = make_uint2(0u, 0u);
-                }
-            }
-#pragma unroll
-            for (int q = 0; q < kR * kMaxG; ++q) {
+            for (int q = 0; q < Q; ++q) {
                 packed[q] = (__popc(ba[q].x) + __popc(ba[q].y)) | ((__popc(bb[q].x) + __popc(bb[q].y)) << 16);
                 incl[q] = packed[q];
             }
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
-                uint32_t y[kR * kMaxG];
+                uint32_t y[Q];
 #pragma unroll
-                for (int q = 0; q < kR * kMaxG; ++q) y[q] = __shfl_up_sync(0xffffffffu, incl[q], o);
+                for (int q = 0; q < Q; ++q) y[q] = __shfl_up_sync(0xffffffffu, incl[q], o);
 #pragma unroll
-                for (int q = 0; q < kR * kMaxG; ++q) incl[q] += (lane >= o) ? y[q] : 0u;
+                for (int q = 0; q < Q; ++q) incl[q] += (lane >= o) ? y[q] : 0u;
             }
-            uint32_t tot_a[kR * kMaxG];
+            uint32_t tot_a[Q];
 #pragma unroll
-            for (int q = 0; q < kR * kMaxG; ++q) tot_a[q] = __shfl_sync(0xffffffffu, incl[q], 31) & 0xFFFFu;
+            for (int q = 0; q < Q; ++q) tot_a[q] = __shfl_sync(0xffffffffu, incl[q], 31) & 0xFFFFu;
             const int4 p0 = pre[u - u0];
 #pragma unroll
-            for (int q = 0; q < kR * kMaxG; ++q) {
+            for (int q = 0; q < Q; ++q) {
                 const int r = q / kMaxG, j = q % kMaxG;
-                if (work && r < rows && j < g) {
+                if (work && r < sg.rows && j < sg.g) {
                     const int4 pj = pre[u - u0 + j];
                     const int rel = r ? (pj.z - p0.z) : (pj.x - p0.x);          // GT j's values in the chunk
                     const uint32_t vsm = st + (r ? prm.st_v1 : prm.st_v0);
@@ -255,7 +296,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             }
             mbar_arrive(bar_scan + 8 * t);
             if (lane == 0) trace_ev(prm, p, i, 3);
-            u += g;
+#pragma unroll
+            for (int q = 0; q < Q; ++q) {
+                ba[q] = na[q];
+                bb[q] = nb[q];
+            }
+            u += sg.g;
         }
         return;
     }
@@ -264,20 +310,22 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
     const int cw = warp - 2, r = cw >> 2, c = cw & 3;
     const uint32_t sh = 2u * (lane & 15);
     const uint32_t lm = (1u << sh) - 1u;
-    const uint32_t ca = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];   // 0x10321032
-    const uint32_t c40 = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];   // 0x40
+    const uint32_t ca = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];       // 0x10321032
+    const uint32_t c40 = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];  // 0x40
     const uint32_t hioff = (uint32_t)(lane >> 4) * 512u;
-    // ldmatrix.trans row addresses: matrix m = lane/8 -> (k half m&1, n half m>>1)
-    const uint32_t xlane = (uint32_t)((((lane >> 3) & 1) * 8 + (lane & 7)) * N + ((lane >> 4) & 1) * 8) * 2u;
+    // ldmatrix.trans rows: matrix m = lane/8 -> (k half m&1, n chunk m>>1); row rr = lane%8.
+    constexpr uint32_t cpr = N / 8;
+    const uint32_t rr = lane & 7, mk = (lane >> 3) & 1, mn = (lane >> 4) & 1;
+    const uint32_t xrow = (uint32_t)(mk * 8 + rr) * cpr;   // + (64 j + 16 c) * cpr per k16 column
+    const uint32_t xsw = x_swz<NT>(rr);                     // swizzle depends on k % 8 == rr only
     float acc[4][NT][4];
     const uint32_t scr = sbase + prm.o_scr + (uint32_t)r * (2u * 64u * N * 4u);
 
     int i = 0;
     long long seg_u0 = u0;
     for (long long u = u0; u < u1; ++i) {
-        const int rb = (int)(u / KG), gc = (int)(u % KG);
-        const int g = (int)min((long long)min(G, KG - gc), u1 - u);
-        const int rows = min(kR, prm.MG - kR * rb);
+        const Stage sg = stage_at(u, u1, KG, G, MG);
+        const int rb = sg.rb, gc = sg.gc, g = sg.g, rows = sg.rows;
         const int slot = i % S, t = i & 1;
         if (gc == 0 || u == u0) {
             seg_u0 = u;
@@ -293,7 +341,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
         mbar_wait(bar_scan + 8 * t, (i / kTblSlots) & 1);
         if (cw == 0 && lane == 0) trace_ev(prm, p, i, 5);
         if (r < rows && !(prm.dbg & 1)) {
-            const uint32_t xs = sbase + prm.o_stage + slot * prm.stage_bytes + prm.st_x + xlane;
+            const uint32_t xs = sbase + prm.o_stage + slot * prm.stage_bytes;
             // this warp's 16 entries of GT j (TCTiles c*4 .. c*4+3, all 4 BTs): 128 contiguous bytes
             const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes + (uint32_t)(r * G) * 1024u + hioff +
                                 (uint32_t)c * 128u;
@@ -322,14 +370,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
 #pragma unroll
                 for (int q = 0; q < 8; ++q) E[q] = lds_v4(tb + (uint32_t)(j + 1) * 1024u + 16u * q);
                 uint32_t bfr[NT][2];
-                const uint32_t xk = xs + (uint32_t)(64 * j + 16 * c) * N * 2u;
+                const uint32_t xk = xs + (xrow + (uint32_t)(64 * j + 16 * c) * cpr) * 16u;
                 if constexpr (NT == 1) {
                     ldsm_x2_trans(xk, bfr[0][0], bfr[0][1]);
                 } else {
 #pragma unroll
                     for (int nt = 0; nt + 1 < NT; nt += 2)
-                        ldsm_x4_trans(xk + nt * 16u, bfr[nt][0], bfr[nt][1], bfr[nt + 1][0], bfr[nt + 1][1]);
-                    if constexpr (NT % 2 == 1) ldsm_x2_trans(xk + (NT - 1) * 16u, bfr[NT - 1][0], bfr[NT - 1][1]);
+                        ldsm_x4_trans(xk + (((uint32_t)nt + mn) ^ xsw) * 16u, bfr[nt][0], bfr[nt][1], bfr[nt + 1][0],
+                                      bfr[nt + 1][1]);
+                    if constexpr (NT % 2 == 1) ldsm_x2_trans(xk + (uint32_t)(NT - 1) * 16u, bfr[NT - 1][0], bfr[NT - 1][1]);
                 }
                 // phase 4: assemble the A fragments (Ra0..Ra3 = BTs TL,BL,TR,BR) and mma
 #pragma unroll
@@ -456,6 +505,7 @@ struct Plan {
 int num_sms() {
     int dev = 0, n = kNumSMsDefault;
     if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    cudaGetLastError();
     return n > 0 ? n : kNumSMsDefault;
 }
 
@@ -463,10 +513,10 @@ int choose_P(long long U) {
     long long cap = num_sms();
     // SPINFER_MAX_CTAS caps the persistent grid (tests use it to force many stages per CTA)
     if (const char *e = getenv("SPINFER_MAX_CTAS")) { long long v = atoll(e); if (v > 0 && v < cap) cap = v; }
-    long long P = min(cap, U);
+    long long P = std::min(cap, U);
     // keep the preloaded offsets (16 B per unit) within 16 KiB of shared memory
     while ((U + P - 1) / P > 1024) P += num_sms();
-    return (int)max(1LL, P);
+    return (int)std::max(1LL, P);
 }
 
 inline uint32_t align_up(uint32_t x, uint32_t a) { return (x + a - 1) / a * a; }
@@ -480,8 +530,9 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
     int dev = 0, smem_max = 232448;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    cudaGetLastError();
     int maxv = max_gt_values > 0 ? max_gt_values : 4096;
-    maxv = min(4096, (maxv + 7) & ~7);
+    maxv = std::min(4096, (maxv + 7) & ~7);
     const uint32_t o_pre = 256;
     const uint32_t pre_bytes = align_up((uint32_t)(16 * upc), 128);
     int gmax = kMaxG, smax = kMaxStages;
@@ -490,8 +541,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
     for (int G = gmax; G >= 1; --G) {
         uint32_t tbl = (uint32_t)kR * G * 64 * 16;
         uint32_t scr = (uint32_t)kR * 2 * 64 * N * 4;
-        uint32_t st_x = (uint32_t)kR * G * 512;
-        uint32_t st_v0 = st_x + (uint32_t)G * 64 * N * 2;
+        uint32_t st_v0 = (uint32_t)G * 64 * N * 2;            // X slab first
         uint32_t vcap = align_up((uint32_t)G * maxv * 2, 16);
         uint32_t st_v1 = st_v0 + vcap;
         uint32_t stage = align_up(st_v1 + vcap, 128);
@@ -503,7 +553,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         pl->S = S;
         Params &q = pl->prm;
         q.KG = KG; q.MG = MG; q.U = pl->U; q.P = pl->P; q.G = G; q.S = S;
-        q.stage_bytes = stage; q.st_x = st_x; q.st_v0 = st_v0; q.st_v1 = st_v1;
+        q.stage_bytes = stage; q.st_v0 = st_v0; q.st_v1 = st_v1;
         q.tbl_bytes = tbl;
         q.o_pre = o_pre;
         q.o_tbl = o_pre + pre_bytes;
@@ -517,11 +567,14 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
 
 template <int NT>
 int launch_nt(const Plan &pl, cudaStream_t st) {
-    static int configured_smem = 0;   // per-instantiation max dynamic smem already set
-    if ((int)pl.smem > configured_smem) {
+    static int configured_smem[64] = {0};   // per device: max dynamic smem already set for this instantiation
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if ((int)pl.smem > configured_smem[dev]) {
         if (cudaFuncSetAttribute(k_spmm<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem) != cudaSuccess)
             return SPINFER_ECUDA;
-        configured_smem = (int)pl.smem;
+        configured_smem[dev] = (int)pl.smem;
     }
     k_spmm<NT><<<pl.P, kThreads, pl.smem, st>>>(pl.prm);
     return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
