@@ -76,6 +76,16 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t
         ::"r"(dst), "l"(src), "r"(bytes), "r"(bar), "l"(policy) : "memory");
 }
 
+// cp.async (LDGSTS) 16 B global -> shared, L2 only; completion tracked by an mbarrier:
+// cp.async.mbarrier.arrive.noinc makes the barrier observe one arrival when all of
+// this thread's prior cp.async operations have completed.
+__device__ __forceinline__ void cp_async_16(uint32_t dst, const void *src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_mbar_arrive_noinc(uint32_t bar) {
+    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
+}
+
 // ---------------------------------------------------------------- shared loads
 __device__ __forceinline__ uint2 lds_v2(uint32_t a) {
     uint2 v;

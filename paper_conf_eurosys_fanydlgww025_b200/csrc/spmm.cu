@@ -198,26 +198,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
                 if (vb0) bulk_g2s(st + prm.st_v0, prm.vals + ps.x, vb0, fb, pol_w);
                 if (vb1) bulk_g2s(st + prm.st_v1, prm.vals + ps.z, vb1, fb, pol_w);
             }
-            // X slab rows [64 gc, 64 (gc + g)) -> smem, 16 B per lane per step, swizzled.
+            // X slab rows [64 gc, 64 (gc + g)) -> smem with asynchronous 16-byte copies
+            // (LDGSTS, L2-resident source), swizzled; each lane's completion arrives on the
+            // full barrier (noinc: one of its 32 expected arrivals).
             const uint4 *xsrc = reinterpret_cast<const uint4 *>(prm.X + (size_t)sg.gc * 64 * N);
             const int nchunk = sg.g * 64 * cpr;
-            for (int e0 = 0; e0 < nchunk; e0 += 32 * 8) {
-                uint4 v[8];
-#pragma unroll
-                for (int q = 0; q < 8; ++q) {
-                    const int e = e0 + q * 32 + lane;
-                    if (e < nchunk) v[q] = ldg_nc_v4(xsrc + e);
-                }
-#pragma unroll
-                for (int q = 0; q < 8; ++q) {
-                    const int e = e0 + q * 32 + lane;
-                    if (e < nchunk) {
-                        const uint32_t k = (uint32_t)(e / cpr), cch = (uint32_t)(e % cpr);
-                        sts_v4(st + (k * cpr + (cch ^ x_swz<NT>(k))) * 16u, v[q]);
-                    }
-                }
+            for (int e = lane; e < nchunk; e += 32) {
+                const uint32_t k = (uint32_t)(e / cpr), cch = (uint32_t)(e % cpr);
+                cp_async_16(st + (k * cpr + (cch ^ x_swz<NT>(k))) * 16u, xsrc + e);
             }
-            mbar_arrive(fb);   // release: this lane's X stores are visible to the consumers' acquire
+            cp_async_mbar_arrive_noinc(fb);
             u += sg.g;
         }
         return;
