@@ -12,16 +12,15 @@
 // Warp roles (10 warps):
 //   warp 0    producer: lane 0 issues one cp.async.bulk (1-D TMA) per GT row for
 //             the stage's packed values (the only large, contiguous stream); the
-//             32 lanes copy the stage's X slab (L2-resident) with 16-byte loads into
-//             a bank-conflict-free swizzled layout. S-stage smem ring, full/empty
+//             32 lanes copy the stage's bitmaps and X slab (L2-resident) with
+//             16-byte cp.async into the slot (X swizzled bank-conflict-free),
+//             completing on the same barrier. S-stage smem ring, full/empty
 //             mbarriers (replaces the paper's LDGSTS.128 double buffer, P:224,
 //             P:293-301; measured: per-copy TMA overhead makes few, large copies
 //             the right shape on B200).
-//   warp 1    scan: loads each staged GroupTile's 64 bitmaps straight from global
-//             memory (coalesced, prefetched one stage ahead), computes every
-//             BitmapTile's base (PopCount prefix over earlier BTs) and
-//             writes a table {bitmap half-word, smem address of that half's first
-//             value} — bitmaps never pass through shared memory otherwise.
+//   warp 1    scan: for each staged GroupTile computes every BitmapTile's base
+//             (PopCount prefix over earlier BTs) and writes a table
+//             {bitmap half-word, smem address of that half's first value}.
 //   warps 2-9 consumers (GT row r = w/4, TCTile column c = w%4): SMBD decode
 //             (MaskedPopCount, Alg. 2, two-phase a0/a1 P:287) into
 //             mma.m16n8k16 A fragments, X via ldmatrix.trans, mma.sync with
@@ -61,7 +60,7 @@ struct Params {
     long long U;
     int P;
     int G, S;
-    uint32_t stage_bytes, st_v0, st_v1;         // stage slot size; value offsets in a slot (X slab at 0)
+    uint32_t stage_bytes, st_bm, st_v0, st_v1;  // stage slot size; offsets in a slot (X slab at 0)
     uint32_t tbl_bytes;
     uint32_t o_pre, o_tbl, o_scr, o_stage;      // region offsets from the smem base
     long long *trace;   // experiments only (SPINFER_TRACE): [kTraceCTAs][kTraceStages][8] clock64 stamps
@@ -207,6 +206,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
                 const uint32_t k = (uint32_t)(e / cpr), cch = (uint32_t)(e % cpr);
                 cp_async_16(st + (k * cpr + (cch ^ x_swz<NT>(k))) * 16u, xsrc + e);
             }
+            // the stage's bitmaps (per GT row: g x 512 contiguous bytes) the same way
+            for (int r = 0; r < sg.rows; ++r) {
+                const uint4 *bsrc = reinterpret_cast<const uint4 *>(prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc) * 64);
+                const uint32_t bdst = st + prm.st_bm + (uint32_t)(r * G) * 512u;
+                for (int e = lane; e < sg.g * 32; e += 32) cp_async_16(bdst + 16u * e, bsrc + e);
+            }
             cp_async_mbar_arrive_noinc(fb);
             u += sg.g;
         }
@@ -217,35 +222,31 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
         // ------------------------------------------------------------ scan
         // Table per staged GT (r, j), 1024 B: [lane-half h][BT in GT storage order] {w, A},
         // so a consumer lane fetches the entries of 2 consecutive BTs with one 16-B load.
-        // Bitmaps come from global memory, prefetched one stage ahead; all rows x g GTs of
-        // a stage are scanned together (static bounds, unconditional full-warp shuffles,
+        // All rows x g GTs of a stage are scanned together (static bounds, unconditional full-warp shuffles,
         // absent GTs scan zeros) so the independent shuffle chains interleave.
         constexpr int Q = kR * kMaxG;
         const bool work = !(prm.dbg & 2);
-        uint2 ba[Q], bb[Q], na[Q], nb[Q];
-        auto fetch = [&](long long u, uint2 (&a)[Q], uint2 (&b)[Q]) {
-            const Stage sg = stage_at(u, u1, KG, G, MG);
-#pragma unroll
-            for (int q = 0; q < Q; ++q) {
-                const int r = q / kMaxG, j = q % kMaxG;
-                if (work && u < u1 && r < sg.rows && j < sg.g) {
-                    const uint64_t *src = prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc + j) * 64;
-                    a[q] = ldg_nc_v2(src + lane);          // BT `lane` of the GT (storage order)
-                    b[q] = ldg_nc_v2(src + 32 + lane);     // BT `lane + 32`
-                } else {
-                    a[q] = make_uint2(0u, 0u);
-                    b[q] = make_uint2(0u, 0u);
-                }
-            }
-        };
-        fetch(u0, ba, bb);
         int i = 0;
         for (long long u = u0; u < u1; ++i) {
             const Stage sg = stage_at(u, u1, KG, G, MG);
             const int slot = i % S, t = i & 1;
-            fetch(u + sg.g, na, nb);                       // next stage's bitmaps in flight
+            mbar_wait(bar_full + 8 * slot, (i / S) & 1);
+            if (lane == 0) trace_ev(prm, p, i, 1);
             if (i >= kTblSlots) mbar_wait(bar_tble + 8 * t, ((i / kTblSlots) - 1) & 1);
             if (lane == 0) trace_ev(prm, p, i, 2);
+            uint2 ba[Q], bb[Q];
+#pragma unroll
+            for (int q = 0; q < Q; ++q) {
+                const int r = q / kMaxG, j = q % kMaxG;
+                const uint32_t bmsm = sbase + prm.o_stage + slot * prm.stage_bytes + prm.st_bm + (uint32_t)(r * G + j) * 512u;
+                if (work && r < sg.rows && j < sg.g) {
+                    ba[q] = lds_v2(bmsm + 8u * lane);          // BT `lane` of the GT (storage order)
+                    bb[q] = lds_v2(bmsm + 256u + 8u * lane);   // BT `lane + 32`
+                } else {
+                    ba[q] = make_uint2(0u, 0u);
+                    bb[q] = make_uint2(0u, 0u);
+                }
+            }
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes;
             uint32_t packed[Q], incl[Q];
@@ -286,11 +287,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             }
             mbar_arrive(bar_scan + 8 * t);
             if (lane == 0) trace_ev(prm, p, i, 3);
-#pragma unroll
-            for (int q = 0; q < Q; ++q) {
-                ba[q] = na[q];
-                bb[q] = nb[q];
-            }
             u += sg.g;
         }
         return;
@@ -531,7 +527,8 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
     for (int G = gmax; G >= 1; --G) {
         uint32_t tbl = (uint32_t)kR * G * 64 * 16;
         uint32_t scr = (uint32_t)kR * 2 * 64 * N * 4;
-        uint32_t st_v0 = (uint32_t)G * 64 * N * 2;            // X slab first
+        uint32_t st_bm = (uint32_t)G * 64 * N * 2;            // X slab first, then bitmaps
+        uint32_t st_v0 = st_bm + (uint32_t)kR * G * 512;
         uint32_t vcap = align_up((uint32_t)G * maxv * 2, 16);
         uint32_t st_v1 = st_v0 + vcap;
         uint32_t stage = align_up(st_v1 + vcap, 128);
@@ -543,7 +540,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         pl->S = S;
         Params &q = pl->prm;
         q.KG = KG; q.MG = MG; q.U = pl->U; q.P = pl->P; q.G = G; q.S = S;
-        q.stage_bytes = stage; q.st_v0 = st_v0; q.st_v1 = st_v1;
+        q.stage_bytes = stage; q.st_bm = st_bm; q.st_v0 = st_v0; q.st_v1 = st_v1;
         q.tbl_bytes = tbl;
         q.o_pre = o_pre;
         q.o_tbl = o_pre + pre_bytes;
