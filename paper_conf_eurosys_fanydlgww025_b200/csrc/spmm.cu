@@ -9,8 +9,8 @@
 // in-kernel "last arriver sums" fix-up (the paper's ReductionWorkspace).
 // A "stage" = up to G consecutive units of one rowblock.
 //
-// Warp roles (10 warps):
-//   warp 0    producer: lane 0 issues one cp.async.bulk (1-D TMA) per GT row for
+// Warp roles (10 warps; ids chosen for scheduler priority, see kProducerWarp):
+//   warp 9    producer: lane 0 issues one cp.async.bulk (1-D TMA) per GT row for
 //             the stage's packed values (the only large, contiguous stream); the
 //             32 lanes copy the stage's bitmaps and X slab (L2-resident) with
 //             16-byte cp.async into the slot (X swizzled bank-conflict-free),
@@ -18,10 +18,10 @@
 //             mbarriers (replaces the paper's LDGSTS.128 double buffer, P:224,
 //             P:293-301; measured: per-copy TMA overhead makes few, large copies
 //             the right shape on B200).
-//   warp 1    scan: for each staged GroupTile computes every BitmapTile's base
+//   warp 8    scan: for each staged GroupTile computes every BitmapTile's base
 //             (PopCount prefix over earlier BTs) and writes a table
 //             {bitmap half-word, smem address of that half's first value}.
-//   warps 2-9 consumers (GT row r = w/4, TCTile column c = w%4): SMBD decode
+//   warps 0-7 consumers (GT row r = w/4, TCTile column c = w%4): SMBD decode
 //             (MaskedPopCount, Alg. 2, two-phase a0/a1 P:287) into
 //             mma.m16n8k16 A fragments, X via ldmatrix.trans, mma.sync with
 //             fp32 accumulators (Listing 1).
@@ -37,6 +37,9 @@ namespace {
 constexpr int kR = 2;               // GT rows per rowblock (128 output rows)
 constexpr int kCW = 8;              // consumer warps = kR rows x 4 TCTile columns
 constexpr int kThreads = 32 * (2 + kCW);
+// Warp ids: the warp scheduler favours the highest warp id among eligible warps, so the
+// two latency-critical single-warp roles get the top ids and the consumers 0..kCW-1.
+constexpr int kScanWarp = kCW, kProducerWarp = kCW + 1;
 constexpr int kTblSlots = 2;
 constexpr int kMaxStages = 8;
 constexpr int kMaxG = 4;            // max GroupTile columns per stage
@@ -177,7 +180,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
     }
     __syncthreads();
 
-    if (warp == 0) {
+    if (warp == kProducerWarp) {
         // ------------------------------------------------------------ producer
         const uint64_t pol_w = policy_evict_first();
         constexpr int cpr = N / 8;                     // 16-byte chunks per X row
@@ -218,7 +221,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
         return;
     }
 
-    if (warp == 1) {
+    if (warp == kScanWarp) {
         // ------------------------------------------------------------ scan
         // Table per staged GT (r, j), 1024 B: [lane-half h][BT in GT storage order] {w, A},
         // so a consumer lane fetches the entries of 2 consecutive BTs with one 16-B load.
@@ -293,7 +296,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
     }
 
     // ---------------------------------------------------------------- consumers
-    const int cw = warp - 2, r = cw >> 2, c = cw & 3;
+    const int cw = warp, r = cw >> 2, c = cw & 3;
     const uint32_t sh = 2u * (lane & 15);
     const uint32_t lm = (1u << sh) - 1u;
     const uint32_t ca = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];       // 0x10321032
