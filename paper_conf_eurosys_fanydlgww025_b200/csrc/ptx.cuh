@@ -50,7 +50,13 @@ __device__ __forceinline__ bool mbar_try_wait_sleep(uint32_t bar, uint32_t parit
         : "=r"(ok) : "r"(bar), "r"(parity), "r"(0x100000u) : "memory");
     return ok != 0;
 }
+// Waits for the phase with the given parity. Hot-path waiters (whose phase is usually
+// already complete or about to be) spin on try_wait; waiters that typically block for a
+// long time (producer on a free slot) use the suspend-hinted form.
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+    while (!mbar_try_wait(bar, parity)) { }
+}
+__device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
     while (!mbar_try_wait_sleep(bar, parity)) { }
 }
 
