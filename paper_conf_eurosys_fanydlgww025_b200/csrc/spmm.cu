@@ -80,18 +80,40 @@ __device__ __forceinline__ int unit_owner(long long u, long long U, int P) {
     return (int)(((u + 1) * (long long)P - 1) / U);
 }
 
-// Stage descriptor: every role walks the same deterministic stage sequence.
-struct Stage {
-    int rb, gc, g, rows;
+// Stage iterator: every role walks the same deterministic stage sequence. All
+// per-stage bookkeeping is incremental (one 64-bit division at kernel start only):
+// ring slot / parity of the S-stage smem ring and of the 2-slot table ring.
+struct StageIter {
+    long long u, u1;
+    int KG, G, MG, S;
+    int rb, gc, g, rows;     // current stage: rowblock, first GT column, #units, #GT rows
+    int i;                   // stage index within the CTA
+    int slot, ph;            // smem ring slot and its phase parity ((i / S) & 1)
+    int t, tph;              // table slot (i & 1) and its parity ((i / 2) & 1)
+    __device__ __forceinline__ void init(long long u0_, long long u1_, int KG_, int G_, int MG_, int S_) {
+        u = u0_; u1 = u1_; KG = KG_; G = G_; MG = MG_; S = S_;
+        rb = (int)(u / KG);
+        gc = (int)(u - (long long)rb * KG);
+        i = 0; slot = 0; ph = 0; t = 0; tph = 0;
+        shape();
+    }
+    __device__ __forceinline__ void shape() {
+        g = min(G, KG - gc);
+        if ((long long)g > u1 - u) g = (int)(u1 - u);
+        rows = min(kR, MG - kR * rb);
+    }
+    __device__ __forceinline__ bool valid() const { return u < u1; }
+    __device__ __forceinline__ void next() {
+        u += g;
+        gc += g;
+        if (gc == KG) { gc = 0; ++rb; }
+        ++i;
+        if (++slot == S) { slot = 0; ph ^= 1; }
+        t ^= 1;
+        if (t == 0) tph ^= 1;
+        shape();
+    }
 };
-__device__ __forceinline__ Stage stage_at(long long u, long long u1, int KG, int G, int MG) {
-    Stage s;
-    s.rb = (int)(u / KG);
-    s.gc = (int)(u - (long long)s.rb * KG);
-    s.g = (int)min((long long)min(G, KG - s.gc), u1 - u);
-    s.rows = min(kR, MG - kR * s.rb);
-    return s;
-}
 
 // X slab swizzle (16-byte chunk granularity): row k of the slab holds N/8 chunks;
 // chunk c of row k is stored at chunk slot c ^ swz(k) so that the 8 row reads of
@@ -185,11 +207,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
         // ------------------------------------------------------------ producer
         const uint64_t pol_w = policy_evict_first();
         constexpr int cpr = N / 8;                     // 16-byte chunks per X row
-        int i = 0;
-        for (long long u = u0; u < u1; ++i) {
-            const Stage sg = stage_at(u, u1, KG, G, MG);
-            const int slot = i % S;
-            if (i >= S) mbar_wait(bar_empty + 8 * slot, ((i / S) - 1) & 1);
+        StageIter it;
+        for (it.init(u0, u1, KG, G, MG, S); it.valid(); it.next()) {
+            const StageIter &sg = it;
+            const long long u = it.u;
+            const int i = it.i, slot = it.slot;
+            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, it.ph ^ 1);
             if (lane == 0) trace_ev(prm, p, i, 0);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const uint32_t fb = bar_full + 8 * slot;
@@ -217,7 +240,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
                 for (int e = lane; e < sg.g * 32; e += 32) cp_async_16(bdst + 16u * e, bsrc + e);
             }
             cp_async_mbar_arrive_noinc(fb);
-            u += sg.g;
         }
         return;
     }
@@ -232,13 +254,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
         constexpr int Q = kMaxG;
         const int r = warp - kScanWarp;               // this scan warp's GT row
         const bool work = !(prm.dbg & 2);
-        int i = 0;
-        for (long long u = u0; u < u1; ++i) {
-            const Stage sg = stage_at(u, u1, KG, G, MG);
-            const int slot = i % S, t = i & 1;
-            mbar_wait(bar_full + 8 * slot, (i / S) & 1);
+        StageIter it;
+        for (it.init(u0, u1, KG, G, MG, S); it.valid(); it.next()) {
+            const StageIter &sg = it;
+            const long long u = it.u;
+            const int i = it.i, slot = it.slot, t = it.t;
+            mbar_wait(bar_full + 8 * slot, it.ph);
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 1);
-            if (i >= kTblSlots) mbar_wait(bar_tble + 8 * t, ((i / kTblSlots) - 1) & 1);
+            if (i >= kTblSlots) mbar_wait(bar_tble + 8 * t, it.tph ^ 1);
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 2);
             uint2 ba[Q], bb[Q];
 #pragma unroll
@@ -293,7 +316,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             }
             mbar_arrive(bar_scan + 8 * t);
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 3);
-            u += sg.g;
         }
         return;
     }
@@ -313,12 +335,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
     float acc[4][NT][4];
     const uint32_t scr = sbase + prm.o_scr + (uint32_t)r * (2u * 64u * N * 4u);
 
-    int i = 0;
     long long seg_u0 = u0;
-    for (long long u = u0; u < u1; ++i) {
-        const Stage sg = stage_at(u, u1, KG, G, MG);
-        const int rb = sg.rb, gc = sg.gc, g = sg.g, rows = sg.rows;
-        const int slot = i % S, t = i & 1;
+    StageIter it;
+    for (it.init(u0, u1, KG, G, MG, S); it.valid(); it.next()) {
+        const long long u = it.u;
+        const int rb = it.rb, gc = it.gc, g = it.g, rows = it.rows;
+        const int i = it.i, slot = it.slot, t = it.t;
         if (gc == 0 || u == u0) {
             seg_u0 = u;
 #pragma unroll
@@ -328,9 +350,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
 #pragma unroll
                     for (int q = 0; q < 4; ++q) acc[a][b][q] = 0.f;
         }
-        mbar_wait(bar_full + 8 * slot, (i / S) & 1);
+        mbar_wait(bar_full + 8 * slot, it.ph);
         if (cw == 0 && lane == 0) trace_ev(prm, p, i, 4);
-        mbar_wait(bar_scan + 8 * t, (i / kTblSlots) & 1);
+        mbar_wait(bar_scan + 8 * t, it.tph);
         if (cw == 0 && lane == 0) trace_ev(prm, p, i, 5);
         if (r < rows && !(prm.dbg & 1)) {
             const uint32_t xs = sbase + prm.o_stage + slot * prm.stage_bytes;
@@ -405,8 +427,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             mbar_arrive(bar_tble + 8 * t);
             if (cw == 0) trace_ev(prm, p, i, 6);
         }
-        u += g;
-        const bool seg_end = (gc + g == KG) || (u == u1);
+        const long long u_end = u + g;
+        const bool seg_end = (gc + g == KG) || (u_end == u1);
         if (seg_end && r < rows) {
             // -------------------------------------------------------- epilogue
             // (1) reduce the 4 TCTile-column partials of GT row r (tree via smem)
@@ -453,7 +475,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             if (c == 0) {
                 const int grow = kR * rb + r;
                 const int row_base = grow * 64;
-                const bool complete = (seg_u0 == (long long)rb * KG) && (u == (long long)(rb + 1) * KG);
+                const bool complete = (seg_u0 == (long long)rb * KG) && (u_end == (long long)(rb + 1) * KG);
                 if (complete) {
                     store_y<NT>(prm.Y, N, row_base, acc, lane);
                 } else {
