@@ -335,9 +335,67 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
     float acc[4][NT][4];
     const uint32_t scr = sbase + prm.o_scr + (uint32_t)r * (2u * 64u * N * 4u);
 
+    // Software pipeline over half-GT steps (8 BTs = TCTile rows 2h', 2h'+1 of GT j):
+    // while step h is assembled and multiplied, the value loads of step h+1 and the
+    // table entries of step h+2 are already in flight. Steps alternate between two
+    // register sets (A: first half of a GT, B: second half) so no copies are needed.
+    // The pipeline runs continuously across stages: during the last step of stage i the
+    // warp already waits for stage i+1 and issues its first loads.
+    uint4 E[4];
+    uint32_t tA0[8], tA1[8], sA[8], tB0[8], tB1[8], sB[8];
+    auto load_E = [&](uint32_t tb, int step) {   // table entries of step `step` (4 x 16 B per lane)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) E[q] = lds_v4(tb + (uint32_t)(step >> 1) * 1024u + (uint32_t)(step & 1) * 64u + 16u * q);
+    };
+    auto issue = [&](uint32_t (&t0)[8], uint32_t (&t1)[8], uint32_t (&s1)[8]) {   // value loads from E
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
+            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;
+            const uint32_t a = A + 2u * __popc(w & lm);
+            s1[k] = ((w >> sh) & 3u) * 0x11u + c40;
+            t0[k] = lds_u16(a);
+            t1[k] = lds_u16(a + 2u);
+        }
+    };
+    auto assemble = [&](const uint32_t (&t0)[8], const uint32_t (&t1)[8], const uint32_t (&s1)[8], int trb,
+                        const uint32_t (&bfr)[NT][2]) {
+#pragma unroll
+        for (int tt = 0; tt < 2; ++tt) {
+            uint32_t afr[4];
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const int k = tt * 4 + b;
+                afr[b] = prmt(t0[k], t1[k], prmt(ca, 0x54103232u, s1[k]));
+            }
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) mma_16816(acc[trb + tt][nt], afr, bfr[nt][0], bfr[nt][1]);
+        }
+    };
+    // this warp's 16 entries of GT j (TCTiles c*4 .. c*4+3, all 4 BTs): 128 contiguous bytes
+    auto table_base = [&](int t) {
+        return sbase + prm.o_tbl + t * prm.tbl_bytes + (uint32_t)(r * G) * 1024u + hioff + (uint32_t)c * 128u;
+    };
+    const bool compute = !(prm.dbg & 1);
+    // Wait for a stage's data and table; if this warp has work in it, start its pipeline.
+    auto begin_stage = [&](const StageIter &s) {
+        mbar_wait(bar_full + 8 * s.slot, s.ph);
+        if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 4);
+        mbar_wait(bar_scan + 8 * s.t, s.tph);
+        if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 5);
+        if (r < s.rows && compute) {
+            const uint32_t tb = table_base(s.t);
+            load_E(tb, 0);
+            issue(tA0, tA1, sA);
+            load_E(tb, 1);
+        }
+    };
+
     long long seg_u0 = u0;
     StageIter it;
-    for (it.init(u0, u1, KG, G, MG, S); it.valid(); it.next()) {
+    it.init(u0, u1, KG, G, MG, S);
+    if (it.valid()) begin_stage(it);
+    for (; it.valid(); it.next()) {
         const long long u = it.u;
         const int rb = it.rb, gc = it.gc, g = it.g, rows = it.rows;
         const int i = it.i, slot = it.slot, t = it.t;
@@ -350,53 +408,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
 #pragma unroll
                     for (int q = 0; q < 4; ++q) acc[a][b][q] = 0.f;
         }
-        mbar_wait(bar_full + 8 * slot, it.ph);
-        if (cw == 0 && lane == 0) trace_ev(prm, p, i, 4);
-        mbar_wait(bar_scan + 8 * t, it.tph);
-        if (cw == 0 && lane == 0) trace_ev(prm, p, i, 5);
-        if (r < rows && !(prm.dbg & 1)) {
+        StageIter nx = it;
+        nx.next();
+        if (r < rows && compute) {
             const uint32_t xs = sbase + prm.o_stage + slot * prm.stage_bytes;
-            // this warp's 16 entries of GT j (TCTiles c*4 .. c*4+3, all 4 BTs): 128 contiguous bytes
-            const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes + (uint32_t)(r * G) * 1024u + hioff +
-                                (uint32_t)c * 128u;
-            // Software pipeline over half-GT steps (8 BTs = TCTile rows 2h', 2h'+1 of GT j):
-            // while step h is assembled and multiplied, the value loads of step h+1 and the
-            // table entries of step h+2 are already in flight. Steps alternate between two
-            // register sets (A: first half of a GT, B: second half) so no copies are needed.
-            uint4 E[4];
-            uint32_t tA0[8], tA1[8], sA[8], tB0[8], tB1[8], sB[8];
-            auto load_E = [&](int step) {   // table entries of step `step` (4 x 16 B per lane)
-#pragma unroll
-                for (int q = 0; q < 4; ++q) E[q] = lds_v4(tb + (uint32_t)(step >> 1) * 1024u + (uint32_t)(step & 1) * 64u + 16u * q);
-            };
-            auto issue = [&](uint32_t (&t0)[8], uint32_t (&t1)[8], uint32_t (&s1)[8]) {   // from E
-#pragma unroll
-                for (int k = 0; k < 8; ++k) {
-                    const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
-                    const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;
-                    const uint32_t a = A + 2u * __popc(w & lm);
-                    s1[k] = ((w >> sh) & 3u) * 0x11u + c40;
-                    t0[k] = lds_u16(a);
-                    t1[k] = lds_u16(a + 2u);
-                }
-            };
-            auto assemble = [&](const uint32_t (&t0)[8], const uint32_t (&t1)[8], const uint32_t (&s1)[8], int trb,
-                                const uint32_t (&bfr)[NT][2]) {
-#pragma unroll
-                for (int tt = 0; tt < 2; ++tt) {
-                    uint32_t afr[4];
-#pragma unroll
-                    for (int b = 0; b < 4; ++b) {
-                        const int k = tt * 4 + b;
-                        afr[b] = prmt(t0[k], t1[k], prmt(ca, 0x54103232u, s1[k]));
-                    }
-#pragma unroll
-                    for (int nt = 0; nt < NT; ++nt) mma_16816(acc[trb + tt][nt], afr, bfr[nt][0], bfr[nt][1]);
-                }
-            };
-            load_E(0);
-            issue(tA0, tA1, sA);
-            load_E(1);
+            const uint32_t tb = table_base(t);
             for (int j = 0; j < g; ++j) {
                 uint32_t bfr[NT][2];
                 const uint32_t xk = xs + (xrow + (uint32_t)(64 * j + 16 * c) * cpr) * 16u;
@@ -411,15 +427,19 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
                 }
                 // step 2j: issue 2j+1 (B), prefetch entries of 2j+2, assemble 2j (A)
                 issue(tB0, tB1, sB);
-                load_E(2 * j + 2);   // past the last GT: in-bounds table/scratch bytes, never used
+                if (j + 1 < g) load_E(tb, 2 * j + 2);
                 assemble(tA0, tA1, sA, 0, bfr);
-                // step 2j+1: issue 2j+2 (A, next GT) if any, prefetch 2j+3, assemble 2j+1 (B)
+                // step 2j+1: issue the next step (A: next GT, or the next stage's first step)
                 if (j + 1 < g) {
                     issue(tA0, tA1, sA);
-                    load_E(2 * j + 3);
+                    load_E(tb, 2 * j + 3);
+                } else if (nx.valid()) {
+                    begin_stage(nx);
                 }
                 assemble(tB0, tB1, sB, 2, bfr);
             }
+        } else if (nx.valid()) {
+            begin_stage(nx);
         }
         __syncwarp();
         if (lane == 0) {
