@@ -259,9 +259,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             const StageIter &sg = it;
             const long long u = it.u;
             const int i = it.i, slot = it.slot, t = it.t;
-            mbar_wait(bar_full + 8 * slot, it.ph);
+            // suspend (not spin) while waiting: these warps have the highest scheduling
+            // priority and would otherwise steal issue slots from the consumers
+            mbar_wait_sleep(bar_full + 8 * slot, it.ph);
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 1);
-            if (i >= kTblSlots) mbar_wait(bar_tble + 8 * t, it.tph ^ 1);
+            if (i >= kTblSlots) mbar_wait_sleep(bar_tble + 8 * t, it.tph ^ 1);
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 2);
             uint2 ba[Q], bb[Q];
 #pragma unroll
