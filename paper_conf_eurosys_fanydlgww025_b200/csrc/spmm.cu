@@ -35,12 +35,19 @@ namespace spinfer {
 namespace {
 
 constexpr int kR = 2;               // GT rows per rowblock (128 output rows)
-constexpr int kCW = 8;              // consumer warps = kR rows x 4 TCTile columns
 constexpr int kScanWarps = kR;      // one scan warp per GT row of the rowblock
-constexpr int kThreads = 32 * (kCW + kScanWarps + 1);
-// Warp ids: the warp scheduler favours the highest warp id among eligible warps, so the
-// two latency-critical single-warp roles get the top ids and the consumers 0..kCW-1.
-constexpr int kScanWarp = kCW, kProducerWarp = kCW + kScanWarps;
+// Consumer layout: kR GT rows x 4 TCTile columns x KQ GT-parities (warp q of a (row,
+// column) pair takes GTs j = q, q+KQ, ... of a stage). KQ = 2 (16 consumer warps) gives
+// the scheduler enough warps to hide ALU/XU/LDS latencies; it needs the accumulators to
+// fit the tighter register budget, so N >= 24 uses KQ = 1.
+template <int NT> struct Cfg {
+    static constexpr int KQ = NT <= 2 ? 2 : 1;
+    static constexpr int CW = kR * 4 * KQ;                        // consumer warps
+    static constexpr int ScanWarp = CW;                           // warp ids: the scheduler favours the
+    static constexpr int ProducerWarp = CW + kScanWarps;          // highest id, so roles go on top
+    static constexpr int Threads = 32 * (CW + kScanWarps + 1);
+    static constexpr int ScrSlots = 2 * KQ;                       // epilogue scratch slots per GT row
+};
 constexpr int kTblSlots = 2;
 constexpr int kMaxStages = 8;
 constexpr int kMaxG = 4;            // max GroupTile columns per stage
@@ -157,8 +164,10 @@ __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const 
 }
 
 template <int NT>
-__global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
+__global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) {
     constexpr int N = NT * 8;
+    constexpr int KQ = Cfg<NT>::KQ, kCW = Cfg<NT>::CW, kThreads = Cfg<NT>::Threads;
+    constexpr int kScanWarp = Cfg<NT>::ScanWarp, kProducerWarp = Cfg<NT>::ProducerWarp;
     extern __shared__ __align__(128) uint8_t smem[];
     const uint32_t sbase = smem_u32(smem);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -212,6 +221,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             const StageIter &sg = it;
             const long long u = it.u;
             const int i = it.i, slot = it.slot;
+            if ((prm.dbg & 4) && i > 0) break;   // experiment: consumers reuse stage 0 forever
             if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, it.ph ^ 1);
             if (lane == 0) trace_ev(prm, p, i, 0);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
@@ -259,6 +269,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
             const StageIter &sg = it;
             const long long u = it.u;
             const int i = it.i, slot = it.slot, t = it.t;
+            if ((prm.dbg & 4) && i > 0) break;
             // suspend (not spin) while waiting: these warps have the highest scheduling
             // priority and would otherwise steal issue slots from the consumers
             mbar_wait_sleep(bar_full + 8 * slot, it.ph);
@@ -323,7 +334,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
     }
 
     // ---------------------------------------------------------------- consumers
-    const int cw = warp, r = cw >> 2, c = cw & 3;
+    const int cw = warp, q = cw % KQ, c = (cw / KQ) & 3, r = cw / (4 * KQ);
     const uint32_t sh = 2u * (lane & 15);
     const uint32_t lm = (1u << sh) - 1u;
     const uint32_t ca = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];       // 0x10321032
@@ -335,7 +346,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
     const uint32_t xrow = (uint32_t)(mk * 8 + rr) * cpr;   // + (64 j + 16 c) * cpr per k16 column
     const uint32_t xsw = x_swz<NT>(rr);                     // swizzle depends on k % 8 == rr only
     float acc[4][NT][4];
-    const uint32_t scr = sbase + prm.o_scr + (uint32_t)r * (2u * 64u * N * 4u);
+    constexpr uint32_t kPart = 64u * N * 4u;                      // one fp32 64 x N partial
+    const uint32_t scr = sbase + prm.o_scr + (uint32_t)r * (Cfg<NT>::ScrSlots * kPart);
 
     // Software pipeline over half-GT steps (8 BTs = TCTile rows 2h', 2h'+1 of GT j):
     // while step h is assembled and multiplied, the value loads of step h+1 and the
@@ -380,23 +392,39 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
     };
     const bool compute = !(prm.dbg & 1);
     // Wait for a stage's data and table; if this warp has work in it, start its pipeline.
+    constexpr bool kPipe = (KQ == 1);          // explicit cross-step software pipeline (8 consumer warps)
+    const bool reuse0 = (prm.dbg & 4) != 0;   // experiment: pure consumer throughput on stage 0's data
+    auto load_x = [&](uint32_t xs, int j, uint32_t (&bfr)[NT][2]) {   // B fragments of GT j, TCTile column c
+        const uint32_t xk = xs + (xrow + (uint32_t)(64 * j + 16 * c) * cpr) * 16u;
+        if constexpr (NT == 1) {
+            ldsm_x2_trans(xk, bfr[0][0], bfr[0][1]);
+        } else {
+#pragma unroll
+            for (int nt = 0; nt + 1 < NT; nt += 2)
+                ldsm_x4_trans(xk + (((uint32_t)nt + mn) ^ xsw) * 16u, bfr[nt][0], bfr[nt][1], bfr[nt + 1][0],
+                              bfr[nt + 1][1]);
+            if constexpr (NT % 2 == 1) ldsm_x2_trans(xk + (uint32_t)(NT - 1) * 16u, bfr[NT - 1][0], bfr[NT - 1][1]);
+        }
+    };
     auto begin_stage = [&](const StageIter &s) {
-        mbar_wait(bar_full + 8 * s.slot, s.ph);
-        if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 4);
-        mbar_wait(bar_scan + 8 * s.t, s.tph);
-        if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 5);
-        if (r < s.rows && compute) {
-            const uint32_t tb = table_base(s.t);
-            load_E(tb, 0);
+        if (!reuse0 || s.i == 0) {
+            mbar_wait(bar_full + 8 * s.slot, s.ph);
+            if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 4);
+            mbar_wait(bar_scan + 8 * s.t, s.tph);
+            if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 5);
+        }
+        if (kPipe && r < s.rows && compute && q < s.g) {
+            const uint32_t tb = table_base(reuse0 ? 0 : s.t);
+            load_E(tb, 2 * q);
             issue(tA0, tA1, sA);
-            load_E(tb, 1);
+            load_E(tb, 2 * q + 1);
         }
     };
 
     long long seg_u0 = u0;
     StageIter it;
     it.init(u0, u1, KG, G, MG, S);
-    if (it.valid()) begin_stage(it);
+    if (kPipe && it.valid()) begin_stage(it);
     for (; it.valid(); it.next()) {
         const long long u = it.u;
         const int rb = it.rb, gc = it.gc, g = it.g, rows = it.rows;
@@ -408,43 +436,50 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
 #pragma unroll
                 for (int b = 0; b < NT; ++b)
 #pragma unroll
-                    for (int q = 0; q < 4; ++q) acc[a][b][q] = 0.f;
+                    for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
         }
+        if constexpr (!kPipe) begin_stage(it);
         StageIter nx = it;
-        nx.next();
-        if (r < rows && compute) {
-            const uint32_t xs = sbase + prm.o_stage + slot * prm.stage_bytes;
-            const uint32_t tb = table_base(t);
-            for (int j = 0; j < g; ++j) {
+        if constexpr (kPipe) nx.next();
+        if (r < rows && compute && q < g && !kPipe) {
+            // KQ = 2: 4 consumer warps per scheduler hide the latencies; one register set.
+            const uint32_t xs = sbase + prm.o_stage + (reuse0 ? 0 : slot) * prm.stage_bytes;
+            const uint32_t tb = table_base(reuse0 ? 0 : t);
+            for (int j = q; j < g; j += KQ) {
                 uint32_t bfr[NT][2];
-                const uint32_t xk = xs + (xrow + (uint32_t)(64 * j + 16 * c) * cpr) * 16u;
-                if constexpr (NT == 1) {
-                    ldsm_x2_trans(xk, bfr[0][0], bfr[0][1]);
-                } else {
+                load_x(xs, j, bfr);
 #pragma unroll
-                    for (int nt = 0; nt + 1 < NT; nt += 2)
-                        ldsm_x4_trans(xk + (((uint32_t)nt + mn) ^ xsw) * 16u, bfr[nt][0], bfr[nt][1], bfr[nt + 1][0],
-                                      bfr[nt + 1][1]);
-                    if constexpr (NT % 2 == 1) ldsm_x2_trans(xk + (uint32_t)(NT - 1) * 16u, bfr[NT - 1][0], bfr[NT - 1][1]);
-                }
-                // step 2j: issue 2j+1 (B), prefetch entries of 2j+2, assemble 2j (A)
-                issue(tB0, tB1, sB);
-                if (j + 1 < g) load_E(tb, 2 * j + 2);
-                assemble(tA0, tA1, sA, 0, bfr);
-                // step 2j+1: issue the next step (A: next GT, or the next stage's first step)
-                if (j + 1 < g) {
+                for (int h = 0; h < 2; ++h) {
+                    load_E(tb, 2 * j + h);
                     issue(tA0, tA1, sA);
-                    load_E(tb, 2 * j + 3);
+                    assemble(tA0, tA1, sA, 2 * h, bfr);
+                }
+            }
+        } else if (r < rows && compute && q < g) {
+            const uint32_t xs = sbase + prm.o_stage + (reuse0 ? 0 : slot) * prm.stage_bytes;
+            const uint32_t tb = table_base(reuse0 ? 0 : t);
+            for (int j = q; j < g; j += KQ) {
+                uint32_t bfr[NT][2];
+                load_x(xs, j, bfr);
+                // step (j, first half): issue (j, second half) into B, prefetch the entries of
+                // this warp's next GT, assemble (j, first half) from A
+                issue(tB0, tB1, sB);
+                if (j + KQ < g) load_E(tb, 2 * (j + KQ));
+                assemble(tA0, tA1, sA, 0, bfr);
+                // step (j, second half): issue the next step (A: next GT, or the next stage's first step)
+                if (j + KQ < g) {
+                    issue(tA0, tA1, sA);
+                    load_E(tb, 2 * (j + KQ) + 1);
                 } else if (nx.valid()) {
                     begin_stage(nx);
                 }
                 assemble(tB0, tB1, sB, 2, bfr);
             }
-        } else if (nx.valid()) {
+        } else if (kPipe && nx.valid()) {
             begin_stage(nx);
         }
         __syncwarp();
-        if (lane == 0) {
+        if (lane == 0 && !reuse0) {
             mbar_arrive(bar_empty + 8 * slot);
             mbar_arrive(bar_tble + 8 * t);
             if (cw == 0) trace_ev(prm, p, i, 6);
@@ -453,48 +488,41 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Params prm) {
         const bool seg_end = (gc + g == KG) || (u_end == u1);
         if (seg_end && r < rows) {
             // -------------------------------------------------------- epilogue
-            // (1) reduce the 4 TCTile-column partials of GT row r (tree via smem)
-            const uint32_t bid = 1u + (uint32_t)r;
-            if (c >= 2) {
+            // (1) reduce the 4*KQ partials of GT row r into warp (c = 0, q = 0), tree via smem
+            const uint32_t bid = 1u + (uint32_t)r, bcnt = 128u * KQ;
+            auto put = [&](uint32_t slot_) {
 #pragma unroll
                 for (int tr = 0; tr < 4; ++tr)
 #pragma unroll
                     for (int nt = 0; nt < NT; ++nt)
-                        sts_f4(scr + (uint32_t)(c - 2) * (64u * N * 4u) + (uint32_t)((tr * NT + nt) * 32 + lane) * 16u,
+                        sts_f4(scr + slot_ * kPart + (uint32_t)((tr * NT + nt) * 32 + lane) * 16u,
                                make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]));
-            }
-            named_bar_sync(bid, 128);
-            if (c < 2) {
+            };
+            auto add = [&](uint32_t slot_) {
 #pragma unroll
                 for (int tr = 0; tr < 4; ++tr)
 #pragma unroll
                     for (int nt = 0; nt < NT; ++nt) {
-                        float4 v = lds_f4(scr + (uint32_t)c * (64u * N * 4u) + (uint32_t)((tr * NT + nt) * 32 + lane) * 16u);
+                        float4 v = lds_f4(scr + slot_ * kPart + (uint32_t)((tr * NT + nt) * 32 + lane) * 16u);
                         acc[tr][nt][0] += v.x; acc[tr][nt][1] += v.y; acc[tr][nt][2] += v.z; acc[tr][nt][3] += v.w;
                     }
+            };
+            if constexpr (KQ == 2) {          // GT parities: q = 1 -> q = 0
+                if (q == 1) put((uint32_t)c);
+                named_bar_sync(bid, bcnt);
+                if (q == 0) add((uint32_t)c);
+                named_bar_sync(bid, bcnt);
             }
-            named_bar_sync(bid, 128);
-            if (c == 1) {
-#pragma unroll
-                for (int tr = 0; tr < 4; ++tr)
-#pragma unroll
-                    for (int nt = 0; nt < NT; ++nt)
-                        sts_f4(scr + (uint32_t)((tr * NT + nt) * 32 + lane) * 16u,
-                               make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]));
-            }
-            named_bar_sync(bid, 128);
-            if (c == 0) {
-#pragma unroll
-                for (int tr = 0; tr < 4; ++tr)
-#pragma unroll
-                    for (int nt = 0; nt < NT; ++nt) {
-                        float4 v = lds_f4(scr + (uint32_t)((tr * NT + nt) * 32 + lane) * 16u);
-                        acc[tr][nt][0] += v.x; acc[tr][nt][1] += v.y; acc[tr][nt][2] += v.z; acc[tr][nt][3] += v.w;
-                    }
-            }
-            named_bar_sync(bid, 128);
+            if (q == 0 && c >= 2) put((uint32_t)(c - 2));     // TCTile columns: 4 -> 2 -> 1
+            named_bar_sync(bid, bcnt);
+            if (q == 0 && c < 2) add((uint32_t)c);
+            named_bar_sync(bid, bcnt);
+            if (q == 0 && c == 1) put(0u);
+            named_bar_sync(bid, bcnt);
+            if (q == 0 && c == 0) add(0u);
+            named_bar_sync(bid, bcnt);
             // (2) write Y, or combine split rowblocks across CTAs (split-K fix-up)
-            if (c == 0) {
+            if (c == 0 && q == 0) {
                 const int grow = kR * rb + r;
                 const int row_base = grow * 64;
                 const bool complete = (seg_u0 == (long long)rb * KG) && (u_end == (long long)(rb + 1) * KG);
@@ -589,7 +617,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
     if (const char *e = getenv("SPINFER_S")) smax = std::max(2, std::min(kMaxStages, atoi(e)));
     for (int G = gmax; G >= 1; --G) {
         uint32_t tbl = (uint32_t)kR * G * 64 * 16;
-        uint32_t scr = (uint32_t)kR * 2 * 64 * N * 4;
+        uint32_t scr = (uint32_t)kR * (N <= 16 ? 4 : 2) * 64 * N * 4;   // Cfg<NT>::ScrSlots partial slots per row
         uint32_t st_bm = (uint32_t)G * 64 * N * 2;            // X slab first, then bitmaps
         uint32_t st_v0 = st_bm + (uint32_t)kR * G * 512;
         uint32_t vcap = align_up((uint32_t)G * maxv * 2, 16);
@@ -626,7 +654,7 @@ int launch_nt(const Plan &pl, cudaStream_t st) {
             return SPINFER_ECUDA;
         configured_smem[dev] = (int)pl.smem;
     }
-    k_spmm<NT><<<pl.P, kThreads, pl.smem, st>>>(pl.prm);
+    k_spmm<NT><<<pl.P, Cfg<NT>::Threads, pl.smem, st>>>(pl.prm);
     return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
 }
 
