@@ -478,6 +478,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         } else if (kPipe && nx.valid()) {
             begin_stage(nx);
         }
+        if (cw == 0 && lane == 0) trace_ev(prm, p, i, 7);   // consumer warp 0 finished the stage's work
         __syncwarp();
         if (lane == 0 && !reuse0) {
             mbar_arrive(bar_empty + 8 * slot);

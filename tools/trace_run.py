@@ -14,8 +14,8 @@ sp.spmm(T, Xd); torch.cuda.synchronize()
 tr = np.fromfile(path, dtype=np.int64).reshape(4, 64, 8)
 for p in range(2):
     t0 = tr[p, 0, 0]
-    print(f"CTA {p}: columns = prod_issue | scan_full | scan_tbl | scan_done | cons_full | cons_scan | cons_rel  (cycles from first issue)")
+    print(f"CTA {p}: columns = prod_issue | scan_full | scan_tbl | scan_done | cons_full | cons_scan | cons_rel | cons_done (cycles from first issue)")
     for i in range(0, 50):
-        row = tr[p, i, :7]
-        if row[0] == 0 and i > 0: break
+        row = tr[p, i, :8]
+        if row[0] == 0 and row[7] == 0 and i > 0: break
         print(i, " ".join(f"{(v - t0) if v else -1:8d}" for v in row))
