@@ -141,12 +141,15 @@ __device__ __forceinline__ uint32_t x_swz(uint32_t k) {
 //   t0 = V[count], t1 = V[count+1]                 (zero-extended u16 loads)
 //   a0 = bit(sh)   ? t0 : 0                        (Phase I)
 //   a1 = bit(sh+1) ? (bit(sh) ? t1 : t0) : 0       (Phase II reuses count)
-// The four (bit(sh), bit(sh+1)) cases are one PRMT of {t0, t1} whose selector is
-// looked up by a second PRMT from y = (w >> sh) & 3; zero halves select the u16
-// loads' zero upper bytes. Selector table (nibbles = source bytes, low half first):
-//   y=0 -> 0x3232 (0,0)   y=1 -> 0x3210 (t0,0)   y=2 -> 0x1032 (0,t0)   y=3 -> 0x5410 (t0,t1)
-// low selector byte  = byte y of 0x10321032, high byte = byte y of 0x54103232,
-// so sel = prmt(0x10321032, 0x54103232, y*0x11 + 0x40).
+// The four (bit(sh), bit(sh+1)) cases are one PRMT of {t0, t1} whose selector depends
+// on y = (w >> sh) & 3; zero halves select the u16 loads' zero upper bytes (byte 2/3 of
+// t0, 6/7 of t1, optionally in sign-replicate mode, which also yields 0x00):
+//   y=0 -> (0,0)  y=1 -> (t0,0)  y=2 -> (0,t0)  y=3 -> (t0,t1)
+// The selector is the quadratic sel(y) = y*(kSelA + kSelB*y) + kSelC (mod 2^16), found by
+// exhaustive search (tools/selector_search.py; pinned in tests/test_host_logic.py):
+//   sel(0)=0x2333 sel(1)=0xab10 sel(2)=0x10af sel(3)=0x5410
+// — two IMADs on the FMA pipe instead of ALU-pipe work (the ALU pipe is half rate on B200).
+constexpr uint32_t kSelA = 0x18fcu, kSelB = 0x6ee1u, kSelC = 0x2333u;
 
 template <int NT>
 __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const float (&acc)[4][NT][4], int lane) {
@@ -193,8 +196,9 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         fence_barrier_init();
         // SMBD selector-table constants, read back into registers by every consumer thread so
         // ptxas keeps them live in registers instead of re-materialising them per PRMT.
-        reinterpret_cast<uint32_t *>(smem)[kConstWord] = 0x10321032u;
-        reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = 0x40u;
+        reinterpret_cast<uint32_t *>(smem)[kConstWord] = kSelA;
+        reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = kSelB;
+        reinterpret_cast<uint32_t *>(smem)[kConstWord + 2] = kSelC;
     }
     // Preload this CTA's GTileOffset entries: pre[u-u0] = {start_r0, end_r0, start_r1, end_r1}.
     for (long long i = threadIdx.x; i < u1 - u0; i += kThreads) {
@@ -337,8 +341,11 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
     const int cw = warp, q = cw % KQ, c = (cw / KQ) & 3, r = cw / (4 * KQ);
     const uint32_t sh = 2u * (lane & 15);
     const uint32_t lm = (1u << sh) - 1u;
-    const uint32_t ca = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];       // 0x10321032
-    const uint32_t c40 = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];  // 0x40
+    const uint32_t mulc = sh ? (1u << (32u - sh)) : 0u;     // w * mulc == w << (32 - sh), 0 for sh = 0
+    // selector polynomial constants, read from smem so ptxas keeps them in registers
+    const uint32_t selA = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];
+    const uint32_t selB = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];
+    const uint32_t selC = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 2];
     const uint32_t hioff = (uint32_t)(lane >> 4) * 512u;
     // ldmatrix.trans rows: matrix m = lane/8 -> (k half m&1, n chunk m>>1); row rr = lane%8.
     constexpr uint32_t cpr = N / 8;
@@ -366,8 +373,12 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         for (int k = 0; k < 8; ++k) {
             const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
             const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;
-            const uint32_t a = A + 2u * __popc(w & lm);
-            s1[k] = ((w >> sh) & 3u) * 0x11u + c40;
+            // MaskedPopCount: popc(w & ((1 << sh) - 1)) == popc(w << (32 - sh)), the shift done
+            // as a multiply (FMA pipe) because the ALU pipe is the scarce one (half rate)
+            const uint32_t a = A + 2u * __popc(w * mulc);
+            // selector = y*(kSelA + kSelB*y) + kSelC: two IMADs instead of a PRMT table lookup
+            const uint32_t y = (w >> sh) & 3u;
+            s1[k] = y * (y * selB + selA) + selC;
             t0[k] = lds_u16(a);
             t1[k] = lds_u16(a + 2u);
         }
@@ -380,7 +391,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
 #pragma unroll
             for (int b = 0; b < 4; ++b) {
                 const int k = tt * 4 + b;
-                afr[b] = prmt(t0[k], t1[k], prmt(ca, 0x54103232u, s1[k]));
+                afr[b] = prmt(t0[k], t1[k], s1[k]);
             }
 #pragma unroll
             for (int nt = 0; nt < NT; ++nt) mma_16816(acc[trb + tt][nt], afr, bfr[nt][0], bfr[nt][1]);
