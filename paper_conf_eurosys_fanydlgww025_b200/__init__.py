@@ -18,7 +18,7 @@ __all__ = ["TCA", "SpinferError", "encode", "decode", "spmm", "spmm_tp", "tp_row
            "workspace_bytes", "storage_bytes", "algorithmic_bytes", "lib", "LIB_PATH"]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libspinfer.so")
+LIB_PATH = os.environ.get("SPINFER_LIB") or os.path.join(_PKG, "libspinfer.so")   # SPINFER_LIB: experiments only
 GT = 64
 
 _STATUS = {0: "SPINFER_OK", -1: "SPINFER_EINVAL", -2: "SPINFER_ENOSPC", -3: "SPINFER_EOVERFLOW",

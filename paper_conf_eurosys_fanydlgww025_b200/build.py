@@ -34,17 +34,22 @@ def up_to_date() -> bool:
     return all(os.path.getmtime(d) <= t for d in deps())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and up_to_date():
+LIB_INSTR = os.path.join(PKG, "libspinfer_instr.so")   # experiments only (stage trace, debug modes)
+
+
+def build(force: bool = False, verbose: bool = False, instrumented: bool = False) -> str:
+    out = LIB_INSTR if instrumented else LIB
+    if not force and not instrumented and up_to_date():
         return LIB
-    cmd = [NVCC, *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), *sources(), "-o", LIB + ".tmp"]
+    cmd = [NVCC, *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), *sources(), "-o", out + ".tmp"]
+    if instrumented:
+        cmd.append("-DSPINFER_INSTRUMENT=1")
     if verbose:
         cmd[1:1] = ["-Xptxas", "-v"]
     subprocess.check_call(cmd)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(out + ".tmp", out)
+    return out
 
 
 if __name__ == "__main__":
-    build(force=True, verbose="-v" in sys.argv)
-    print(LIB)
+    print(build(force=True, verbose="-v" in sys.argv, instrumented="--instrumented" in sys.argv))

@@ -52,7 +52,7 @@ constexpr int kTblSlots = 2;
 constexpr int kMaxStages = 8;
 constexpr int kMaxG = 4;            // max GroupTile columns per stage
 constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector-table constants
-constexpr int kTraceCTAs = 4, kTraceStages = 64;
+constexpr int kTraceCTAs = 4, kTraceStages = 64, kTraceEv = 16;
 // Workspace = [fix-up counters: one int32 per GT row, fixed-size region][split-K partials].
 // The counter region has the same size for every shape so that one zeroed
 // workspace can serve calls of different shapes (partials never overlap counters).
@@ -78,8 +78,22 @@ struct Params {
     int dbg;            // experiments only (SPINFER_DEBUG_MODE): bit0 = consumers skip decode/MMA, bit1 = scan skips work
 };
 
+// Experiment instrumentation (stage timeline, debug modes) is compiled in only with
+// -DSPINFER_INSTRUMENT=1 (tools/build_instrumented.sh); the product build has none of it.
+#ifndef SPINFER_INSTRUMENT
+#define SPINFER_INSTRUMENT 0
+#endif
 __device__ __forceinline__ void trace_ev(const Params &prm, int p, int i, int ev) {
-    if (prm.trace && p < kTraceCTAs && i < kTraceStages) prm.trace[((size_t)p * kTraceStages + i) * 8 + ev] = clock64();
+#if SPINFER_INSTRUMENT
+    if (prm.trace && p < kTraceCTAs && i < kTraceStages) prm.trace[((size_t)p * kTraceStages + i) * kTraceEv + ev] = clock64();
+#endif
+}
+__device__ __forceinline__ int dbg_mode(const Params &prm) {
+#if SPINFER_INSTRUMENT
+    return prm.dbg;
+#else
+    return 0;
+#endif
 }
 
 __device__ __forceinline__ long long unit_start(long long p, long long U, int P) { return p * U / P; }
@@ -88,37 +102,40 @@ __device__ __forceinline__ int unit_owner(long long u, long long U, int P) {
 }
 
 // Stage iterator: every role walks the same deterministic stage sequence. All
-// per-stage bookkeeping is incremental (one 64-bit division at kernel start only):
-// ring slot / parity of the S-stage smem ring and of the 2-slot table ring.
+// per-stage bookkeeping is incremental and 32-bit (one 64-bit division at kernel start
+// only); loop-invariant sizes stay in the parameter bank, so the live state is a few
+// registers (16 consumer warps run at <= 96 registers; spills would go to L2 because the
+// shared-memory carve-out leaves almost no L1).
 struct StageIter {
-    long long u, u1;
-    int KG, G, MG, S;
+    int du, du1;             // current unit offset from u0, and the CTA's unit count
     int rb, gc, g, rows;     // current stage: rowblock, first GT column, #units, #GT rows
-    int i;                   // stage index within the CTA
-    int slot, ph;            // smem ring slot and its phase parity ((i / S) & 1)
-    int t, tph;              // table slot (i & 1) and its parity ((i / 2) & 1)
-    __device__ __forceinline__ void init(long long u0_, long long u1_, int KG_, int G_, int MG_, int S_) {
-        u = u0_; u1 = u1_; KG = KG_; G = G_; MG = MG_; S = S_;
-        rb = (int)(u / KG);
-        gc = (int)(u - (long long)rb * KG);
-        i = 0; slot = 0; ph = 0; t = 0; tph = 0;
-        shape();
+    int i, slot;             // stage index within the CTA, smem ring slot
+    uint32_t ph;             // bit0: ring parity ((i / S) & 1), bit1: table slot (i & 1), bit2: its parity
+    __device__ __forceinline__ void init(long long u0, long long u1, const Params &prm) {
+        du = 0;
+        du1 = (int)(u1 - u0);
+        rb = (int)(u0 / prm.KG);
+        gc = (int)(u0 - (long long)rb * prm.KG);
+        i = 0; slot = 0; ph = 0;
+        shape(prm);
     }
-    __device__ __forceinline__ void shape() {
-        g = min(G, KG - gc);
-        if ((long long)g > u1 - u) g = (int)(u1 - u);
-        rows = min(kR, MG - kR * rb);
+    __device__ __forceinline__ void shape(const Params &prm) {
+        g = min(min(prm.G, prm.KG - gc), du1 - du);
+        rows = min(kR, prm.MG - kR * rb);
     }
-    __device__ __forceinline__ bool valid() const { return u < u1; }
-    __device__ __forceinline__ void next() {
-        u += g;
+    __device__ __forceinline__ bool valid() const { return du < du1; }
+    __device__ __forceinline__ int t() const { return (ph >> 1) & 1; }
+    __device__ __forceinline__ uint32_t par() const { return ph & 1; }
+    __device__ __forceinline__ uint32_t tpar() const { return (ph >> 2) & 1; }
+    __device__ __forceinline__ void next(const Params &prm) {
+        du += g;
         gc += g;
-        if (gc == KG) { gc = 0; ++rb; }
+        if (gc == prm.KG) { gc = 0; ++rb; }
         ++i;
-        if (++slot == S) { slot = 0; ph ^= 1; }
-        t ^= 1;
-        if (t == 0) tph ^= 1;
-        shape();
+        if (++slot == prm.S) { slot = 0; ph ^= 1u; }
+        ph ^= 2u;
+        if (!(ph & 2u)) ph ^= 4u;
+        shape(prm);
     }
 };
 
@@ -221,12 +238,12 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         const uint64_t pol_w = policy_evict_first();
         constexpr int cpr = N / 8;                     // 16-byte chunks per X row
         StageIter it;
-        for (it.init(u0, u1, KG, G, MG, S); it.valid(); it.next()) {
+        for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
             const StageIter &sg = it;
-            const long long u = it.u;
+            const long long u = u0 + it.du;
             const int i = it.i, slot = it.slot;
-            if ((prm.dbg & 4) && i > 0) break;   // experiment: consumers reuse stage 0 forever
-            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, it.ph ^ 1);
+            if ((dbg_mode(prm) & 4) && i > 0) break;   // experiment: consumers reuse stage 0 forever
+            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, it.par() ^ 1u);
             if (lane == 0) trace_ev(prm, p, i, 0);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const uint32_t fb = bar_full + 8 * slot;
@@ -267,18 +284,18 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         // independent shuffle chains interleave.
         constexpr int Q = kMaxG;
         const int r = warp - kScanWarp;               // this scan warp's GT row
-        const bool work = !(prm.dbg & 2);
+        const bool work = !(dbg_mode(prm) & 2);
         StageIter it;
-        for (it.init(u0, u1, KG, G, MG, S); it.valid(); it.next()) {
+        for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
             const StageIter &sg = it;
-            const long long u = it.u;
-            const int i = it.i, slot = it.slot, t = it.t;
-            if ((prm.dbg & 4) && i > 0) break;
+            const long long u = u0 + it.du;
+            const int i = it.i, slot = it.slot, t = it.t();
+            if ((dbg_mode(prm) & 4) && i > 0) break;
             // suspend (not spin) while waiting: these warps have the highest scheduling
             // priority and would otherwise steal issue slots from the consumers
-            mbar_wait_sleep(bar_full + 8 * slot, it.ph);
+            mbar_wait_sleep(bar_full + 8 * slot, it.par());
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 1);
-            if (i >= kTblSlots) mbar_wait_sleep(bar_tble + 8 * t, it.tph ^ 1);
+            if (i >= kTblSlots) mbar_wait_sleep(bar_tble + 8 * t, it.tpar() ^ 1u);
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 2);
             uint2 ba[Q], bb[Q];
 #pragma unroll
@@ -340,7 +357,6 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
     // ---------------------------------------------------------------- consumers
     const int cw = warp, q = cw % KQ, c = (cw / KQ) & 3, r = cw / (4 * KQ);
     const uint32_t sh = 2u * (lane & 15);
-    const uint32_t lm = (1u << sh) - 1u;
     const uint32_t mulc = sh ? (1u << (32u - sh)) : 0u;     // w * mulc == w << (32 - sh), 0 for sh = 0
     // selector polynomial constants, read from smem so ptxas keeps them in registers
     const uint32_t selA = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];
@@ -401,10 +417,10 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
     auto table_base = [&](int t) {
         return sbase + prm.o_tbl + t * prm.tbl_bytes + (uint32_t)(r * G) * 1024u + hioff + (uint32_t)c * 128u;
     };
-    const bool compute = !(prm.dbg & 1);
+    const bool compute = !(dbg_mode(prm) & 1);
     // Wait for a stage's data and table; if this warp has work in it, start its pipeline.
     constexpr bool kPipe = (KQ == 1);          // explicit cross-step software pipeline (8 consumer warps)
-    const bool reuse0 = (prm.dbg & 4) != 0;   // experiment: pure consumer throughput on stage 0's data
+    const bool reuse0 = (dbg_mode(prm) & 4) != 0;   // experiment: pure consumer throughput on stage 0's data
     auto load_x = [&](uint32_t xs, int j, uint32_t (&bfr)[NT][2]) {   // B fragments of GT j, TCTile column c
         const uint32_t xk = xs + (xrow + (uint32_t)(64 * j + 16 * c) * cpr) * 16u;
         if constexpr (NT == 1) {
@@ -419,29 +435,28 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
     };
     auto begin_stage = [&](const StageIter &s) {
         if (!reuse0 || s.i == 0) {
-            mbar_wait(bar_full + 8 * s.slot, s.ph);
+            mbar_wait(bar_full + 8 * s.slot, s.par());
             if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 4);
-            mbar_wait(bar_scan + 8 * s.t, s.tph);
+            mbar_wait(bar_scan + 8 * s.t(), s.tpar());
             if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 5);
         }
         if (kPipe && r < s.rows && compute && q < s.g) {
-            const uint32_t tb = table_base(reuse0 ? 0 : s.t);
+            const uint32_t tb = table_base(reuse0 ? 0 : s.t());
             load_E(tb, 2 * q);
             issue(tA0, tA1, sA);
             load_E(tb, 2 * q + 1);
         }
     };
 
-    long long seg_u0 = u0;
+    bool seg_full_start = false;      // current rowblock segment started at the rowblock's first unit
     StageIter it;
-    it.init(u0, u1, KG, G, MG, S);
+    it.init(u0, u1, prm);
     if (kPipe && it.valid()) begin_stage(it);
-    for (; it.valid(); it.next()) {
-        const long long u = it.u;
+    for (; it.valid(); it.next(prm)) {
         const int rb = it.rb, gc = it.gc, g = it.g, rows = it.rows;
-        const int i = it.i, slot = it.slot, t = it.t;
-        if (gc == 0 || u == u0) {
-            seg_u0 = u;
+        const int i = it.i, slot = it.slot, t = it.t();
+        if (gc == 0 || it.du == 0) {
+            seg_full_start = (gc == 0);
 #pragma unroll
             for (int a = 0; a < 4; ++a)
 #pragma unroll
@@ -451,12 +466,13 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         }
         if constexpr (!kPipe) begin_stage(it);
         StageIter nx = it;
-        if constexpr (kPipe) nx.next();
+        if constexpr (kPipe) nx.next(prm);
         if (r < rows && compute && q < g && !kPipe) {
             // KQ = 2: 4 consumer warps per scheduler hide the latencies; one register set.
             const uint32_t xs = sbase + prm.o_stage + (reuse0 ? 0 : slot) * prm.stage_bytes;
             const uint32_t tb = table_base(reuse0 ? 0 : t);
             for (int j = q; j < g; j += KQ) {
+                if (cw == 0 && lane == 0) trace_ev(prm, p, i, 8 + j);
                 uint32_t bfr[NT][2];
                 load_x(xs, j, bfr);
 #pragma unroll
@@ -496,8 +512,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
             mbar_arrive(bar_tble + 8 * t);
             if (cw == 0) trace_ev(prm, p, i, 6);
         }
-        const long long u_end = u + g;
-        const bool seg_end = (gc + g == KG) || (u_end == u1);
+        const bool seg_end = (gc + g == KG) || (it.du + g == it.du1);
         if (seg_end && r < rows) {
             // -------------------------------------------------------- epilogue
             // (1) reduce the 4*KQ partials of GT row r into warp (c = 0, q = 0), tree via smem
@@ -537,7 +552,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
             if (c == 0 && q == 0) {
                 const int grow = kR * rb + r;
                 const int row_base = grow * 64;
-                const bool complete = (seg_u0 == (long long)rb * KG) && (u_end == (long long)(rb + 1) * KG);
+                const bool complete = seg_full_start && (gc + g == KG);
                 if (complete) {
                     store_y<NT>(prm.Y, N, row_base, acc, lane);
                 } else {
@@ -701,7 +716,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     q.trace = nullptr;
     static long long *trace_buf = nullptr;
     const char *trace_path = getenv("SPINFER_TRACE");
-    const size_t trace_n = (size_t)kTraceCTAs * kTraceStages * 8;
+    const size_t trace_n = (size_t)kTraceCTAs * kTraceStages * kTraceEv;
     if (trace_path) {
         if (!trace_buf && cudaMalloc(&trace_buf, trace_n * 8) != cudaSuccess) return SPINFER_ECUDA;
         cudaMemsetAsync(trace_buf, 0, trace_n * 8, st);
@@ -716,7 +731,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
         default: break;
     }
     if (trace_path && rc == SPINFER_OK) {   // debug only: synchronous dump of the stage timeline
-        static long long host[kTraceCTAs * kTraceStages * 8];
+        static long long host[kTraceCTAs * kTraceStages * kTraceEv];
         cudaMemcpyAsync(host, trace_buf, sizeof(host), cudaMemcpyDeviceToHost, st);
         cudaStreamSynchronize(st);
         if (FILE *f = fopen(trace_path, "wb")) { fwrite(host, 1, sizeof(host), f); fclose(f); }
