@@ -435,9 +435,11 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
     };
     auto begin_stage = [&](const StageIter &s) {
         if (!reuse0 || s.i == 0) {
-            mbar_wait(bar_full + 8 * s.slot, s.par());
+            // suspend rather than spin: a spinning consumer steals issue slots from the
+            // other 15 consumer warps that still have decode work
+            mbar_wait_sleep(bar_full + 8 * s.slot, s.par());
             if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 4);
-            mbar_wait(bar_scan + 8 * s.t(), s.tpar());
+            mbar_wait_sleep(bar_scan + 8 * s.t(), s.tpar());
             if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 5);
         }
         if (kPipe && r < s.rows && compute && q < s.g) {
