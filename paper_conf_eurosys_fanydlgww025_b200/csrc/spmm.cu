@@ -48,7 +48,6 @@ template <int NT> struct Cfg {
     static constexpr int Threads = 32 * (CW + kScanWarps + 1);
     static constexpr int ScrSlots = 2 * KQ;                       // epilogue scratch slots per GT row
 };
-constexpr int kTblSlots = 2;
 constexpr int kMaxStages = 8;
 constexpr int kMaxG = 4;            // max GroupTile columns per stage
 constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector-table constants
@@ -110,7 +109,7 @@ struct StageIter {
     int du, du1;             // current unit offset from u0, and the CTA's unit count
     int rb, gc, g, rows;     // current stage: rowblock, first GT column, #units, #GT rows
     int i, slot;             // stage index within the CTA, smem ring slot
-    uint32_t ph;             // bit0: ring parity ((i / S) & 1), bit1: table slot (i & 1), bit2: its parity
+    uint32_t ph;             // ring parity ((i / S) & 1)
     __device__ __forceinline__ void init(long long u0, long long u1, const Params &prm) {
         du = 0;
         du1 = (int)(u1 - u0);
@@ -124,17 +123,13 @@ struct StageIter {
         rows = min(kR, prm.MG - kR * rb);
     }
     __device__ __forceinline__ bool valid() const { return du < du1; }
-    __device__ __forceinline__ int t() const { return (ph >> 1) & 1; }
-    __device__ __forceinline__ uint32_t par() const { return ph & 1; }
-    __device__ __forceinline__ uint32_t tpar() const { return (ph >> 2) & 1; }
+    __device__ __forceinline__ uint32_t par() const { return ph; }
     __device__ __forceinline__ void next(const Params &prm) {
         du += g;
         gc += g;
         if (gc == prm.KG) { gc = 0; ++rb; }
         ++i;
         if (++slot == prm.S) { slot = 0; ph ^= 1u; }
-        ph ^= 2u;
-        if (!(ph & 2u)) ph ^= 4u;
         shape(prm);
     }
 };
@@ -198,7 +193,9 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
 
     // barriers: full[S], empty[S], scanned[2], tbl_empty[2]
     const uint32_t bar_full = sbase, bar_empty = sbase + 8 * kMaxStages;
-    const uint32_t bar_scan = sbase + 16 * kMaxStages, bar_tble = bar_scan + 8 * kTblSlots;
+    // barriers: full[S] (data landed), empty[S] (consumers done), scanned[S] (table written;
+    // the scan warps acquired full[s] first, so consumers wait on scanned[s] only)
+    const uint32_t bar_scan = sbase + 16 * kMaxStages;
     int4 *pre = reinterpret_cast<int4 *>(smem + prm.o_pre);
 
     if (threadIdx.x == 0) {
@@ -206,10 +203,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
             mbar_init(bar_full + 8 * s, 32);      // the 32 producer lanes (+ TMA transaction bytes)
             mbar_init(bar_empty + 8 * s, kCW);
         }
-        for (int t = 0; t < kTblSlots; ++t) {
-            mbar_init(bar_scan + 8 * t, 32 * kScanWarps);
-            mbar_init(bar_tble + 8 * t, kCW);
-        }
+        for (int s = 0; s < S; ++s) mbar_init(bar_scan + 8 * s, 32 * kScanWarps);
         fence_barrier_init();
         // SMBD selector-table constants, read back into registers by every consumer thread so
         // ptxas keeps them live in registers instead of re-materialising them per PRMT.
@@ -289,13 +283,12 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
             const StageIter &sg = it;
             const long long u = u0 + it.du;
-            const int i = it.i, slot = it.slot, t = it.t();
+            const int i = it.i, slot = it.slot;
             if ((dbg_mode(prm) & 4) && i > 0) break;
             // suspend (not spin) while waiting: these warps have the highest scheduling
             // priority and would otherwise steal issue slots from the consumers
             mbar_wait_sleep(bar_full + 8 * slot, it.par());
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 1);
-            if (i >= kTblSlots) mbar_wait_sleep(bar_tble + 8 * t, it.tpar() ^ 1u);
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 2);
             uint2 ba[Q], bb[Q];
 #pragma unroll
@@ -311,7 +304,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
                 }
             }
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
-            const uint32_t tb = sbase + prm.o_tbl + t * prm.tbl_bytes;
+            const uint32_t tb = sbase + prm.o_tbl + slot * prm.tbl_bytes;   // one table per ring slot
             uint32_t packed[Q], incl[Q];
 #pragma unroll
             for (int q = 0; q < Q; ++q) {
@@ -348,7 +341,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
                     sts_v2(te + 768u, bb[q].y, Ab + 2u * __popc(bb[q].x));
                 }
             }
-            mbar_arrive(bar_scan + 8 * t);
+            mbar_arrive(bar_scan + 8 * slot);
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 3);
         }
         return;
@@ -414,8 +407,8 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         }
     };
     // this warp's 16 entries of GT j (TCTiles c*4 .. c*4+3, all 4 BTs): 128 contiguous bytes
-    auto table_base = [&](int t) {
-        return sbase + prm.o_tbl + t * prm.tbl_bytes + (uint32_t)(r * G) * 1024u + hioff + (uint32_t)c * 128u;
+    auto table_base = [&](int slot_) {
+        return sbase + prm.o_tbl + slot_ * prm.tbl_bytes + (uint32_t)(r * G) * 1024u + hioff + (uint32_t)c * 128u;
     };
     const bool compute = !(dbg_mode(prm) & 1);
     // Wait for a stage's data and table; if this warp has work in it, start its pipeline.
@@ -437,13 +430,12 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         if (!reuse0 || s.i == 0) {
             // suspend rather than spin: a spinning consumer steals issue slots from the
             // other 15 consumer warps that still have decode work
-            mbar_wait_sleep(bar_full + 8 * s.slot, s.par());
+            mbar_wait_sleep(bar_scan + 8 * s.slot, s.par());   // implies full[s.slot] (see above)
             if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 4);
-            mbar_wait_sleep(bar_scan + 8 * s.t(), s.tpar());
             if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 5);
         }
         if (kPipe && r < s.rows && compute && q < s.g) {
-            const uint32_t tb = table_base(reuse0 ? 0 : s.t());
+            const uint32_t tb = table_base(reuse0 ? 0 : s.slot);
             load_E(tb, 2 * q);
             issue(tA0, tA1, sA);
             load_E(tb, 2 * q + 1);
@@ -456,7 +448,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
     if (kPipe && it.valid()) begin_stage(it);
     for (; it.valid(); it.next(prm)) {
         const int rb = it.rb, gc = it.gc, g = it.g, rows = it.rows;
-        const int i = it.i, slot = it.slot, t = it.t();
+        const int i = it.i, slot = it.slot;
         if (gc == 0 || it.du == 0) {
             seg_full_start = (gc == 0);
 #pragma unroll
@@ -472,7 +464,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         if (r < rows && compute && q < g && !kPipe) {
             // KQ = 2: 4 consumer warps per scheduler hide the latencies; one register set.
             const uint32_t xs = sbase + prm.o_stage + (reuse0 ? 0 : slot) * prm.stage_bytes;
-            const uint32_t tb = table_base(reuse0 ? 0 : t);
+            const uint32_t tb = table_base(reuse0 ? 0 : slot);
             for (int j = q; j < g; j += KQ) {
                 if (cw == 0 && lane == 0) trace_ev(prm, p, i, 8 + j);
                 uint32_t bfr[NT][2];
@@ -486,7 +478,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
             }
         } else if (r < rows && compute && q < g) {
             const uint32_t xs = sbase + prm.o_stage + (reuse0 ? 0 : slot) * prm.stage_bytes;
-            const uint32_t tb = table_base(reuse0 ? 0 : t);
+            const uint32_t tb = table_base(reuse0 ? 0 : slot);
             for (int j = q; j < g; j += KQ) {
                 uint32_t bfr[NT][2];
                 load_x(xs, j, bfr);
@@ -510,8 +502,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         if (cw == 0 && lane == 0) trace_ev(prm, p, i, 7);   // consumer warp 0 finished the stage's work
         __syncwarp();
         if (lane == 0 && !reuse0) {
-            mbar_arrive(bar_empty + 8 * slot);
-            mbar_arrive(bar_tble + 8 * t);
+            mbar_arrive(bar_empty + 8 * slot);   // frees the ring slot and its table
             if (cw == 0) trace_ev(prm, p, i, 6);
         }
         const bool seg_end = (gc + g == KG) || (it.du + g == it.du1);
@@ -652,7 +643,8 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         uint32_t vcap = align_up((uint32_t)G * maxv * 2, 16);
         uint32_t st_v1 = st_v0 + vcap;
         uint32_t stage = align_up(st_v1 + vcap, 128);
-        uint32_t fixed = o_pre + pre_bytes + kTblSlots * tbl + scr + 128;   // +slack for the t1 over-read
+        uint32_t fixed = o_pre + pre_bytes + scr + 128;   // +slack for the t1 over-read
+        stage += tbl;                                     // each ring slot carries its table (accounted with it)
         if ((long long)fixed + 2LL * stage > smem_max) continue;
         int S = (int)std::min<long long>(smax, ((long long)smem_max - fixed) / stage);
         if (S < 3 && G > 1) continue;
@@ -660,11 +652,12 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         pl->S = S;
         Params &q = pl->prm;
         q.KG = KG; q.MG = MG; q.U = pl->U; q.P = pl->P; q.G = G; q.S = S;
+        stage -= tbl;
         q.stage_bytes = stage; q.st_bm = st_bm; q.st_v0 = st_v0; q.st_v1 = st_v1;
         q.tbl_bytes = tbl;
         q.o_pre = o_pre;
         q.o_tbl = o_pre + pre_bytes;
-        q.o_scr = q.o_tbl + kTblSlots * tbl;
+        q.o_scr = q.o_tbl + (uint32_t)S * tbl;
         q.o_stage = q.o_scr + scr;
         pl->smem = (size_t)q.o_stage + (size_t)S * stage + 128;
         return true;
