@@ -50,7 +50,6 @@ template <int NT> struct Cfg {
 };
 constexpr int kMaxStages = 8;
 constexpr int kMaxG = 4;            // max GroupTile columns per stage
-constexpr int kPrefetchStages = 6;  // L2 prefetch distance of the producer, in stages
 constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector-table constants
 constexpr int kTraceCTAs = 4, kTraceStages = 64, kTraceEv = 16;
 // Workspace = [fix-up counters: one int32 per GT row, fixed-size region][split-K partials].
@@ -232,32 +231,12 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
         // ------------------------------------------------------------ producer
         const uint64_t pol_w = policy_evict_first();
         constexpr int cpr = N / 8;                     // 16-byte chunks per X row
-        // L2 prefetch runs kPrefetchStages stages ahead of the smem ring so that ring refills
-        // hit L2: the ring alone (3-4 stages) cannot cover the loaded-HBM latency.
-        StageIter pf;
-        pf.init(u0, u1, prm);
-        auto prefetch = [&](const StageIter &s) {
-            const long long us = u0 + s.du;
-            const int4 ps = pre[us - u0], pe = pre[us - u0 + s.g - 1];
-            for (int r = 0; r < s.rows; ++r) {
-                const int start = r ? ps.z : ps.x, end = r ? pe.w : pe.y;
-                if (end > start) bulk_prefetch_l2(prm.vals + start, 2u * (uint32_t)(end - start));
-                bulk_prefetch_l2(prm.bm + ((size_t)(kR * s.rb + r) * KG + s.gc) * 64, (uint32_t)s.g * 512u);
-            }
-        };
-        if (lane == 0) {
-            for (int k = 0; k < kPrefetchStages && pf.valid(); ++k, pf.next(prm)) prefetch(pf);
-        }
         StageIter it;
         for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
             const StageIter &sg = it;
             const long long u = u0 + it.du;
             const int i = it.i, slot = it.slot;
             if ((dbg_mode(prm) & 4) && i > 0) break;   // experiment: consumers reuse stage 0 forever
-            if (lane == 0 && pf.valid()) {
-                prefetch(pf);
-                pf.next(prm);
-            }
             if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, it.par() ^ 1u);
             if (lane == 0) trace_ev(prm, p, i, 0);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
