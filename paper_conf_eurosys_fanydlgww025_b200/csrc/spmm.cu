@@ -31,6 +31,11 @@
 #include "internal.cuh"
 #include "ptx.cuh"
 
+// experiments: force the 8-consumer-warp variant for N <= 16
+#ifndef SPINFER_FORCE_KQ1
+#define SPINFER_FORCE_KQ1 0
+#endif
+
 namespace spinfer {
 namespace {
 
@@ -41,7 +46,7 @@ constexpr int kScanWarps = kR;      // one scan warp per GT row of the rowblock
 // the scheduler enough warps to hide ALU/XU/LDS latencies; it needs the accumulators to
 // fit the tighter register budget, so N >= 24 uses KQ = 1.
 template <int NT> struct Cfg {
-    static constexpr int KQ = NT <= 2 ? 2 : 1;
+    static constexpr int KQ = (NT <= 2 && !SPINFER_FORCE_KQ1) ? 2 : 1;
     static constexpr int CW = kR * 4 * KQ;                        // consumer warps
     static constexpr int ScanWarp = CW;                           // warp ids: the scheduler favours the
     static constexpr int ProducerWarp = CW + kScanWarps;          // highest id, so roles go on top
@@ -146,22 +151,21 @@ __device__ __forceinline__ uint32_t x_swz(uint32_t k) {
 }
 
 // SMBD for one BitmapTile and one lane, split into phases so
-// a warp keeps many shared-memory loads in flight. The scan warp's table entry
-// for (BT, lane-half h) is {w, A}: w = bitmap word h (bits 32h..32h+31), A = smem
-// byte address of the first value of that half. With sh = 2*(lane%16), lm = (1<<sh)-1:
-//   count = PopCount(w & lm)                       (MaskedPopCount, Alg. 2)
-//   t0 = V[count], t1 = V[count+1]                 (zero-extended u16 loads)
-//   a0 = bit(sh)   ? t0 : 0                        (Phase I)
-//   a1 = bit(sh+1) ? (bit(sh) ? t1 : t0) : 0       (Phase II reuses count)
-// The four (bit(sh), bit(sh+1)) cases are one PRMT of {t0, t1} whose selector depends
-// on y = (w >> sh) & 3; zero halves select the u16 loads' zero upper bytes (byte 2/3 of
-// t0, 6/7 of t1, optionally in sign-replicate mode, which also yields 0x00):
-//   y=0 -> (0,0)  y=1 -> (t0,0)  y=2 -> (0,t0)  y=3 -> (t0,t1)
+// a warp keeps many shared-memory loads in flight. The scan warps' table entry for
+// (BT, lane-half h) is {w, A}: w = bitmap word h (bits 32h..32h+31), A = smem byte
+// address of the first value of that half, minus 4. With sh = 2*(lane%16):
+//   z  = w << (30 - sh)          top two bits = y = (bit sh, bit sh+1) of w
+//   c2 = PopCount(z)             = MaskedPopCount (Alg. 2) + bit sh + bit sh+1
+//   t_lo = V[c2 - 2], t_hi = V[c2 - 1]   (zero-extended u16 loads)
+//   a0 = bit sh ? (bit sh+1 ? t_lo : t_hi) : 0     (Phase I)
+//   a1 = bit sh+1 ? t_hi : 0                        (Phase II reuses the count)
+// The four y cases are one PRMT of {t_lo, t_hi}; zero halves select the u16 loads'
+// zero upper bytes (bytes 2/3 of t_lo, 6/7 of t_hi, optionally in sign-replicate mode):
+//   y=0 -> (0,0)  y=1 -> (t_hi,0)  y=2 -> (0,t_hi)  y=3 -> (t_lo,t_hi)
 // The selector is the quadratic sel(y) = y*(kSelA + kSelB*y) + kSelC (mod 2^16), found by
-// exhaustive search (tools/selector_search.py; pinned in tests/test_host_logic.py):
-//   sel(0)=0x2333 sel(1)=0xab10 sel(2)=0x10af sel(3)=0x5410
-// — two IMADs on the FMA pipe instead of ALU-pipe work (the ALU pipe is half rate on B200).
-constexpr uint32_t kSelA = 0x18fcu, kSelB = 0x6ee1u, kSelC = 0x2333u;
+// exhaustive search (tools/selector_search.py; pinned in tests/test_host_logic.py) —
+// two IMADs on the FMA pipe instead of ALU-pipe work (the ALU pipe is half rate on B200).
+constexpr uint32_t kSelA = 0x7f62u, kSelB = 0x4cbfu, kSelC = 0x2333u;
 
 template <int NT>
 __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const float (&acc)[4][NT][4], int lane) {
@@ -335,10 +339,11 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
                     const uint32_t Aa = vsm + 2u * (uint32_t)(rel + (int)ea);
                     const uint32_t Ab = vsm + 2u * (uint32_t)(rel + (int)eb);
                     const uint32_t te = tb + (uint32_t)(r * G + j) * 1024u + 8u * lane;
-                    sts_v2(te, ba[q].x, Aa);
-                    sts_v2(te + 512u, ba[q].y, Aa + 2u * __popc(ba[q].x));
-                    sts_v2(te + 256u, bb[q].x, Ab);
-                    sts_v2(te + 768u, bb[q].y, Ab + 2u * __popc(bb[q].x));
+                    // entries hold (first value address - 4): the consumers address V[c2 - 2]
+                    sts_v2(te, ba[q].x, Aa - 4u);
+                    sts_v2(te + 512u, ba[q].y, Aa - 4u + 2u * __popc(ba[q].x));
+                    sts_v2(te + 256u, bb[q].x, Ab - 4u);
+                    sts_v2(te + 768u, bb[q].y, Ab - 4u + 2u * __popc(bb[q].x));
                 }
             }
             mbar_arrive(bar_scan + 8 * slot);
@@ -350,7 +355,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
     // ---------------------------------------------------------------- consumers
     const int cw = warp, q = cw % KQ, c = (cw / KQ) & 3, r = cw / (4 * KQ);
     const uint32_t sh = 2u * (lane & 15);
-    const uint32_t mulc = sh ? (1u << (32u - sh)) : 0u;     // w * mulc == w << (32 - sh), 0 for sh = 0
+    const uint32_t mulc = 1u << (30u - sh);                   // w * mulc == w << (30 - sh)
     // selector polynomial constants, read from smem so ptxas keeps them in registers
     const uint32_t selA = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];
     const uint32_t selB = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];
@@ -381,15 +386,15 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
 #pragma unroll
         for (int k = 0; k < 8; ++k) {
             const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
-            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;
-            // MaskedPopCount: popc(w & ((1 << sh) - 1)) == popc(w << (32 - sh)), the shift done
-            // as a multiply (FMA pipe) because the ALU pipe is the scarce one (half rate)
-            const uint32_t a = A + 2u * __popc(w * mulc);
-            // selector = y*(kSelA + kSelB*y) + kSelC: two IMADs instead of a PRMT table lookup
-            const uint32_t y = (w >> sh) & 3u;
-            s1[k] = y * (y * selB + selA) + selC;
-            t0[k] = lds_u16(a);
-            t1[k] = lds_u16(a + 2u);
+            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;   // (first value of the half) - 4 bytes
+            // z = w << (30 - sh) as a multiply (FMA pipe): its top two bits are the lane's pair
+            // y = (bit sh, bit sh+1) and popc(z) = c2 = MaskedPopCount + b0 + b1 (Alg. 2)
+            const uint32_t z = w * mulc;
+            const uint32_t a = A + 2u * __popc(z);        // &V[c2 - 2]
+            const uint32_t y = z >> 30;
+            s1[k] = y * (y * selB + selA) + selC;          // selector polynomial (see kSelA)
+            t0[k] = lds_u16(a);                            // V[c2 - 2]
+            t1[k] = lds_u16(a + 2u);                       // V[c2 - 1]
         }
     };
     auto assemble = [&](const uint32_t (&t0)[8], const uint32_t (&t1)[8], const uint32_t (&s1)[8], int trb,

@@ -1,7 +1,7 @@
 """Host-side logic of the CUDA path that can be checked without a GPU (-m "not gpu")."""
 import random
 
-KSEL = (0x18FC, 0x6EE1, 0x2333)   # csrc/spmm.cu kSelA, kSelB, kSelC
+KSEL = (0x7F62, 0x4CBF, 0x2333)   # csrc/spmm.cu kSelA, kSelB, kSelC
 
 
 def prmt(a, b, sel):
@@ -18,27 +18,41 @@ def prmt(a, b, sel):
 
 
 def test_selector_polynomial_matches_two_phase_decode():
-    """sel(y) = y*(A + B*y) + C reproduces Phase I / Phase II of P:287 for all bit pairs."""
+    """sel(y) = y*(A + B*y) + C reproduces Phase I / Phase II of P:287 for all bit pairs,
+    with t_lo = V[c2 - 2], t_hi = V[c2 - 1], c2 = MaskedPopCount + b0 + b1."""
     A, B, C = KSEL
     rng = random.Random(0)
     for y in range(4):
         sel = (y * ((A + B * y) & 0xFFFFFFFF) + C) & 0xFFFFFFFF
         b0, b1 = y & 1, y >> 1
         for _ in range(2000):
-            v0, v1 = rng.randrange(65536), rng.randrange(65536)   # V[count], V[count+1]
-            lo = v0 if b0 else 0
-            hi = (v1 if b0 else v0) if b1 else 0
-            assert prmt(v0, v1, sel) == (hi << 16) | lo
+            V = [rng.randrange(65536) for _ in range(8)]
+            cnt = rng.randrange(2, 6)                       # MaskedPopCount (values before the pair)
+            c2 = cnt + b0 + b1
+            t_lo, t_hi = V[c2 - 2], V[c2 - 1]
+            lo = V[cnt] if b0 else 0                        # Phase I
+            hi = V[cnt + b0] if b1 else 0                   # Phase II
+            assert prmt(t_lo, t_hi, sel) == (hi << 16) | lo
 
 
-def test_masked_popcount_as_multiply():
-    """popc(w & ((1 << sh) - 1)) == popc((w * 2^(32-sh)) mod 2^32), multiplier 0 for sh = 0."""
+def test_selector_search_reproduces_constants():
+    import importlib.util, os
+    spec = importlib.util.spec_from_file_location(
+        "sel", os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tools", "selector_search.py"))
+    m = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(m)
+    assert KSEL in m.search()
+
+
+def test_pair_count_and_bits_as_multiply():
+    """z = w * 2^(30-sh) mod 2^32: z >> 30 = bits (sh, sh+1) and popc(z) = popc(w & ((4 << sh) - 1))."""
     rng = random.Random(1)
     for _ in range(5000):
         w = rng.getrandbits(32)
         sh = 2 * rng.randrange(16)
-        mul = (1 << (32 - sh)) & 0xFFFFFFFF if sh else 0
-        assert bin((w * mul) & 0xFFFFFFFF).count("1") == bin(w & ((1 << sh) - 1)).count("1")
+        z = (w * (1 << (30 - sh))) & 0xFFFFFFFF
+        assert z >> 30 == (w >> sh) & 3
+        assert bin(z).count("1") == bin(w & ((4 << sh) - 1)).count("1")
 
 
 def test_stream_k_partition():
