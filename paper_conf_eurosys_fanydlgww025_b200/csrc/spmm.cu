@@ -54,7 +54,7 @@ template <int NT> struct Cfg {
     static constexpr int ScrSlots = 2 * KQ;                       // epilogue scratch slots per GT row
 };
 constexpr int kMaxStages = 8;
-constexpr int kMaxG = 4;            // max GroupTile columns per stage
+constexpr int kMaxG = 6;            // max GroupTile columns per stage
 constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector-table constants
 constexpr int kTraceCTAs = 4, kTraceStages = 64, kTraceEv = 16;
 // Workspace = [fix-up counters: one int32 per GT row, fixed-size region][split-K partials].
@@ -77,7 +77,7 @@ struct Params {
     int G, S;
     uint32_t stage_bytes, st_bm, st_v0, st_v1;  // stage slot size; offsets in a slot (X slab at 0)
     uint32_t tbl_bytes;
-    uint32_t o_pre, o_tbl, o_scr, o_stage;      // region offsets from the smem base
+    uint32_t o_pre, o_tbl, o_stage;             // region offsets from the smem base
     long long *trace;   // experiments only (SPINFER_TRACE): [kTraceCTAs][kTraceStages][8] clock64 stamps
     int dbg;            // experiments only (SPINFER_DEBUG_MODE): bit0 = consumers skip decode/MMA, bit1 = scan skips work
 };
@@ -368,7 +368,6 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
     const uint32_t xsw = x_swz<NT>(rr);                     // swizzle depends on k % 8 == rr only
     float acc[4][NT][4];
     constexpr uint32_t kPart = 64u * N * 4u;                      // one fp32 64 x N partial
-    const uint32_t scr = sbase + prm.o_scr + (uint32_t)r * (Cfg<NT>::ScrSlots * kPart);
 
     // Software pipeline over half-GT steps (8 BTs = TCTile rows 2h', 2h'+1 of GT j):
     // while step h is assembled and multiplied, the value loads of step h+1 and the
@@ -505,16 +504,15 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
             begin_stage(nx);
         }
         if (cw == 0 && lane == 0) trace_ev(prm, p, i, 7);   // consumer warp 0 finished the stage's work
-        __syncwarp();
-        if (lane == 0 && !reuse0) {
-            mbar_arrive(bar_empty + 8 * slot);   // frees the ring slot and its table
-            if (cw == 0) trace_ev(prm, p, i, 6);
-        }
         const bool seg_end = (gc + g == KG) || (it.du + g == it.du1);
         if (seg_end && r < rows) {
             // -------------------------------------------------------- epilogue
-            // (1) reduce the 4*KQ partials of GT row r into warp (c = 0, q = 0), tree via smem
+            // (1) reduce the 4*KQ partials of GT row r into warp (c = 0, q = 0), tree via smem.
+            // Scratch = this stage's value region of GT row r: only row r's consumer warps read
+            // it, so once they all pass the first barrier it is free (the slot is released below).
             const uint32_t bid = 1u + (uint32_t)r, bcnt = 128u * KQ;
+            const uint32_t scr = sbase + prm.o_stage + slot * prm.stage_bytes + (r ? prm.st_v1 : prm.st_v0);
+            named_bar_sync(bid, bcnt);
             auto put = [&](uint32_t slot_) {
 #pragma unroll
                 for (int tr = 0; tr < 4; ++tr)
@@ -594,6 +592,11 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
                 }
             }
         }
+        __syncwarp();
+        if (lane == 0 && !reuse0) {
+            mbar_arrive(bar_empty + 8 * slot);   // frees the ring slot and its table
+            if (cw == 0) trace_ev(prm, p, i, 6);
+        }
     }
 }
 
@@ -642,13 +645,13 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
     if (const char *e = getenv("SPINFER_S")) smax = std::max(2, std::min(kMaxStages, atoi(e)));
     for (int G = gmax; G >= 1; --G) {
         uint32_t tbl = (uint32_t)kR * G * 64 * 16;
-        uint32_t scr = (uint32_t)kR * (N <= 16 ? 4 : 2) * 64 * N * 4;   // Cfg<NT>::ScrSlots partial slots per row
+        const uint32_t scr_row = (uint32_t)(N <= 16 ? 4 : 2) * 64 * N * 4;   // Cfg<NT>::ScrSlots partials, epilogue scratch per row
         uint32_t st_bm = (uint32_t)G * 64 * N * 2;            // X slab first, then bitmaps
         uint32_t st_v0 = st_bm + (uint32_t)kR * G * 512;
-        uint32_t vcap = align_up((uint32_t)G * maxv * 2, 16);
+        uint32_t vcap = align_up(std::max((uint32_t)G * maxv * 2, scr_row), 16);   // also the epilogue scratch
         uint32_t st_v1 = st_v0 + vcap;
         uint32_t stage = align_up(st_v1 + vcap, 128);
-        uint32_t fixed = o_pre + pre_bytes + scr + 128;   // +slack for the t1 over-read
+        uint32_t fixed = o_pre + pre_bytes + 128;   // +slack for the t1 over-read
         stage += tbl;                                     // each ring slot carries its table (accounted with it)
         if ((long long)fixed + 2LL * stage > smem_max) continue;
         int S = (int)std::min<long long>(smax, ((long long)smem_max - fixed) / stage);
@@ -662,8 +665,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         q.tbl_bytes = tbl;
         q.o_pre = o_pre;
         q.o_tbl = o_pre + pre_bytes;
-        q.o_scr = q.o_tbl + (uint32_t)S * tbl;
-        q.o_stage = q.o_scr + scr;
+        q.o_stage = q.o_tbl + (uint32_t)S * tbl;
         pl->smem = (size_t)q.o_stage + (size_t)S * stage + 128;
         return true;
     }
