@@ -85,6 +85,13 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t
 // cp.async (LDGSTS) 16 B global -> shared, L2 only; completion tracked by an mbarrier:
 // cp.async.mbarrier.arrive.noinc makes the barrier observe one arrival when all of
 // this thread's prior cp.async operations have completed.
+// 2-D TMA tile load (tensor map in param/const space, coordinates innermost first).
+__device__ __forceinline__ void tma_2d_g2s(uint32_t dst, const void *tmap, int c0, int c1, uint32_t bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%2, %3}], [%4];"
+        ::"r"(dst), "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(bar) : "memory");
+}
 __device__ __forceinline__ void cp_async_16(uint32_t dst, const void *src) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
 }

@@ -10,14 +10,14 @@
 // A "stage" = up to G consecutive units of one rowblock.
 //
 // Warp roles (11 warps; ids chosen for scheduler priority, see kProducerWarp):
-//   warp 10   producer: lane 0 issues one cp.async.bulk (1-D TMA) per GT row for
-//             the stage's packed values (the only large, contiguous stream); the
-//             32 lanes copy the stage's bitmaps and X slab (L2-resident) with
-//             16-byte cp.async into the slot (X swizzled bank-conflict-free),
-//             completing on the same barrier. S-stage smem ring, full/empty
-//             mbarriers (replaces the paper's LDGSTS.128 double buffer, P:224,
-//             P:293-301; measured: per-copy TMA overhead makes few, large copies
-//             the right shape on B200).
+//   top warp  producer: one lane issues, per stage, one cp.async.bulk (1-D TMA) per
+//             GT row for the packed values and one for the bitmaps (both contiguous
+//             per GT row), and one 2-D tensor TMA per GroupTile column for the X slab
+//             (hardware 32B/64B swizzle = the ldmatrix bank-conflict-free layout),
+//             all completing on the slot's full mbarrier. S-stage smem ring,
+//             full/empty mbarriers (replaces the paper's LDGSTS.128 double buffer,
+//             P:224; measured: issuing the bitmaps and X as 16-byte
+//             cp.async cost the producer ~1.6K cycles per stage).
 //   warps 8,9 scan (one per GT row): for each staged GroupTile computes every BitmapTile's base
 //             (PopCount prefix over earlier BTs) and writes a table
 //             {bitmap half-word, smem address of that half's first value}.
@@ -25,6 +25,7 @@
 //             (MaskedPopCount, Alg. 2, two-phase a0/a1 P:287) into
 //             mma.m16n8k16 A fragments, X via ldmatrix.trans, mma.sync with
 //             fp32 accumulators (Listing 1).
+#include <cuda.h>   // CUtensorMap (type + enums only; the encoder comes via cudaGetDriverEntryPoint)
 #include <algorithm>
 #include <cstdio>
 #include <cstdlib>
@@ -51,10 +52,12 @@ template <int NT> struct Cfg {
     static constexpr int ScanWarp = CW;                           // warp ids: the scheduler favours the
     static constexpr int ProducerWarp = CW + kScanWarps;          // highest id, so roles go on top
     static constexpr int Threads = 32 * (CW + kScanWarps + 1);
-    static constexpr int ScrSlots = 2 * KQ;                       // epilogue scratch slots per GT row
 };
 constexpr int kMaxStages = 8;
-constexpr int kMaxG = 6;            // max GroupTile columns per stage
+#ifndef SPINFER_MAXG
+#define SPINFER_MAXG 4
+#endif
+constexpr int kMaxG = SPINFER_MAXG;  // max GroupTile columns per stage (the scan unrolls over it)
 constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector-table constants
 constexpr int kTraceCTAs = 4, kTraceStages = 64, kTraceEv = 16;
 // Workspace = [fix-up counters: one int32 per GT row, fixed-size region][split-K partials].
@@ -64,6 +67,7 @@ constexpr int kMaxCounters = 16384;                 // M <= 1,048,576 rows
 constexpr size_t kCounterBytes = (size_t)kMaxCounters * 4;
 
 struct Params {
+    CUtensorMap tmap_x;          // X [K][N] fp16, box {N, 64}, swizzle 32B (N=16) / 64B (N=32) / none
     const int32_t *off;
     const uint64_t *bm;
     const uint16_t *vals;
@@ -143,6 +147,9 @@ struct StageIter {
 // chunk c of row k is stored at chunk slot c ^ swz(k) so that the 8 row reads of
 // one ldmatrix phase hit 8 distinct bank groups (N = 16: rows are 32 B apart,
 // rows k and k+4 would collide; N = 32: rows k, k+2). N = 8 and 24 are conflict-free.
+// The TMA writes this layout: its SWIZZLE_32B / SWIZZLE_64B modes XOR the chunk index
+// with smem address bits 7 (/ 7-8), i.e. with (k >> 2) & 1 (N = 16) and (k >> 1) & 3
+// (N = 32) for a slab that starts 1024-byte aligned.
 template <int NT>
 __device__ __forceinline__ uint32_t x_swz(uint32_t k) {
     if constexpr (NT == 2) return (k >> 2) & 1u;
@@ -183,11 +190,14 @@ __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const 
 }
 
 template <int NT>
-__global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) {
+__global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_constant__ Params prm) {
     constexpr int N = NT * 8;
     constexpr int KQ = Cfg<NT>::KQ, kCW = Cfg<NT>::CW, kThreads = Cfg<NT>::Threads;
     constexpr int kScanWarp = Cfg<NT>::ScanWarp, kProducerWarp = Cfg<NT>::ProducerWarp;
-    extern __shared__ __align__(128) uint8_t smem[];
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    // ring slots are 1024-byte aligned relative to this base: the TMA swizzle pattern of the
+    // X slab is a function of the smem address bits (x_swz assumes slab-relative row index)
+    uint8_t *const smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     const uint32_t sbase = smem_u32(smem);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int p = blockIdx.x;
@@ -204,10 +214,10 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
-            mbar_init(bar_full + 8 * s, 32);      // the 32 producer lanes (+ TMA transaction bytes)
+            mbar_init(bar_full + 8 * s, 1);       // the producer's arrive.expect_tx (+ TMA transaction bytes)
             mbar_init(bar_empty + 8 * s, kCW);
         }
-        for (int s = 0; s < S; ++s) mbar_init(bar_scan + 8 * s, 32 * kScanWarps);
+        for (int s = 0; s < S; ++s) mbar_init(bar_scan + 8 * s, kScanWarps);   // one elected arrive per scan warp
         fence_barrier_init();
         // SMBD selector-table constants, read back into registers by every consumer thread so
         // ptxas keeps them live in registers instead of re-materialising them per PRMT.
@@ -233,8 +243,9 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
 
     if (warp == kProducerWarp) {
         // ------------------------------------------------------------ producer
+        if (lane != 0) return;
         const uint64_t pol_w = policy_evict_first();
-        constexpr int cpr = N / 8;                     // 16-byte chunks per X row
+        const uint32_t xbytes = 64u * N * 2u;          // one GroupTile column of X
         StageIter it;
         for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
             const StageIter &sg = it;
@@ -242,33 +253,21 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
             const int i = it.i, slot = it.slot;
             if ((dbg_mode(prm) & 4) && i > 0) break;   // experiment: consumers reuse stage 0 forever
             if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, it.par() ^ 1u);
-            if (lane == 0) trace_ev(prm, p, i, 0);
+            trace_ev(prm, p, i, 0);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const uint32_t fb = bar_full + 8 * slot;
-            if (lane == 0) {
-                const int4 ps = pre[u - u0], pe = pre[u - u0 + sg.g - 1];
-                const uint32_t vb0 = 2u * (uint32_t)(pe.y - ps.x);
-                const uint32_t vb1 = sg.rows > 1 ? 2u * (uint32_t)(pe.w - ps.z) : 0u;
-                mbar_expect_tx(fb, vb0 + vb1);
-                if (vb0) bulk_g2s(st + prm.st_v0, prm.vals + ps.x, vb0, fb, pol_w);
-                if (vb1) bulk_g2s(st + prm.st_v1, prm.vals + ps.z, vb1, fb, pol_w);
-            }
-            // X slab rows [64 gc, 64 (gc + g)) -> smem with asynchronous 16-byte copies
-            // (LDGSTS, L2-resident source), swizzled; each lane's completion arrives on the
-            // full barrier (noinc: one of its 32 expected arrivals).
-            const uint4 *xsrc = reinterpret_cast<const uint4 *>(prm.X + (size_t)sg.gc * 64 * N);
-            const int nchunk = sg.g * 64 * cpr;
-            for (int e = lane; e < nchunk; e += 32) {
-                const uint32_t k = (uint32_t)(e / cpr), cch = (uint32_t)(e % cpr);
-                cp_async_16(st + (k * cpr + (cch ^ x_swz<NT>(k))) * 16u, xsrc + e);
-            }
-            // the stage's bitmaps (per GT row: g x 512 contiguous bytes) the same way
-            for (int r = 0; r < sg.rows; ++r) {
-                const uint4 *bsrc = reinterpret_cast<const uint4 *>(prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc) * 64);
-                const uint32_t bdst = st + prm.st_bm + (uint32_t)(r * G) * 512u;
-                for (int e = lane; e < sg.g * 32; e += 32) cp_async_16(bdst + 16u * e, bsrc + e);
-            }
-            cp_async_mbar_arrive_noinc(fb);
+            const int4 ps = pre[u - u0], pe = pre[u - u0 + sg.g - 1];
+            const uint32_t vb0 = 2u * (uint32_t)(pe.y - ps.x);
+            const uint32_t vb1 = sg.rows > 1 ? 2u * (uint32_t)(pe.w - ps.z) : 0u;
+            const uint32_t bmb = (uint32_t)sg.g * 512u;
+            mbar_arrive_expect_tx(fb, vb0 + vb1 + (uint32_t)sg.rows * bmb + (uint32_t)sg.g * xbytes);
+            if (vb0) bulk_g2s(st + prm.st_v0, prm.vals + ps.x, vb0, fb, pol_w);
+            if (vb1) bulk_g2s(st + prm.st_v1, prm.vals + ps.z, vb1, fb, pol_w);
+            for (int r = 0; r < sg.rows; ++r)
+                bulk_g2s(st + prm.st_bm + (uint32_t)(r * G) * 512u,
+                         prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc) * 64, bmb, fb, pol_w);
+            // X slab rows [64 gc, 64 (gc + g)): L2-resident (every CTA reads X), default policy
+            for (int j = 0; j < sg.g; ++j) tma_2d_g2s(st + (uint32_t)j * xbytes, &prm.tmap_x, 0, 64 * (sg.gc + j), fb);
         }
         return;
     }
@@ -346,7 +345,10 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const Params prm) 
                     sts_v2(te + 768u, bb[q].y, Ab - 4u + 2u * __popc(bb[q].x));
                 }
             }
-            mbar_arrive(bar_scan + 8 * slot);
+            // one arrive per warp: every mbarrier event wakes all sleeping waiters of the CTA,
+            // so 64 per-thread arrivals would cost each waiting consumer ~60 extra polls
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar_scan + 8 * slot);
             if (lane == 0 && r == 0) trace_ev(prm, p, i, 3);
         }
         return;
@@ -626,6 +628,35 @@ int choose_P(long long U) {
 
 inline uint32_t align_up(uint32_t x, uint32_t a) { return (x + a - 1) / a * a; }
 
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link).
+using EncodeTiledFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                   const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N) {
+    static EncodeTiledFn fn = nullptr;
+    if (!fn) {
+        void *f = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess || !f) {
+            cudaGetLastError();
+            return SPINFER_ECUDA;
+        }
+        fn = reinterpret_cast<EncodeTiledFn>(f);
+    }
+    const cuuint64_t dims[2] = {(cuuint64_t)N, (cuuint64_t)K};
+    const cuuint64_t strides[1] = {(cuuint64_t)N * 2};
+    const cuuint32_t box[2] = {(cuuint32_t)N, 64u};
+    const cuuint32_t estr[2] = {1u, 1u};
+    const CUtensorMapSwizzle sw = N == 16 ? CU_TENSOR_MAP_SWIZZLE_32B : N == 32 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                                               : CU_TENSOR_MAP_SWIZZLE_NONE;
+    CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, const_cast<uint16_t *>(X), dims, strides, box, estr,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? SPINFER_OK : SPINFER_EINVAL;
+}
+
 bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
     const int MG = M / kGT, KG = K / kGT;
     const int nRB = (MG + kR - 1) / kR;
@@ -645,13 +676,13 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
     if (const char *e = getenv("SPINFER_S")) smax = std::max(2, std::min(kMaxStages, atoi(e)));
     for (int G = gmax; G >= 1; --G) {
         uint32_t tbl = (uint32_t)kR * G * 64 * 16;
-        const uint32_t scr_row = (uint32_t)(N <= 16 ? 4 : 2) * 64 * N * 4;   // Cfg<NT>::ScrSlots partials, epilogue scratch per row
+        const uint32_t scr_row = (uint32_t)(N <= 16 ? 4 : 2) * 64 * N * 4;   // 2*KQ fp32 partials: the epilogue scratch per GT row
         uint32_t st_bm = (uint32_t)G * 64 * N * 2;            // X slab first, then bitmaps
         uint32_t st_v0 = st_bm + (uint32_t)kR * G * 512;
         uint32_t vcap = align_up(std::max((uint32_t)G * maxv * 2, scr_row), 16);   // also the epilogue scratch
         uint32_t st_v1 = st_v0 + vcap;
-        uint32_t stage = align_up(st_v1 + vcap, 128);
-        uint32_t fixed = o_pre + pre_bytes + 128;   // +slack for the t1 over-read
+        uint32_t stage = align_up(st_v1 + vcap, 1024);   // slots stay 1024-aligned (X swizzle)
+        uint32_t fixed = o_pre + pre_bytes + 128 + 2048;   // +slack: t1 over-read, base and ring alignment
         stage += tbl;                                     // each ring slot carries its table (accounted with it)
         if ((long long)fixed + 2LL * stage > smem_max) continue;
         int S = (int)std::min<long long>(smax, ((long long)smem_max - fixed) / stage);
@@ -665,8 +696,8 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         q.tbl_bytes = tbl;
         q.o_pre = o_pre;
         q.o_tbl = o_pre + pre_bytes;
-        q.o_stage = q.o_tbl + (uint32_t)S * tbl;
-        pl->smem = (size_t)q.o_stage + (size_t)S * stage + 128;
+        q.o_stage = align_up(q.o_tbl + (uint32_t)S * tbl, 1024);
+        pl->smem = (size_t)q.o_stage + (size_t)S * stage + 128 + 1024;   // +1024: runtime base alignment
         return true;
     }
     return false;
@@ -706,6 +737,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     if (need == 0) return SPINFER_EINVAL;
     if (ws_bytes < need || ws == nullptr) return SPINFER_ENOSPC;
     Params &q = pl.prm;
+    if (int rc = encode_x_map(&q.tmap_x, X, K, N)) return rc;
     q.off = T->gtile_offset;
     q.bm = T->bitmap;
     q.vals = T->values;
