@@ -54,6 +54,9 @@ template <int NT> struct Cfg {
     static constexpr int Threads = 32 * (CW + kScanWarps + 1);
 };
 constexpr int kMaxStages = 8;
+#ifndef SPINFER_PIPEMIX
+#define SPINFER_PIPEMIX 1
+#endif
 #ifndef SPINFER_MAXG
 #define SPINFER_MAXG 4
 #endif
@@ -81,7 +84,7 @@ struct Params {
     int G, S;
     uint32_t stage_bytes, st_bm, st_v0, st_v1;  // stage slot size; offsets in a slot (X slab at 0)
     uint32_t tbl_bytes;
-    uint32_t o_pre, o_tbl, o_stage;             // region offsets from the smem base
+    uint32_t o_pre, o_desc, o_tbl, o_stage;     // region offsets from the smem base
     long long *trace;   // experiments only (SPINFER_TRACE): [kTraceCTAs][kTraceStages][8] clock64 stamps
     int dbg;            // experiments only (SPINFER_DEBUG_MODE): bit0 = consumers skip decode/MMA, bit1 = scan skips work
 };
@@ -143,6 +146,24 @@ struct StageIter {
     }
 };
 
+// Per-CTA stage descriptor (built once in shared memory by scan warp 0): the consumer
+// loop then carries only the stage index across its decode loop. (Keeping the StageIter
+// live in registers made ptxas spill it; local memory goes to L2 here because the
+// shared-memory carve-out leaves almost no L1, so each stage paid ~800-cycle reloads.)
+//   w0: rb [0,20) | slot [20,24) | parity 24 | zero-acc 25 | segment end 26 | complete 27 | rows-1 28
+//   w1: gc [0,16) | g [16,24)
+struct StageDesc {
+    uint32_t w0, w1;
+    __device__ __forceinline__ int rb() const { return (int)(w0 & 0xFFFFFu); }
+    __device__ __forceinline__ int slot() const { return (int)((w0 >> 20) & 15u); }
+    __device__ __forceinline__ uint32_t par() const { return (w0 >> 24) & 1u; }
+    __device__ __forceinline__ bool zero() const { return (w0 >> 25) & 1u; }
+    __device__ __forceinline__ bool seg_end() const { return (w0 >> 26) & 1u; }
+    __device__ __forceinline__ bool complete() const { return (w0 >> 27) & 1u; }
+    __device__ __forceinline__ int rows() const { return 1 + (int)((w0 >> 28) & 1u); }
+    __device__ __forceinline__ int g() const { return (int)((w1 >> 16) & 0xFFu); }
+};
+
 // X slab swizzle (16-byte chunk granularity): row k of the slab holds N/8 chunks;
 // chunk c of row k is stored at chunk slot c ^ swz(k) so that the 8 row reads of
 // one ldmatrix phase hit 8 distinct bank groups (N = 16: rows are 32 B apart,
@@ -194,6 +215,8 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     constexpr int N = NT * 8;
     constexpr int KQ = Cfg<NT>::KQ, kCW = Cfg<NT>::CW, kThreads = Cfg<NT>::Threads;
     constexpr int kScanWarp = Cfg<NT>::ScanWarp, kProducerWarp = Cfg<NT>::ProducerWarp;
+    // named barriers: 0 = __syncthreads, 1..kR = epilogue (per GT row), kDescBar = descriptors ready
+    constexpr uint32_t kDescBar = 1 + kR;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     // ring slots are 1024-byte aligned relative to this base: the TMA swizzle pattern of the
     // X slab is a function of the smem address bits (x_swz assumes slab-relative row index)
@@ -282,6 +305,27 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         constexpr int Q = kMaxG;
         const int r = warp - kScanWarp;               // this scan warp's GT row
         const bool work = !(dbg_mode(prm) & 2);
+        if (r == 0) {
+            // stage descriptors for the consumers (in the shadow of the first data latency)
+            if (lane == 0) {
+                StageIter d;
+                int n = 0;
+                bool full_start = false;
+                for (d.init(u0, u1, prm); d.valid(); d.next(prm), ++n) {
+                    const bool zero = (d.gc == 0 || d.du == 0);
+                    if (zero) full_start = (d.gc == 0);
+                    const bool seg_end = (d.gc + d.g == KG) || (d.du + d.g == d.du1);
+                    const bool complete = seg_end && full_start && (d.gc + d.g == KG);
+                    const uint32_t w0 = (uint32_t)d.rb | ((uint32_t)d.slot << 20) | (d.ph << 24) | ((uint32_t)zero << 25) |
+                                        ((uint32_t)seg_end << 26) | ((uint32_t)complete << 27) |
+                                        ((uint32_t)(d.rows - 1) << 28);
+                    sts_v2(sbase + prm.o_desc + 8u * (uint32_t)n, w0, (uint32_t)d.gc | ((uint32_t)d.g << 16));
+                }
+                reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3] = (uint32_t)n;
+            }
+            __syncwarp();
+            named_bar_arrive(kDescBar, 32u * (kCW + 1));
+        }
         StageIter it;
         for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
             const StageIter &sg = it;
@@ -355,19 +399,39 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     }
 
     // ---------------------------------------------------------------- consumers
-    const int cw = warp, q = cw % KQ, c = (cw / KQ) & 3, r = cw / (4 * KQ);
-    const uint32_t sh = 2u * (lane & 15);
-    const uint32_t mulc = 1u << (30u - sh);                   // w * mulc == w << (30 - sh)
+    // Per-warp/lane constants are re-derived from a volatile %tid.x read wherever they are
+    // used (a few ALU ops per stage): values kept live across the decode loop get spilled,
+    // and a spill reload is an L2 round trip here.
+    struct Ctx {
+        int cw, q, c, r, lane;
+        uint32_t mulc, hioff, xrow, xsw, mn, four;
+    };
+    auto ctx = [&]() {
+        const uint32_t t = tid_volatile();
+        Ctx x;
+        x.lane = (int)(t & 31u);
+        x.cw = (int)(t >> 5);
+        x.q = x.cw % KQ;
+        x.c = (x.cw / KQ) & 3;
+        x.r = x.cw / (4 * KQ);
+        x.mulc = 1u << (30u - 2u * (t & 15u));               // w * mulc == w << (30 - sh), sh = 2 (lane % 16)
+#if SPINFER_PIPEMIX & 1
+        x.mulc = opaque_u32(x.mulc);   // hide the power of two: IMAD (FMA pipe) instead of SHF (ALU pipe)
+#endif
+        x.four = opaque_u32(4u);
+        x.hioff = ((t >> 4) & 1u) * 512u;
+        // ldmatrix.trans rows: matrix m = lane/8 -> (k half m&1, n chunk m>>1); row rr = lane%8.
+        const uint32_t rr = t & 7u, mk = (t >> 3) & 1u;
+        x.mn = (t >> 4) & 1u;
+        x.xrow = (mk * 8u + rr) * (uint32_t)(N / 8);          // + (64 j + 16 c) * cpr per k16 column
+        x.xsw = x_swz<NT>(rr);                                // swizzle depends on k % 8 == rr only
+        return x;
+    };
     // selector polynomial constants, read from smem so ptxas keeps them in registers
     const uint32_t selA = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];
     const uint32_t selB = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];
     const uint32_t selC = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 2];
-    const uint32_t hioff = (uint32_t)(lane >> 4) * 512u;
-    // ldmatrix.trans rows: matrix m = lane/8 -> (k half m&1, n chunk m>>1); row rr = lane%8.
     constexpr uint32_t cpr = N / 8;
-    const uint32_t rr = lane & 7, mk = (lane >> 3) & 1, mn = (lane >> 4) & 1;
-    const uint32_t xrow = (uint32_t)(mk * 8 + rr) * cpr;   // + (64 j + 16 c) * cpr per k16 column
-    const uint32_t xsw = x_swz<NT>(rr);                     // swizzle depends on k % 8 == rr only
     float acc[4][NT][4];
     constexpr uint32_t kPart = 64u * N * 4u;                      // one fp32 64 x N partial
 
@@ -383,16 +447,20 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
 #pragma unroll
         for (int q = 0; q < 4; ++q) E[q] = lds_v4(tb + (uint32_t)(step >> 1) * 1024u + (uint32_t)(step & 1) * 64u + 16u * q);
     };
-    auto issue = [&](uint32_t (&t0)[8], uint32_t (&t1)[8], uint32_t (&s1)[8]) {   // value loads from E
+    auto issue = [&](const Ctx &x, uint32_t (&t0)[8], uint32_t (&t1)[8], uint32_t (&s1)[8]) {   // value loads from E
 #pragma unroll
         for (int k = 0; k < 8; ++k) {
             const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
             const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;   // (first value of the half) - 4 bytes
             // z = w << (30 - sh) as a multiply (FMA pipe): its top two bits are the lane's pair
             // y = (bit sh, bit sh+1) and popc(z) = c2 = MaskedPopCount + b0 + b1 (Alg. 2)
-            const uint32_t z = w * mulc;
+            const uint32_t z = w * x.mulc;
             const uint32_t a = A + 2u * __popc(z);        // &V[c2 - 2]
+#if SPINFER_PIPEMIX & 2
+            const uint32_t y = __umulhi(z, x.four);       // IMAD.HI (FMA pipe) instead of SHF (ALU pipe)
+#else
             const uint32_t y = z >> 30;
+#endif
             s1[k] = y * (y * selB + selA) + selC;          // selector polynomial (see kSelA)
             t0[k] = lds_u16(a);                            // V[c2 - 2]
             t1[k] = lds_u16(a + 2u);                       // V[c2 - 1]
@@ -413,107 +481,113 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         }
     };
     // this warp's 16 entries of GT j (TCTiles c*4 .. c*4+3, all 4 BTs): 128 contiguous bytes
-    auto table_base = [&](int slot_) {
-        return sbase + prm.o_tbl + slot_ * prm.tbl_bytes + (uint32_t)(r * G) * 1024u + hioff + (uint32_t)c * 128u;
+    auto table_base = [&](const Ctx &x, int slot_) {
+        return sbase + prm.o_tbl + slot_ * prm.tbl_bytes + (uint32_t)(x.r * G) * 1024u + x.hioff + (uint32_t)x.c * 128u;
     };
     const bool compute = !(dbg_mode(prm) & 1);
     // Wait for a stage's data and table; if this warp has work in it, start its pipeline.
     constexpr bool kPipe = (KQ == 1);          // explicit cross-step software pipeline (8 consumer warps)
     const bool reuse0 = (dbg_mode(prm) & 4) != 0;   // experiment: pure consumer throughput on stage 0's data
-    auto load_x = [&](uint32_t xs, int j, uint32_t (&bfr)[NT][2]) {   // B fragments of GT j, TCTile column c
-        const uint32_t xk = xs + (xrow + (uint32_t)(64 * j + 16 * c) * cpr) * 16u;
+    auto load_x = [&](const Ctx &x, uint32_t xs, int j, uint32_t (&bfr)[NT][2]) {   // B fragments of GT j, TCTile column c
+        const uint32_t xk = xs + (x.xrow + (uint32_t)(64 * j + 16 * x.c) * cpr) * 16u;
         if constexpr (NT == 1) {
             ldsm_x2_trans(xk, bfr[0][0], bfr[0][1]);
         } else {
 #pragma unroll
             for (int nt = 0; nt + 1 < NT; nt += 2)
-                ldsm_x4_trans(xk + (((uint32_t)nt + mn) ^ xsw) * 16u, bfr[nt][0], bfr[nt][1], bfr[nt + 1][0],
+                ldsm_x4_trans(xk + (((uint32_t)nt + x.mn) ^ x.xsw) * 16u, bfr[nt][0], bfr[nt][1], bfr[nt + 1][0],
                               bfr[nt + 1][1]);
             if constexpr (NT % 2 == 1) ldsm_x2_trans(xk + (uint32_t)(NT - 1) * 16u, bfr[NT - 1][0], bfr[NT - 1][1]);
         }
     };
-    auto begin_stage = [&](const StageIter &s) {
-        if (!reuse0 || s.i == 0) {
+    auto begin_stage = [&](const Ctx &x, const StageDesc &s, int si) {
+        if (!reuse0 || si == 0) {
             // suspend rather than spin: a spinning consumer steals issue slots from the
             // other 15 consumer warps that still have decode work
-            mbar_wait_sleep(bar_scan + 8 * s.slot, s.par());   // implies full[s.slot] (see above)
-            if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 4);
-            if (cw == 0 && lane == 0) trace_ev(prm, p, s.i, 5);
+            mbar_wait_sleep(bar_scan + 8 * s.slot(), s.par());   // implies full[slot] (see above)
+            if (x.cw == 0 && x.lane == 0) trace_ev(prm, p, si, 4);
+            if (x.cw == 0 && x.lane == 0) trace_ev(prm, p, si, 5);
         }
-        if (kPipe && r < s.rows && compute && q < s.g) {
-            const uint32_t tb = table_base(reuse0 ? 0 : s.slot);
-            load_E(tb, 2 * q);
-            issue(tA0, tA1, sA);
-            load_E(tb, 2 * q + 1);
+        if (kPipe && x.r < s.rows() && compute && x.q < s.g()) {
+            const uint32_t tb = table_base(x, reuse0 ? 0 : s.slot());
+            load_E(tb, 2 * x.q);
+            issue(x, tA0, tA1, sA);
+            load_E(tb, 2 * x.q + 1);
         }
     };
-
-    bool seg_full_start = false;      // current rowblock segment started at the rowblock's first unit
-    StageIter it;
-    it.init(u0, u1, prm);
-    if (kPipe && it.valid()) begin_stage(it);
-    for (; it.valid(); it.next(prm)) {
-        const int rb = it.rb, gc = it.gc, g = it.g, rows = it.rows;
-        const int i = it.i, slot = it.slot;
-        if (gc == 0 || it.du == 0) {
-            seg_full_start = (gc == 0);
+    const uint32_t desc = sbase + prm.o_desc;
+    auto rd = [&](int si) {   // volatile shared load: re-read, never kept live across the decode loop
+        const uint2 v = lds_v2(desc + 8u * (uint32_t)si);
+        return StageDesc{v.x, v.y};
+    };
+    named_bar_sync(kDescBar, 32u * (kCW + 1));
+    auto nst = [&]() { return (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3]; };
+    if (kPipe && nst() > 0) begin_stage(ctx(), rd(0), 0);
+    for (int i = 0; i < nst(); ++i) {
+        const Ctx x = ctx();
+        const int q = x.q, c = x.c, r = x.r, cw = x.cw, lane = x.lane;
+        {
+            const StageDesc d = rd(i);
+            if (d.zero()) {
 #pragma unroll
-            for (int a = 0; a < 4; ++a)
+                for (int a = 0; a < 4; ++a)
 #pragma unroll
-                for (int b = 0; b < NT; ++b)
+                    for (int b = 0; b < NT; ++b)
 #pragma unroll
-                    for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
+                        for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
+            }
+            if constexpr (!kPipe) begin_stage(x, d, i);
         }
-        if constexpr (!kPipe) begin_stage(it);
-        StageIter nx = it;
-        if constexpr (kPipe) nx.next(prm);
-        if (r < rows && compute && q < g && !kPipe) {
+        const StageDesc d = rd(i);
+        const int g = d.g(), slot = d.slot();
+        if (d.rows() > r && compute && q < g && !kPipe) {
             // KQ = 2: 4 consumer warps per scheduler hide the latencies; one register set.
             const uint32_t xs = sbase + prm.o_stage + (reuse0 ? 0 : slot) * prm.stage_bytes;
-            const uint32_t tb = table_base(reuse0 ? 0 : slot);
+            const uint32_t tb = table_base(x, reuse0 ? 0 : slot);
             for (int j = q; j < g; j += KQ) {
                 if (cw == 0 && lane == 0) trace_ev(prm, p, i, 8 + j);
                 uint32_t bfr[NT][2];
-                load_x(xs, j, bfr);
+                load_x(x, xs, j, bfr);
 #pragma unroll
                 for (int h = 0; h < 2; ++h) {
                     load_E(tb, 2 * j + h);
-                    issue(tA0, tA1, sA);
+                    issue(x, tA0, tA1, sA);
                     assemble(tA0, tA1, sA, 2 * h, bfr);
                 }
             }
-        } else if (r < rows && compute && q < g) {
+        } else if (d.rows() > r && compute && q < g) {
             const uint32_t xs = sbase + prm.o_stage + (reuse0 ? 0 : slot) * prm.stage_bytes;
-            const uint32_t tb = table_base(reuse0 ? 0 : slot);
+            const uint32_t tb = table_base(x, reuse0 ? 0 : slot);
             for (int j = q; j < g; j += KQ) {
                 uint32_t bfr[NT][2];
-                load_x(xs, j, bfr);
+                load_x(x, xs, j, bfr);
                 // step (j, first half): issue (j, second half) into B, prefetch the entries of
                 // this warp's next GT, assemble (j, first half) from A
-                issue(tB0, tB1, sB);
+                issue(x, tB0, tB1, sB);
                 if (j + KQ < g) load_E(tb, 2 * (j + KQ));
                 assemble(tA0, tA1, sA, 0, bfr);
                 // step (j, second half): issue the next step (A: next GT, or the next stage's first step)
                 if (j + KQ < g) {
-                    issue(tA0, tA1, sA);
+                    issue(x, tA0, tA1, sA);
                     load_E(tb, 2 * (j + KQ) + 1);
-                } else if (nx.valid()) {
-                    begin_stage(nx);
+                } else if (i + 1 < nst()) {
+                    begin_stage(x, rd(i + 1), i + 1);
                 }
                 assemble(tB0, tB1, sB, 2, bfr);
             }
-        } else if (kPipe && nx.valid()) {
-            begin_stage(nx);
+        } else if (kPipe && i + 1 < nst()) {
+            begin_stage(x, rd(i + 1), i + 1);
         }
         if (cw == 0 && lane == 0) trace_ev(prm, p, i, 7);   // consumer warp 0 finished the stage's work
-        const bool seg_end = (gc + g == KG) || (it.du + g == it.du1);
-        if (seg_end && r < rows) {
+        const StageDesc e = rd(i);
+        const int rb = e.rb(), rows = e.rows();
+        if (e.seg_end() && r < rows) {
             // -------------------------------------------------------- epilogue
             // (1) reduce the 4*KQ partials of GT row r into warp (c = 0, q = 0), tree via smem.
             // Scratch = this stage's value region of GT row r: only row r's consumer warps read
             // it, so once they all pass the first barrier it is free (the slot is released below).
             const uint32_t bid = 1u + (uint32_t)r, bcnt = 128u * KQ;
-            const uint32_t scr = sbase + prm.o_stage + slot * prm.stage_bytes + (r ? prm.st_v1 : prm.st_v0);
+            const uint32_t scr = sbase + prm.o_stage + e.slot() * prm.stage_bytes + (r ? prm.st_v1 : prm.st_v0);
             named_bar_sync(bid, bcnt);
             auto put = [&](uint32_t slot_) {
 #pragma unroll
@@ -550,8 +624,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             if (c == 0 && q == 0) {
                 const int grow = kR * rb + r;
                 const int row_base = grow * 64;
-                const bool complete = seg_full_start && (gc + g == KG);
-                if (complete) {
+                if (e.complete()) {
                     store_y<NT>(prm.Y, N, row_base, acc, lane);
                 } else {
                     const int pf = unit_owner((long long)rb * KG, U, prm.P);
@@ -596,7 +669,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         }
         __syncwarp();
         if (lane == 0 && !reuse0) {
-            mbar_arrive(bar_empty + 8 * slot);   // frees the ring slot and its table
+            mbar_arrive(bar_empty + 8 * e.slot());   // frees the ring slot and its table
             if (cw == 0) trace_ev(prm, p, i, 6);
         }
     }
@@ -682,7 +755,9 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         uint32_t vcap = align_up(std::max((uint32_t)G * maxv * 2, scr_row), 16);   // also the epilogue scratch
         uint32_t st_v1 = st_v0 + vcap;
         uint32_t stage = align_up(st_v1 + vcap, 1024);   // slots stay 1024-aligned (X swizzle)
-        uint32_t fixed = o_pre + pre_bytes + 128 + 2048;   // +slack: t1 over-read, base and ring alignment
+        // stage descriptors: at most one per unit, and no more than ceil(units/G) + rowblock splits
+        const uint32_t desc_bytes = align_up((uint32_t)(8 * std::min<long long>(upc, upc / G + upc / KG + 3)), 128);
+        uint32_t fixed = o_pre + pre_bytes + desc_bytes + 128 + 2048;   // +slack: t1 over-read, base and ring alignment
         stage += tbl;                                     // each ring slot carries its table (accounted with it)
         if ((long long)fixed + 2LL * stage > smem_max) continue;
         int S = (int)std::min<long long>(smax, ((long long)smem_max - fixed) / stage);
@@ -695,7 +770,8 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         q.stage_bytes = stage; q.st_bm = st_bm; q.st_v0 = st_v0; q.st_v1 = st_v1;
         q.tbl_bytes = tbl;
         q.o_pre = o_pre;
-        q.o_tbl = o_pre + pre_bytes;
+        q.o_desc = o_pre + pre_bytes;
+        q.o_tbl = q.o_desc + desc_bytes;
         q.o_stage = align_up(q.o_tbl + (uint32_t)S * tbl, 1024);
         pl->smem = (size_t)q.o_stage + (size_t)S * stage + 128 + 1024;   // +1024: runtime base alignment
         return true;
