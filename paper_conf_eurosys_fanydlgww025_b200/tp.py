@@ -61,11 +61,16 @@ def gather_rows(Y_full: torch.Tensor, M: int, world: int, rank: int, group=None)
         # equal chunks: one all_gather_into_tensor straight into Y_full (no copy-out)
         dist.all_gather_into_tensor(Y_full, mine.clone() if Y_full.is_cuda else mine.contiguous(), group=group)
     else:
-        parts = [Y_full[bb:bb + cc] for bb, cc in spans]
-        outs = [torch.empty_like(p) for p in parts]
-        dist.all_gather(outs, mine.contiguous(), group=group)
-        for p, o in zip(parts, outs):
-            p.copy_(o)
+        # uneven chunks (M/64 not divisible by world): pad every chunk to the largest one and
+        # gather into one buffer (all_gather with unequal sizes is not portable across backends)
+        cmax = max(sizes)
+        send = Y_full.new_zeros((cmax,) + tuple(Y_full.shape[1:]))
+        send[:c] = mine
+        recv = Y_full.new_empty((world * cmax,) + tuple(Y_full.shape[1:]))
+        dist.all_gather_into_tensor(recv, send, group=group)
+        for r, (bb, cc) in enumerate(spans):
+            if r != rank:
+                Y_full[bb:bb + cc] = recv[r * cmax: r * cmax + cc]
     return Y_full
 
 
