@@ -66,6 +66,26 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
 __device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
     while (!mbar_try_wait_sleep(bar, parity)) { }
 }
+// Non-blocking probe of a phase.
+__device__ __forceinline__ bool mbar_test_wait(uint32_t bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
+    return ok != 0;
+}
+// For waiters that usually block for a long time (scan on data, producer on a free slot):
+// the hinted try_wait sleeps until ANY mbarrier event of the CTA, i.e. it wakes ~25 times
+// per stage; a timed back-off (plain nanosleep, not woken by barrier traffic) polls a few times.
+__device__ __forceinline__ void mbar_wait_backoff(uint32_t bar, uint32_t parity, uint32_t ns0, uint32_t ns_max) {
+    uint32_t ns = ns0;
+    while (!mbar_test_wait(bar, parity)) {
+        __nanosleep(ns);
+        ns = ns < ns_max ? 2 * ns : ns_max;
+    }
+}
 
 // ---------------------------------------------------------------- L2 policies
 __device__ __forceinline__ uint64_t policy_evict_first() {

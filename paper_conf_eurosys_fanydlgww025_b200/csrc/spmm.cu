@@ -54,6 +54,12 @@ template <int NT> struct Cfg {
     static constexpr int Threads = 32 * (CW + kScanWarps + 1);
 };
 constexpr int kMaxStages = 8;
+#ifndef SPINFER_SCANSPIN
+#define SPINFER_SCANSPIN 0
+#endif
+#ifndef SPINFER_CONSSPIN
+#define SPINFER_CONSSPIN 0
+#endif
 #ifndef SPINFER_PIPEMIX
 #define SPINFER_PIPEMIX 1
 #endif
@@ -62,7 +68,8 @@ constexpr int kMaxStages = 8;
 #endif
 constexpr int kMaxG = SPINFER_MAXG;  // max GroupTile columns per stage (the scan unrolls over it)
 constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector-table constants
-constexpr int kTraceCTAs = 4, kTraceStages = 64, kTraceEv = 16;
+constexpr int kPendWord = 52;       // smem words 52..55: pending split-K fix-ups [GT row][first/last segment]
+constexpr int kTraceCTAs = 4, kTraceStages = 64, kTraceW = 20, kTraceEv = 4;   // stage 63 = kernel-level events
 // Workspace = [fix-up counters: one int32 per GT row, fixed-size region][split-K partials].
 // The counter region has the same size for every shape so that one zeroed
 // workspace can serve calls of different shapes (partials never overlap counters).
@@ -94,9 +101,20 @@ struct Params {
 #ifndef SPINFER_INSTRUMENT
 #define SPINFER_INSTRUMENT 0
 #endif
-__device__ __forceinline__ void trace_ev(const Params &prm, int p, int i, int ev) {
+// trace[p][stage][warp][ev] (lane 0 of the warp records): consumers ev0 wait start, ev1 wait
+// end, ev2 decode end, ev3 slot released; scan ev0/ev1 wait, ev3 table published; producer
+// ev0 wait start, ev1 copies issued. Stage kTraceStages-1: ev0 entry, ev1 after the initial
+// __syncthreads, ev2 main loop done, ev3 exit.
+__device__ __forceinline__ void trace_ev(const Params &prm, int p, int i, int w, int ev) {
 #if SPINFER_INSTRUMENT
-    if (prm.trace && p < kTraceCTAs && i < kTraceStages) prm.trace[((size_t)p * kTraceStages + i) * kTraceEv + ev] = clock64();
+    if (prm.trace && p < kTraceCTAs && i < kTraceStages - 1 && w < kTraceW)
+        prm.trace[(((size_t)p * kTraceStages + i) * kTraceW + w) * kTraceEv + ev] = clock64();
+#endif
+}
+__device__ __forceinline__ void trace_k(const Params &prm, int p, int w, int ev) {
+#if SPINFER_INSTRUMENT
+    if (prm.trace && p < kTraceCTAs && w < kTraceW)
+        prm.trace[(((size_t)p * kTraceStages + kTraceStages - 1) * kTraceW + w) * kTraceEv + ev] = clock64();
 #endif
 }
 __device__ __forceinline__ int dbg_mode(const Params &prm) {
@@ -151,9 +169,9 @@ struct StageIter {
 // live in registers made ptxas spill it; local memory goes to L2 here because the
 // shared-memory carve-out leaves almost no L1, so each stage paid ~800-cycle reloads.)
 //   w0: rb [0,20) | slot [20,24) | parity 24 | zero-acc 25 | segment end 26 | complete 27 | rows-1 28
-//   w1: gc [0,16) | g [16,24)
+//   w1: gc [0,16) | g [16,24);  tbl, stg: the slot's table and stage region offsets
 struct StageDesc {
-    uint32_t w0, w1;
+    uint32_t w0, w1, tbl, stg;   // tbl / stg: smem offsets (from the aligned base) of the slot's table / stage
     __device__ __forceinline__ int rb() const { return (int)(w0 & 0xFFFFFu); }
     __device__ __forceinline__ int slot() const { return (int)((w0 >> 20) & 15u); }
     __device__ __forceinline__ uint32_t par() const { return (w0 >> 24) & 1u; }
@@ -235,6 +253,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     const uint32_t bar_scan = sbase + 16 * kMaxStages;
     int4 *pre = reinterpret_cast<int4 *>(smem + prm.o_pre);
 
+    if (lane == 0) trace_k(prm, p, warp, 0);
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
             mbar_init(bar_full + 8 * s, 1);       // the producer's arrive.expect_tx (+ TMA transaction bytes)
@@ -247,6 +266,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         reinterpret_cast<uint32_t *>(smem)[kConstWord] = kSelA;
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = kSelB;
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 2] = kSelC;
+        for (int k = 0; k < 2 * kR; ++k) reinterpret_cast<int *>(smem)[kPendWord + k] = -1;
     }
     // Preload this CTA's GTileOffset entries: pre[u-u0] = {start_r0, end_r0, start_r1, end_r1}.
     for (long long i = threadIdx.x; i < u1 - u0; i += kThreads) {
@@ -263,6 +283,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         pre[i] = v;
     }
     __syncthreads();
+    if (lane == 0) trace_k(prm, p, warp, 1);
 
     if (warp == kProducerWarp) {
         // ------------------------------------------------------------ producer
@@ -275,8 +296,8 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             const long long u = u0 + it.du;
             const int i = it.i, slot = it.slot;
             if ((dbg_mode(prm) & 4) && i > 0) break;   // experiment: consumers reuse stage 0 forever
+            trace_ev(prm, p, i, warp, 0);
             if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, it.par() ^ 1u);
-            trace_ev(prm, p, i, 0);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const uint32_t fb = bar_full + 8 * slot;
             const int4 ps = pre[u - u0], pe = pre[u - u0 + sg.g - 1];
@@ -291,7 +312,9 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                          prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc) * 64, bmb, fb, pol_w);
             // X slab rows [64 gc, 64 (gc + g)): L2-resident (every CTA reads X), default policy
             for (int j = 0; j < sg.g; ++j) tma_2d_g2s(st + (uint32_t)j * xbytes, &prm.tmap_x, 0, 64 * (sg.gc + j), fb);
+            trace_ev(prm, p, i, warp, 1);
         }
+        trace_k(prm, p, warp, 3);
         return;
     }
 
@@ -319,7 +342,10 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                     const uint32_t w0 = (uint32_t)d.rb | ((uint32_t)d.slot << 20) | (d.ph << 24) | ((uint32_t)zero << 25) |
                                         ((uint32_t)seg_end << 26) | ((uint32_t)complete << 27) |
                                         ((uint32_t)(d.rows - 1) << 28);
-                    sts_v2(sbase + prm.o_desc + 8u * (uint32_t)n, w0, (uint32_t)d.gc | ((uint32_t)d.g << 16));
+                    const uint32_t sl = (dbg_mode(prm) & 4) ? 0u : (uint32_t)d.slot;   // experiment: reuse slot 0
+                    sts_v4(sbase + prm.o_desc + 16u * (uint32_t)n,
+                           make_uint4(w0, (uint32_t)d.gc | ((uint32_t)d.g << 16), prm.o_tbl + sl * prm.tbl_bytes,
+                                      prm.o_stage + sl * prm.stage_bytes));
                 }
                 reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3] = (uint32_t)n;
             }
@@ -334,9 +360,13 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             if ((dbg_mode(prm) & 4) && i > 0) break;
             // suspend (not spin) while waiting: these warps have the highest scheduling
             // priority and would otherwise steal issue slots from the consumers
+            if (lane == 0) trace_ev(prm, p, i, warp, 0);
+#if SPINFER_SCANSPIN
+            mbar_wait(bar_full + 8 * slot, it.par());
+#else
             mbar_wait_sleep(bar_full + 8 * slot, it.par());
-            if (lane == 0 && r == 0) trace_ev(prm, p, i, 1);
-            if (lane == 0 && r == 0) trace_ev(prm, p, i, 2);
+#endif
+            if (lane == 0) trace_ev(prm, p, i, warp, 1);
             uint2 ba[Q], bb[Q];
 #pragma unroll
             for (int q = 0; q < Q; ++q) {
@@ -393,45 +423,33 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             // so 64 per-thread arrivals would cost each waiting consumer ~60 extra polls
             __syncwarp();
             if (lane == 0) mbar_arrive(bar_scan + 8 * slot);
-            if (lane == 0 && r == 0) trace_ev(prm, p, i, 3);
+            if (lane == 0) trace_ev(prm, p, i, warp, 3);
         }
+        if (lane == 0) trace_k(prm, p, warp, 3);
         return;
     }
 
     // ---------------------------------------------------------------- consumers
-    // Per-warp/lane constants are re-derived from a volatile %tid.x read wherever they are
-    // used (a few ALU ops per stage): values kept live across the decode loop get spilled,
-    // and a spill reload is an L2 round trip here.
-    struct Ctx {
-        int cw, q, c, r, lane;
-        uint32_t mulc, hioff, xrow, xsw, mn, four;
-    };
-    auto ctx = [&]() {
-        const uint32_t t = tid_volatile();
-        Ctx x;
-        x.lane = (int)(t & 31u);
-        x.cw = (int)(t >> 5);
-        x.q = x.cw % KQ;
-        x.c = (x.cw / KQ) & 3;
-        x.r = x.cw / (4 * KQ);
-        x.mulc = 1u << (30u - 2u * (t & 15u));               // w * mulc == w << (30 - sh), sh = 2 (lane % 16)
+    // Lane constants, computed once: this lane's byte offset inside a slot's table (GT row r,
+    // TCTile column c, lane-half h) and inside a slot's X slab (ldmatrix row and swizzled chunk),
+    // the SMBD shift multiplier, and the warp's (q, r). Everything stage-dependent comes from
+    // the stage descriptor (one 16-byte shared load per stage).
+    const int q = warp % KQ, c = (warp / KQ) & 3, r = warp / (4 * KQ);
+    uint32_t mulc = 1u << (30u - 2u * (uint32_t)(lane & 15));   // w * mulc == w << (30 - sh), sh = 2 (lane % 16)
 #if SPINFER_PIPEMIX & 1
-        x.mulc = opaque_u32(x.mulc);   // hide the power of two: IMAD (FMA pipe) instead of SHF (ALU pipe)
+    mulc = opaque_u32(mulc);   // hide the power of two: IMAD (FMA pipe) instead of SHF (ALU pipe)
 #endif
-        x.four = opaque_u32(4u);
-        x.hioff = ((t >> 4) & 1u) * 512u;
-        // ldmatrix.trans rows: matrix m = lane/8 -> (k half m&1, n chunk m>>1); row rr = lane%8.
-        const uint32_t rr = t & 7u, mk = (t >> 3) & 1u;
-        x.mn = (t >> 4) & 1u;
-        x.xrow = (mk * 8u + rr) * (uint32_t)(N / 8);          // + (64 j + 16 c) * cpr per k16 column
-        x.xsw = x_swz<NT>(rr);                                // swizzle depends on k % 8 == rr only
-        return x;
-    };
+    const uint32_t four = opaque_u32(4u);
+    (void)four;
+    constexpr uint32_t cpr = N / 8;
+    const uint32_t tbl_lane = (uint32_t)(r * G) * 1024u + (uint32_t)(lane >> 4) * 512u + (uint32_t)c * 128u;
+    // ldmatrix.trans rows: matrix m = lane/8 -> (k half m&1, n chunk m>>1); row rr = lane%8.
+    const uint32_t rr = lane & 7, mk = (lane >> 3) & 1, mn = (lane >> 4) & 1;
+    const uint32_t x_lane = ((mk * 8u + rr) + 16u * (uint32_t)c) * cpr * 16u + ((mn ^ x_swz<NT>(rr)) * 16u);
     // selector polynomial constants, read from smem so ptxas keeps them in registers
     const uint32_t selA = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];
     const uint32_t selB = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];
     const uint32_t selC = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 2];
-    constexpr uint32_t cpr = N / 8;
     float acc[4][NT][4];
     constexpr uint32_t kPart = 64u * N * 4u;                      // one fp32 64 x N partial
 
@@ -445,22 +463,18 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     uint32_t tA0[8], tA1[8], sA[8], tB0[8], tB1[8], sB[8];
     auto load_E = [&](uint32_t tb, int step) {   // table entries of step `step` (4 x 16 B per lane)
 #pragma unroll
-        for (int q = 0; q < 4; ++q) E[q] = lds_v4(tb + (uint32_t)(step >> 1) * 1024u + (uint32_t)(step & 1) * 64u + 16u * q);
+        for (int k = 0; k < 4; ++k) E[k] = lds_v4(tb + (uint32_t)(step >> 1) * 1024u + (uint32_t)(step & 1) * 64u + 16u * k);
     };
-    auto issue = [&](const Ctx &x, uint32_t (&t0)[8], uint32_t (&t1)[8], uint32_t (&s1)[8]) {   // value loads from E
+    auto issue = [&](uint32_t (&t0)[8], uint32_t (&t1)[8], uint32_t (&s1)[8]) {   // value loads from E
 #pragma unroll
         for (int k = 0; k < 8; ++k) {
             const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
             const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;   // (first value of the half) - 4 bytes
             // z = w << (30 - sh) as a multiply (FMA pipe): its top two bits are the lane's pair
             // y = (bit sh, bit sh+1) and popc(z) = c2 = MaskedPopCount + b0 + b1 (Alg. 2)
-            const uint32_t z = w * x.mulc;
+            const uint32_t z = w * mulc;
             const uint32_t a = A + 2u * __popc(z);        // &V[c2 - 2]
-#if SPINFER_PIPEMIX & 2
-            const uint32_t y = __umulhi(z, x.four);       // IMAD.HI (FMA pipe) instead of SHF (ALU pipe)
-#else
             const uint32_t y = z >> 30;
-#endif
             s1[k] = y * (y * selB + selA) + selC;          // selector polynomial (see kSelA)
             t0[k] = lds_u16(a);                            // V[c2 - 2]
             t1[k] = lds_u16(a + 2u);                       // V[c2 - 1]
@@ -480,52 +494,50 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             for (int nt = 0; nt < NT; ++nt) mma_16816(acc[trb + tt][nt], afr, bfr[nt][0], bfr[nt][1]);
         }
     };
-    // this warp's 16 entries of GT j (TCTiles c*4 .. c*4+3, all 4 BTs): 128 contiguous bytes
-    auto table_base = [&](const Ctx &x, int slot_) {
-        return sbase + prm.o_tbl + slot_ * prm.tbl_bytes + (uint32_t)(x.r * G) * 1024u + x.hioff + (uint32_t)x.c * 128u;
-    };
     const bool compute = !(dbg_mode(prm) & 1);
-    // Wait for a stage's data and table; if this warp has work in it, start its pipeline.
     constexpr bool kPipe = (KQ == 1);          // explicit cross-step software pipeline (8 consumer warps)
     const bool reuse0 = (dbg_mode(prm) & 4) != 0;   // experiment: pure consumer throughput on stage 0's data
-    auto load_x = [&](const Ctx &x, uint32_t xs, int j, uint32_t (&bfr)[NT][2]) {   // B fragments of GT j, TCTile column c
-        const uint32_t xk = xs + (x.xrow + (uint32_t)(64 * j + 16 * x.c) * cpr) * 16u;
+    auto load_x = [&](uint32_t xs, int j, uint32_t (&bfr)[NT][2]) {   // B fragments of GT j, TCTile column c
+        const uint32_t xk = xs + (uint32_t)(64 * j) * cpr * 16u;     // xs includes this lane's x_lane
         if constexpr (NT == 1) {
             ldsm_x2_trans(xk, bfr[0][0], bfr[0][1]);
         } else {
 #pragma unroll
-            for (int nt = 0; nt + 1 < NT; nt += 2)
-                ldsm_x4_trans(xk + (((uint32_t)nt + x.mn) ^ x.xsw) * 16u, bfr[nt][0], bfr[nt][1], bfr[nt + 1][0],
-                              bfr[nt + 1][1]);
-            if constexpr (NT % 2 == 1) ldsm_x2_trans(xk + (uint32_t)(NT - 1) * 16u, bfr[NT - 1][0], bfr[NT - 1][1]);
-        }
-    };
-    auto begin_stage = [&](const Ctx &x, const StageDesc &s, int si) {
-        if (!reuse0 || si == 0) {
-            // suspend rather than spin: a spinning consumer steals issue slots from the
-            // other 15 consumer warps that still have decode work
-            mbar_wait_sleep(bar_scan + 8 * s.slot(), s.par());   // implies full[slot] (see above)
-            if (x.cw == 0 && x.lane == 0) trace_ev(prm, p, si, 4);
-            if (x.cw == 0 && x.lane == 0) trace_ev(prm, p, si, 5);
-        }
-        if (kPipe && x.r < s.rows() && compute && x.q < s.g()) {
-            const uint32_t tb = table_base(x, reuse0 ? 0 : s.slot());
-            load_E(tb, 2 * x.q);
-            issue(x, tA0, tA1, sA);
-            load_E(tb, 2 * x.q + 1);
+            for (int nt = 0; nt + 1 < NT; nt += 2)     // chunk (nt + mn) ^ swz == (mn ^ swz) ^ nt for even nt
+                ldsm_x4_trans(xk ^ ((uint32_t)nt * 16u), bfr[nt][0], bfr[nt][1], bfr[nt + 1][0], bfr[nt + 1][1]);
+            if constexpr (NT % 2 == 1)
+                ldsm_x2_trans(xk - ((mn ^ x_swz<NT>(rr)) * 16u) + (uint32_t)(NT - 1) * 16u, bfr[NT - 1][0], bfr[NT - 1][1]);
         }
     };
     const uint32_t desc = sbase + prm.o_desc;
     auto rd = [&](int si) {   // volatile shared load: re-read, never kept live across the decode loop
-        const uint2 v = lds_v2(desc + 8u * (uint32_t)si);
-        return StageDesc{v.x, v.y};
+        const uint4 v = lds_v4(desc + 16u * (uint32_t)si);
+        return StageDesc{v.x, v.y, v.z, v.w};
+    };
+    auto begin_stage = [&](const StageDesc &s, int si) {
+        if (lane == 0) trace_ev(prm, p, si, warp, 0);
+        if (!reuse0 || si == 0) {
+            // suspend rather than spin: a spinning consumer steals issue slots from the
+            // other 15 consumer warps that still have decode work
+#if SPINFER_CONSSPIN
+            mbar_wait(bar_scan + 8 * s.slot(), s.par());
+#else
+            mbar_wait_sleep(bar_scan + 8 * s.slot(), s.par());   // implies full[slot] (see above)
+#endif
+            if (lane == 0) trace_ev(prm, p, si, warp, 1);
+        }
+        if (kPipe && r < s.rows() && compute && q < s.g()) {
+            const uint32_t tb = sbase + s.tbl + tbl_lane;
+            load_E(tb, 2 * q);
+            issue(tA0, tA1, sA);
+            load_E(tb, 2 * q + 1);
+        }
     };
     named_bar_sync(kDescBar, 32u * (kCW + 1));
-    auto nst = [&]() { return (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3]; };
-    if (kPipe && nst() > 0) begin_stage(ctx(), rd(0), 0);
-    for (int i = 0; i < nst(); ++i) {
-        const Ctx x = ctx();
-        const int q = x.q, c = x.c, r = x.r, cw = x.cw, lane = x.lane;
+    const int nst = (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3];
+    if (kPipe && nst > 0) begin_stage(rd(0), 0);
+    for (int i = 0; i < nst; ++i) {
+        const int cw = warp;
         {
             const StageDesc d = rd(i);
             if (d.zero()) {
@@ -536,49 +548,48 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
 #pragma unroll
                         for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
             }
-            if constexpr (!kPipe) begin_stage(x, d, i);
+            if constexpr (!kPipe) begin_stage(d, i);
         }
         const StageDesc d = rd(i);
-        const int g = d.g(), slot = d.slot();
+        const int g = d.g();
         if (d.rows() > r && compute && q < g && !kPipe) {
             // KQ = 2: 4 consumer warps per scheduler hide the latencies; one register set.
-            const uint32_t xs = sbase + prm.o_stage + (reuse0 ? 0 : slot) * prm.stage_bytes;
-            const uint32_t tb = table_base(x, reuse0 ? 0 : slot);
+            const uint32_t xs = sbase + d.stg + x_lane;
+            const uint32_t tb = sbase + d.tbl + tbl_lane;
             for (int j = q; j < g; j += KQ) {
-                if (cw == 0 && lane == 0) trace_ev(prm, p, i, 8 + j);
                 uint32_t bfr[NT][2];
-                load_x(x, xs, j, bfr);
+                load_x(xs, j, bfr);
 #pragma unroll
                 for (int h = 0; h < 2; ++h) {
                     load_E(tb, 2 * j + h);
-                    issue(x, tA0, tA1, sA);
+                    issue(tA0, tA1, sA);
                     assemble(tA0, tA1, sA, 2 * h, bfr);
                 }
             }
         } else if (d.rows() > r && compute && q < g) {
-            const uint32_t xs = sbase + prm.o_stage + (reuse0 ? 0 : slot) * prm.stage_bytes;
-            const uint32_t tb = table_base(x, reuse0 ? 0 : slot);
+            const uint32_t xs = sbase + d.stg + x_lane;
+            const uint32_t tb = sbase + d.tbl + tbl_lane;
             for (int j = q; j < g; j += KQ) {
                 uint32_t bfr[NT][2];
-                load_x(x, xs, j, bfr);
+                load_x(xs, j, bfr);
                 // step (j, first half): issue (j, second half) into B, prefetch the entries of
                 // this warp's next GT, assemble (j, first half) from A
-                issue(x, tB0, tB1, sB);
+                issue(tB0, tB1, sB);
                 if (j + KQ < g) load_E(tb, 2 * (j + KQ));
                 assemble(tA0, tA1, sA, 0, bfr);
                 // step (j, second half): issue the next step (A: next GT, or the next stage's first step)
                 if (j + KQ < g) {
-                    issue(x, tA0, tA1, sA);
+                    issue(tA0, tA1, sA);
                     load_E(tb, 2 * (j + KQ) + 1);
-                } else if (i + 1 < nst()) {
-                    begin_stage(x, rd(i + 1), i + 1);
+                } else if (i + 1 < nst) {
+                    begin_stage(rd(i + 1), i + 1);
                 }
                 assemble(tB0, tB1, sB, 2, bfr);
             }
-        } else if (kPipe && i + 1 < nst()) {
-            begin_stage(x, rd(i + 1), i + 1);
+        } else if (kPipe && i + 1 < nst) {
+            begin_stage(rd(i + 1), i + 1);
         }
-        if (cw == 0 && lane == 0) trace_ev(prm, p, i, 7);   // consumer warp 0 finished the stage's work
+        if (lane == 0) trace_ev(prm, p, i, cw, 2);   // decode done
         const StageDesc e = rd(i);
         const int rb = e.rb(), rows = e.rows();
         if (e.seg_end() && r < rows) {
@@ -587,7 +598,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             // Scratch = this stage's value region of GT row r: only row r's consumer warps read
             // it, so once they all pass the first barrier it is free (the slot is released below).
             const uint32_t bid = 1u + (uint32_t)r, bcnt = 128u * KQ;
-            const uint32_t scr = sbase + prm.o_stage + e.slot() * prm.stage_bytes + (r ? prm.st_v1 : prm.st_v0);
+            const uint32_t scr = sbase + e.stg + (r ? prm.st_v1 : prm.st_v0);
             named_bar_sync(bid, bcnt);
             auto put = [&](uint32_t slot_) {
 #pragma unroll
@@ -627,8 +638,9 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                 if (e.complete()) {
                     store_y<NT>(prm.Y, N, row_base, acc, lane);
                 } else {
-                    const int pf = unit_owner((long long)rb * KG, U, prm.P);
-                    const int pl = unit_owner((long long)(rb + 1) * KG - 1, U, prm.P);
+                    // split rowblock: park the fp32 partial in the workspace now (plain stores) and
+                    // combine after the main loop, so the fence/atomic/partial-load latency of the
+                    // fix-up never holds a ring slot (it used to stall the producer for ~us)
                     const int myslot = (rb == (int)(u0 / KG)) ? 0 : 1;
                     float4 *part = reinterpret_cast<float4 *>(prm.ws_part) + (((size_t)p * 2 + myslot) * kR + r) * (64 * N / 4);
 #pragma unroll
@@ -637,42 +649,65 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                         for (int nt = 0; nt < NT; ++nt)
                             part[(tr * NT + nt) * 32 + lane] =
                                 make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]);
-                    __threadfence();
-                    __syncwarp();
-                    int old = 0;
-                    if (lane == 0) old = atomicAdd(prm.ws_cnt + grow, 1);
-                    old = __shfl_sync(0xffffffffu, old, 0);
-                    if (old == pl - pf) {   // last contributor: sum all partials in CTA order
-                        __threadfence();
-#pragma unroll
-                        for (int tr = 0; tr < 4; ++tr)
-#pragma unroll
-                            for (int nt = 0; nt < NT; ++nt)
-#pragma unroll
-                                for (int q = 0; q < 4; ++q) acc[tr][nt][q] = 0.f;
-                        for (int q = pf; q <= pl; ++q) {
-                            const int sl = (rb == (int)(unit_start(q, U, prm.P) / KG)) ? 0 : 1;
-                            const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part) + (((size_t)q * 2 + sl) * kR + r) * (64 * N / 4);
-#pragma unroll
-                            for (int tr = 0; tr < 4; ++tr)
-#pragma unroll
-                                for (int nt = 0; nt < NT; ++nt) {
-                                    float4 v = ldg_cg_f4(pp + (tr * NT + nt) * 32 + lane);
-                                    acc[tr][nt][0] += v.x; acc[tr][nt][1] += v.y; acc[tr][nt][2] += v.z; acc[tr][nt][3] += v.w;
-                                }
-                        }
-                        store_y<NT>(prm.Y, N, row_base, acc, lane);
-                        if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed
-                    }
+                    if (lane == 0) reinterpret_cast<volatile int *>(smem)[kPendWord + 2 * r + myslot] = rb;
                 }
             }
         }
         __syncwarp();
         if (lane == 0 && !reuse0) {
             mbar_arrive(bar_empty + 8 * e.slot());   // frees the ring slot and its table
-            if (cw == 0) trace_ev(prm, p, i, 6);
+            trace_ev(prm, p, i, cw, 3);
         }
     }
+
+    if (lane == 0) trace_k(prm, p, warp, 2);
+    // ---------------------------------------------------------------- split-K fix-up
+    // (the paper's ReductionWorkspace): for each split rowblock this CTA contributed
+    // to, count the contribution; the last contributor sums all partials in CTA order
+    // (deterministic) and writes Y, then re-zeroes the counter.
+    {
+        if (c == 0 && q == 0) {
+            const int pend[2] = {reinterpret_cast<volatile int *>(smem)[kPendWord + 2 * r],
+                                 reinterpret_cast<volatile int *>(smem)[kPendWord + 2 * r + 1]};
+            if (pend[0] >= 0 || pend[1] >= 0) __threadfence();   // partial stores before the counts
+#pragma unroll
+            for (int k = 0; k < 2; ++k) {
+                const int rb = pend[k];
+                if (rb < 0) continue;
+                const int grow = kR * rb + r;
+                const int pf = unit_owner((long long)rb * KG, U, prm.P);
+                const int pl = unit_owner((long long)(rb + 1) * KG - 1, U, prm.P);
+                __syncwarp();
+                int old = 0;
+                if (lane == 0) old = atomicAdd(prm.ws_cnt + grow, 1);
+                old = __shfl_sync(0xffffffffu, old, 0);
+                if (old == pl - pf) {   // last contributor: sum all partials in CTA order
+                    __threadfence();
+                    float acc2[4][NT][4];
+#pragma unroll
+                    for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                        for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) acc2[tr][nt][e] = 0.f;
+                    for (int qq = pf; qq <= pl; ++qq) {
+                        const int sl = (rb == (int)(unit_start(qq, U, prm.P) / KG)) ? 0 : 1;
+                        const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part) + (((size_t)qq * 2 + sl) * kR + r) * (64 * N / 4);
+#pragma unroll
+                        for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt) {
+                                float4 v = ldg_cg_f4(pp + (tr * NT + nt) * 32 + lane);
+                                acc2[tr][nt][0] += v.x; acc2[tr][nt][1] += v.y; acc2[tr][nt][2] += v.z; acc2[tr][nt][3] += v.w;
+                            }
+                    }
+                    store_y<NT>(prm.Y, N, grow * 64, acc2, lane);
+                    if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed
+                }
+            }
+        }
+    }
+    if (lane == 0) trace_k(prm, p, warp, 3);
 }
 
 struct Plan {
@@ -756,7 +791,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         uint32_t st_v1 = st_v0 + vcap;
         uint32_t stage = align_up(st_v1 + vcap, 1024);   // slots stay 1024-aligned (X swizzle)
         // stage descriptors: at most one per unit, and no more than ceil(units/G) + rowblock splits
-        const uint32_t desc_bytes = align_up((uint32_t)(8 * std::min<long long>(upc, upc / G + upc / KG + 3)), 128);
+        const uint32_t desc_bytes = align_up((uint32_t)(16 * std::min<long long>(upc, upc / G + upc / KG + 3)), 128);
         uint32_t fixed = o_pre + pre_bytes + desc_bytes + 128 + 2048;   // +slack: t1 over-read, base and ring alignment
         stage += tbl;                                     // each ring slot carries its table (accounted with it)
         if ((long long)fixed + 2LL * stage > smem_max) continue;
@@ -826,7 +861,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     q.trace = nullptr;
     static long long *trace_buf = nullptr;
     const char *trace_path = getenv("SPINFER_TRACE");
-    const size_t trace_n = (size_t)kTraceCTAs * kTraceStages * kTraceEv;
+    const size_t trace_n = (size_t)kTraceCTAs * kTraceStages * kTraceW * kTraceEv;
     if (trace_path) {
         if (!trace_buf && cudaMalloc(&trace_buf, trace_n * 8) != cudaSuccess) return SPINFER_ECUDA;
         cudaMemsetAsync(trace_buf, 0, trace_n * 8, st);
@@ -841,7 +876,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
         default: break;
     }
     if (trace_path && rc == SPINFER_OK) {   // debug only: synchronous dump of the stage timeline
-        static long long host[kTraceCTAs * kTraceStages * kTraceEv];
+        static long long host[kTraceCTAs * kTraceStages * kTraceW * kTraceEv];
         cudaMemcpyAsync(host, trace_buf, sizeof(host), cudaMemcpyDeviceToHost, st);
         cudaStreamSynchronize(st);
         if (FILE *f = fopen(trace_path, "wb")) { fwrite(host, 1, sizeof(host), f); fclose(f); }
