@@ -86,12 +86,12 @@ struct Params {
     float *ws_part;
     int32_t *ws_cnt;
     int KG, MG;
-    long long U;
+    uint32_t U;                                 // units (rowblock x GT column); U * P < 2^32
     int P;
     int G, S;
     uint32_t stage_bytes, st_bm, st_v0, st_v1;  // stage slot size; offsets in a slot (X slab at 0)
     uint32_t tbl_bytes;
-    uint32_t o_pre, o_desc, o_tbl, o_stage;     // region offsets from the smem base
+    uint32_t o_desc, o_tbl, o_stage;            // region offsets from the smem base
     long long *trace;   // experiments only (SPINFER_TRACE): [kTraceCTAs][kTraceStages][8] clock64 stamps
     int dbg;            // experiments only (SPINFER_DEBUG_MODE): bit0 = consumers skip decode/MMA, bit1 = scan skips work
 };
@@ -125,26 +125,24 @@ __device__ __forceinline__ int dbg_mode(const Params &prm) {
 #endif
 }
 
-__device__ __forceinline__ long long unit_start(long long p, long long U, int P) { return p * U / P; }
-__device__ __forceinline__ int unit_owner(long long u, long long U, int P) {
-    return (int)(((u + 1) * (long long)P - 1) / U);
+// Stream-K partition in 32-bit arithmetic (the host guarantees U * P < 2^32).
+__device__ __forceinline__ int unit_start(int p, uint32_t U, int P) { return (int)((uint32_t)p * U / (uint32_t)P); }
+__device__ __forceinline__ int unit_owner(int u, uint32_t U, int P) {
+    return (int)(((uint32_t)(u + 1) * (uint32_t)P - 1u) / U);
 }
 
 // Stage iterator: every role walks the same deterministic stage sequence. All
-// per-stage bookkeeping is incremental and 32-bit (one 64-bit division at kernel start
-// only); loop-invariant sizes stay in the parameter bank, so the live state is a few
-// registers (16 consumer warps run at <= 96 registers; spills would go to L2 because the
-// shared-memory carve-out leaves almost no L1).
+// per-stage bookkeeping is incremental and 32-bit (one division at kernel start).
 struct StageIter {
     int du, du1;             // current unit offset from u0, and the CTA's unit count
     int rb, gc, g, rows;     // current stage: rowblock, first GT column, #units, #GT rows
     int i, slot;             // stage index within the CTA, smem ring slot
     uint32_t ph;             // ring parity ((i / S) & 1)
-    __device__ __forceinline__ void init(long long u0, long long u1, const Params &prm) {
+    __device__ __forceinline__ void init(int u0, int u1, const Params &prm) {
         du = 0;
-        du1 = (int)(u1 - u0);
-        rb = (int)(u0 / prm.KG);
-        gc = (int)(u0 - (long long)rb * prm.KG);
+        du1 = u1 - u0;
+        rb = (int)((uint32_t)u0 / (uint32_t)prm.KG);
+        gc = u0 - rb * prm.KG;
         i = 0; slot = 0; ph = 0;
         shape(prm);
     }
@@ -231,7 +229,7 @@ __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const 
 template <int NT>
 __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_constant__ Params prm) {
     constexpr int N = NT * 8;
-    constexpr int KQ = Cfg<NT>::KQ, kCW = Cfg<NT>::CW, kThreads = Cfg<NT>::Threads;
+    constexpr int KQ = Cfg<NT>::KQ, kCW = Cfg<NT>::CW;
     constexpr int kScanWarp = Cfg<NT>::ScanWarp, kProducerWarp = Cfg<NT>::ProducerWarp;
     // named barriers: 0 = __syncthreads, 1..kR = epilogue (per GT row), kDescBar = descriptors ready
     constexpr uint32_t kDescBar = 1 + kR;
@@ -242,16 +240,15 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     const uint32_t sbase = smem_u32(smem);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int p = blockIdx.x;
-    const long long U = prm.U;
-    const int KG = prm.KG, G = prm.G, S = prm.S, MG = prm.MG;
-    const long long u0 = unit_start(p, U, prm.P), u1 = unit_start(p + 1, U, prm.P);
+    const uint32_t U = prm.U;
+    const int KG = prm.KG, G = prm.G, S = prm.S;
+    const int u0 = unit_start(p, U, prm.P), u1 = unit_start(p + 1, U, prm.P);
 
     // barriers: full[S], empty[S], scanned[2], tbl_empty[2]
     const uint32_t bar_full = sbase, bar_empty = sbase + 8 * kMaxStages;
     // barriers: full[S] (data landed), empty[S] (consumers done), scanned[S] (table written;
     // the scan warps acquired full[s] first, so consumers wait on scanned[s] only)
     const uint32_t bar_scan = sbase + 16 * kMaxStages;
-    int4 *pre = reinterpret_cast<int4 *>(smem + prm.o_pre);
 
     if (lane == 0) trace_k(prm, p, warp, 0);
     if (threadIdx.x == 0) {
@@ -268,19 +265,21 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 2] = kSelC;
         for (int k = 0; k < 2 * kR; ++k) reinterpret_cast<int *>(smem)[kPendWord + k] = -1;
     }
-    // Preload this CTA's GTileOffset entries: pre[u-u0] = {start_r0, end_r0, start_r1, end_r1}.
-    for (long long i = threadIdx.x; i < u1 - u0; i += kThreads) {
-        long long u = u0 + i;
-        int rb = (int)(u / KG), gc = (int)(u % KG);
-        int4 v = make_int4(0, 0, 0, 0);
-        long long g0 = (long long)(kR * rb) * KG + gc;
+    // The producer's first GTileOffset reads go out before the block barrier (no shared state).
+    StageIter pit;
+    int4 poff = make_int4(0, 0, 0, 0);   // {start, end} of the stage's values, GT rows 0 and 1
+    auto load_off = [&](const StageIter &sg) {
+        const int g0 = kR * sg.rb * KG + sg.gc;
+        int4 v;
         v.x = __ldg(prm.off + g0);
-        v.y = __ldg(prm.off + g0 + 1);
-        if (kR * rb + 1 < MG) {
-            v.z = __ldg(prm.off + g0 + KG);
-            v.w = __ldg(prm.off + g0 + KG + 1);
-        }
-        pre[i] = v;
+        v.y = __ldg(prm.off + g0 + sg.g);
+        v.z = sg.rows > 1 ? __ldg(prm.off + g0 + KG) : 0;
+        v.w = sg.rows > 1 ? __ldg(prm.off + g0 + KG + sg.g) : 0;
+        return v;
+    };
+    if (warp == kProducerWarp && lane == 0) {
+        pit.init(u0, u1, prm);
+        if (pit.valid()) poff = load_off(pit);
     }
     __syncthreads();
     if (lane == 0) trace_k(prm, p, warp, 1);
@@ -290,28 +289,32 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         if (lane != 0) return;
         const uint64_t pol_w = policy_evict_first();
         const uint32_t xbytes = 64u * N * 2u;          // one GroupTile column of X
-        StageIter it;
-        for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
-            const StageIter &sg = it;
-            const long long u = u0 + it.du;
-            const int i = it.i, slot = it.slot;
+        for (; pit.valid();) {
+            const StageIter sg = pit;
+            const int i = sg.i, slot = sg.slot;
             if ((dbg_mode(prm) & 4) && i > 0) break;   // experiment: consumers reuse stage 0 forever
             trace_ev(prm, p, i, warp, 0);
-            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, it.par() ^ 1u);
+            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, sg.par() ^ 1u);
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const uint32_t fb = bar_full + 8 * slot;
-            const int4 ps = pre[u - u0], pe = pre[u - u0 + sg.g - 1];
-            const uint32_t vb0 = 2u * (uint32_t)(pe.y - ps.x);
-            const uint32_t vb1 = sg.rows > 1 ? 2u * (uint32_t)(pe.w - ps.z) : 0u;
             const uint32_t bmb = (uint32_t)sg.g * 512u;
-            mbar_arrive_expect_tx(fb, vb0 + vb1 + (uint32_t)sg.rows * bmb + (uint32_t)sg.g * xbytes);
-            if (vb0) bulk_g2s(st + prm.st_v0, prm.vals + ps.x, vb0, fb, pol_w);
-            if (vb1) bulk_g2s(st + prm.st_v1, prm.vals + ps.z, vb1, fb, pol_w);
+            // X and bitmaps first (no offsets needed); the arrive comes with the value bytes last,
+            // so the phase cannot complete before every transaction is registered
+            mbar_expect_tx(fb, (uint32_t)sg.rows * bmb + (uint32_t)sg.g * xbytes);
             for (int r = 0; r < sg.rows; ++r)
                 bulk_g2s(st + prm.st_bm + (uint32_t)(r * G) * 512u,
                          prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc) * 64, bmb, fb, pol_w);
             // X slab rows [64 gc, 64 (gc + g)): L2-resident (every CTA reads X), default policy
             for (int j = 0; j < sg.g; ++j) tma_2d_g2s(st + (uint32_t)j * xbytes, &prm.tmap_x, 0, 64 * (sg.gc + j), fb);
+            const int4 o = poff;
+            const uint32_t vb0 = 2u * (uint32_t)(o.y - o.x);
+            const uint32_t vb1 = sg.rows > 1 ? 2u * (uint32_t)(o.w - o.z) : 0u;
+            if (vb0) bulk_g2s(st + prm.st_v0, prm.vals + o.x, vb0, fb, pol_w);
+            if (vb1) bulk_g2s(st + prm.st_v1, prm.vals + o.z, vb1, fb, pol_w);
+            mbar_arrive_expect_tx(fb, vb0 + vb1);
+            // next stage's offsets: in flight while this warp waits for a free slot
+            pit.next(prm);
+            if (pit.valid()) poff = load_off(pit);
             trace_ev(prm, p, i, warp, 1);
         }
         trace_k(prm, p, warp, 3);
@@ -355,7 +358,6 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         StageIter it;
         for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
             const StageIter &sg = it;
-            const long long u = u0 + it.du;
             const int i = it.i, slot = it.slot;
             if ((dbg_mode(prm) & 4) && i > 0) break;
             // suspend (not spin) while waiting: these warps have the highest scheduling
@@ -397,15 +399,14 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                 for (int q = 0; q < Q; ++q) incl[q] += (lane >= o) ? y[q] : 0u;
             }
             uint32_t tot_a[Q];
-#pragma unroll
-            for (int q = 0; q < Q; ++q) tot_a[q] = __shfl_sync(0xffffffffu, incl[q], 31) & 0xFFFFu;
-            const int4 p0 = pre[u - u0];
+            int rel = 0;   // GT j's first value within the row's chunk: earlier GTs' counts, each padded
+                           // to a multiple of 8 values (the GTileOffset rule, encode.cu)
 #pragma unroll
             for (int q = 0; q < Q; ++q) {
+                const uint32_t t = __shfl_sync(0xffffffffu, incl[q], 31);
+                tot_a[q] = t & 0xFFFFu;
                 const int j = q;
                 if (work && r < sg.rows && j < sg.g) {
-                    const int4 pj = pre[u - u0 + j];
-                    const int rel = r ? (pj.z - p0.z) : (pj.x - p0.x);          // GT j's values in the chunk
                     const uint32_t vsm = st + (r ? prm.st_v1 : prm.st_v0);
                     const uint32_t excl = incl[q] - packed[q];
                     const uint32_t ea = excl & 0xFFFFu, eb = tot_a[q] + (excl >> 16);   // PopCount prefix
@@ -418,6 +419,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                     sts_v2(te + 256u, bb[q].x, Ab - 4u);
                     sts_v2(te + 768u, bb[q].y, Ab - 4u + 2u * __popc(bb[q].x));
                 }
+                rel += (int)(((t & 0xFFFFu) + (t >> 16) + 7u) & ~7u);
             }
             // one arrive per warp: every mbarrier event wakes all sleeping waiters of the CTA,
             // so 64 per-thread arrivals would cost each waiting consumer ~60 extra polls
@@ -641,7 +643,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                     // split rowblock: park the fp32 partial in the workspace now (plain stores) and
                     // combine after the main loop, so the fence/atomic/partial-load latency of the
                     // fix-up never holds a ring slot (it used to stall the producer for ~us)
-                    const int myslot = (rb == (int)(u0 / KG)) ? 0 : 1;
+                    const int myslot = (rb == u0 / KG) ? 0 : 1;
                     float4 *part = reinterpret_cast<float4 *>(prm.ws_part) + (((size_t)p * 2 + myslot) * kR + r) * (64 * N / 4);
 #pragma unroll
                     for (int tr = 0; tr < 4; ++tr)
@@ -675,8 +677,8 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                 const int rb = pend[k];
                 if (rb < 0) continue;
                 const int grow = kR * rb + r;
-                const int pf = unit_owner((long long)rb * KG, U, prm.P);
-                const int pl = unit_owner((long long)(rb + 1) * KG - 1, U, prm.P);
+                const int pf = unit_owner(rb * KG, U, prm.P);
+                const int pl = unit_owner((rb + 1) * KG - 1, U, prm.P);
                 __syncwarp();
                 int old = 0;
                 if (lane == 0) old = atomicAdd(prm.ws_cnt + grow, 1);
@@ -691,7 +693,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
 #pragma unroll
                             for (int e = 0; e < 4; ++e) acc2[tr][nt][e] = 0.f;
                     for (int qq = pf; qq <= pl; ++qq) {
-                        const int sl = (rb == (int)(unit_start(qq, U, prm.P) / KG)) ? 0 : 1;
+                        const int sl = (rb == unit_start(qq, U, prm.P) / KG) ? 0 : 1;
                         const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part) + (((size_t)qq * 2 + sl) * kR + r) * (64 * N / 4);
 #pragma unroll
                         for (int tr = 0; tr < 4; ++tr)
@@ -729,7 +731,7 @@ int choose_P(long long U) {
     // SPINFER_MAX_CTAS caps the persistent grid (tests use it to force many stages per CTA)
     if (const char *e = getenv("SPINFER_MAX_CTAS")) { long long v = atoll(e); if (v > 0 && v < cap) cap = v; }
     long long P = std::min(cap, U);
-    // keep the preloaded offsets (16 B per unit) within 16 KiB of shared memory
+    // keep the per-CTA stage descriptors (<= 16 B per unit) within a few KiB of shared memory
     while ((U + P - 1) / P > 1024) P += num_sms();
     return (int)std::max(1LL, P);
 }
@@ -768,17 +770,18 @@ int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N) {
 bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
     const int MG = M / kGT, KG = K / kGT;
     const int nRB = (MG + kR - 1) / kR;
-    pl->U = (long long)nRB * KG;
-    pl->P = choose_P(pl->U);
-    const long long upc = (pl->U + pl->P - 1) / pl->P;
+    const long long U = (long long)nRB * KG;
+    pl->P = choose_P(U);
+    if ((unsigned long long)U * (unsigned long long)pl->P >= (1ull << 32)) return false;   // 32-bit unit math
+    pl->U = U;
+    const long long upc = (U + pl->P - 1) / pl->P;
     int dev = 0, smem_max = 232448;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     cudaGetLastError();
     int maxv = max_gt_values > 0 ? max_gt_values : 4096;
     maxv = std::min(4096, (maxv + 7) & ~7);
-    const uint32_t o_pre = 256;
-    const uint32_t pre_bytes = align_up((uint32_t)(16 * upc), 128);
+    const uint32_t o_desc = 256;
     int gmax = kMaxG, smax = kMaxStages;
     if (const char *e = getenv("SPINFER_G")) gmax = std::max(1, std::min(kMaxG, atoi(e)));
     if (const char *e = getenv("SPINFER_S")) smax = std::max(2, std::min(kMaxStages, atoi(e)));
@@ -792,7 +795,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         uint32_t stage = align_up(st_v1 + vcap, 1024);   // slots stay 1024-aligned (X swizzle)
         // stage descriptors: at most one per unit, and no more than ceil(units/G) + rowblock splits
         const uint32_t desc_bytes = align_up((uint32_t)(16 * std::min<long long>(upc, upc / G + upc / KG + 3)), 128);
-        uint32_t fixed = o_pre + pre_bytes + desc_bytes + 128 + 2048;   // +slack: t1 over-read, base and ring alignment
+        uint32_t fixed = o_desc + desc_bytes + 128 + 2048;   // +slack: t1 over-read, base and ring alignment
         stage += tbl;                                     // each ring slot carries its table (accounted with it)
         if ((long long)fixed + 2LL * stage > smem_max) continue;
         int S = (int)std::min<long long>(smax, ((long long)smem_max - fixed) / stage);
@@ -800,12 +803,11 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
         pl->G = G;
         pl->S = S;
         Params &q = pl->prm;
-        q.KG = KG; q.MG = MG; q.U = pl->U; q.P = pl->P; q.G = G; q.S = S;
+        q.KG = KG; q.MG = MG; q.U = (uint32_t)U; q.P = pl->P; q.G = G; q.S = S;
         stage -= tbl;
         q.stage_bytes = stage; q.st_bm = st_bm; q.st_v0 = st_v0; q.st_v1 = st_v1;
         q.tbl_bytes = tbl;
-        q.o_pre = o_pre;
-        q.o_desc = o_pre + pre_bytes;
+        q.o_desc = o_desc;
         q.o_tbl = q.o_desc + desc_bytes;
         q.o_stage = align_up(q.o_tbl + (uint32_t)S * tbl, 1024);
         pl->smem = (size_t)q.o_stage + (size_t)S * stage + 128 + 1024;   // +1024: runtime base alignment
