@@ -538,10 +538,13 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     named_bar_sync(kDescBar, 32u * (kCW + 1));
     const int nst = (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3];
     if (kPipe && nst > 0) begin_stage(rd(0), 0);
+    // the next stage's descriptor is fetched during the current stage's decode (a shared load
+    // at a stage boundary waits behind the decode traffic in the MIO queue)
+    StageDesc dn = rd(0);
     for (int i = 0; i < nst; ++i) {
         const int cw = warp;
+        const StageDesc d = dn;
         {
-            const StageDesc d = rd(i);
             if (d.zero()) {
 #pragma unroll
                 for (int a = 0; a < 4; ++a)
@@ -552,7 +555,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             }
             if constexpr (!kPipe) begin_stage(d, i);
         }
-        const StageDesc d = rd(i);
+        if (i + 1 < nst) dn = rd(i + 1);
         const int g = d.g();
         if (d.rows() > r && compute && q < g && !kPipe) {
             // KQ = 2: 4 consumer warps per scheduler hide the latencies; one register set.
@@ -592,7 +595,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             begin_stage(rd(i + 1), i + 1);
         }
         if (lane == 0) trace_ev(prm, p, i, cw, 2);   // decode done
-        const StageDesc e = rd(i);
+        const StageDesc e = d;
         const int rb = e.rb(), rows = e.rows();
         if (e.seg_end() && r < rows) {
             // -------------------------------------------------------- epilogue
