@@ -35,15 +35,16 @@ def up_to_date() -> bool:
 
 
 LIB_INSTR = os.path.join(PKG, "libspinfer_instr.so")   # experiments only (stage trace, debug modes)
+LIB_DBG = os.path.join(PKG, "libspinfer_dbg.so")       # experiments only (debug modes, no trace)
 
 
-def build(force: bool = False, verbose: bool = False, instrumented: bool = False) -> str:
-    out = LIB_INSTR if instrumented else LIB
+def build(force: bool = False, verbose: bool = False, instrumented: int = 0) -> str:
+    out = {0: LIB, 1: LIB_INSTR, 2: LIB_DBG}[int(instrumented)]
     if not force and not instrumented and up_to_date():
         return LIB
     cmd = [NVCC, *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), *sources(), "-o", out + ".tmp"]
     if instrumented:
-        cmd.append("-DSPINFER_INSTRUMENT=1")
+        cmd.append(f"-DSPINFER_INSTRUMENT={int(instrumented)}")
     if verbose:
         cmd[1:1] = ["-Xptxas", "-v"]
     subprocess.check_call(cmd)
@@ -52,4 +53,5 @@ def build(force: bool = False, verbose: bool = False, instrumented: bool = False
 
 
 if __name__ == "__main__":
-    print(build(force=True, verbose="-v" in sys.argv, instrumented="--instrumented" in sys.argv))
+    print(build(force=True, verbose="-v" in sys.argv,
+                instrumented=1 if "--instrumented" in sys.argv else 2 if "--debug-modes" in sys.argv else 0))

@@ -49,9 +49,10 @@ constexpr int kScanWarps = kR;      // one scan warp per GT row of the rowblock
 template <int NT> struct Cfg {
     static constexpr int KQ = (NT <= 2 && !SPINFER_FORCE_KQ1) ? 2 : 1;
     static constexpr int CW = kR * 4 * KQ;                        // consumer warps
-    static constexpr int ScanWarp = CW;                           // warp ids: the scheduler favours the
-    static constexpr int ProducerWarp = CW + kScanWarps;          // highest id, so roles go on top
-    static constexpr int Threads = 32 * (CW + kScanWarps + 1);
+    static constexpr int FixWarp = CW;                            // warp ids: the scheduler favours the
+    static constexpr int ScanWarp = CW + 1;                       // highest id, so roles go on top
+    static constexpr int ProducerWarp = CW + 1 + kScanWarps;
+    static constexpr int Threads = 32 * (CW + kScanWarps + 2);
 };
 constexpr int kMaxStages = 8;
 #ifndef SPINFER_SCANSPIN
@@ -68,7 +69,6 @@ constexpr int kMaxStages = 8;
 #endif
 constexpr int kMaxG = SPINFER_MAXG;  // max GroupTile columns per stage (the scan unrolls over it)
 constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector-table constants
-constexpr int kPendWord = 52;       // smem words 52..55: pending split-K fix-ups [GT row][first/last segment]
 constexpr int kTraceCTAs = 4, kTraceStages = 64, kTraceW = 20, kTraceEv = 4;   // stage 63 = kernel-level events
 // Workspace = [fix-up counters: one int32 per GT row, fixed-size region][split-K partials].
 // The counter region has the same size for every shape so that one zeroed
@@ -97,7 +97,8 @@ struct Params {
 };
 
 // Experiment instrumentation (stage timeline, debug modes) is compiled in only with
-// -DSPINFER_INSTRUMENT=1 (tools/build_instrumented.sh); the product build has none of it.
+// -DSPINFER_INSTRUMENT=1 (stage trace + debug modes) or =2 (debug modes only: trace stores
+// slow down the traced CTAs, which then set the kernel time); the product build has none of it.
 #ifndef SPINFER_INSTRUMENT
 #define SPINFER_INSTRUMENT 0
 #endif
@@ -106,13 +107,13 @@ struct Params {
 // ev0 wait start, ev1 copies issued. Stage kTraceStages-1: ev0 entry, ev1 after the initial
 // __syncthreads, ev2 main loop done, ev3 exit.
 __device__ __forceinline__ void trace_ev(const Params &prm, int p, int i, int w, int ev) {
-#if SPINFER_INSTRUMENT
+#if SPINFER_INSTRUMENT == 1
     if (prm.trace && p < kTraceCTAs && i < kTraceStages - 1 && w < kTraceW)
         prm.trace[(((size_t)p * kTraceStages + i) * kTraceW + w) * kTraceEv + ev] = clock64();
 #endif
 }
 __device__ __forceinline__ void trace_k(const Params &prm, int p, int w, int ev) {
-#if SPINFER_INSTRUMENT
+#if SPINFER_INSTRUMENT == 1
     if (prm.trace && p < kTraceCTAs && w < kTraceW)
         prm.trace[(((size_t)p * kTraceStages + kTraceStages - 1) * kTraceW + w) * kTraceEv + ev] = clock64();
 #endif
@@ -131,34 +132,64 @@ __device__ __forceinline__ int unit_owner(int u, uint32_t U, int P) {
     return (int)(((uint32_t)(u + 1) * (uint32_t)P - 1u) / U);
 }
 
-// Stage iterator: every role walks the same deterministic stage sequence. All
-// per-stage bookkeeping is incremental and 32-bit (one division at kernel start).
+// Stage iterator: every role walks the same deterministic stage sequence. A CTA's unit
+// range [u0, u1) is processed in the order: A = the tail of the rowblock it starts inside
+// (split with the previous CTA), C = the head of the rowblock it ends inside (split with
+// the next CTA), then the full rowblocks in between. The split segments, whose results need
+// the cross-CTA fix-up, are therefore finished early and their fix-up latency hides behind
+// the full rowblocks; every CTA ends on a complete rowblock (plain Y stores).
+// Per-stage bookkeeping is incremental 32-bit arithmetic (a division per part switch).
 struct StageIter {
-    int du, du1;             // current unit offset from u0, and the CTA's unit count
+    int u, ue, us;           // current unit, end and start of the current part
+    int ns0, ne0, ns1, ne1;  // remaining parts, in order (empty: start == end)
     int rb, gc, g, rows;     // current stage: rowblock, first GT column, #units, #GT rows
     int i, slot;             // stage index within the CTA, smem ring slot
     uint32_t ph;             // ring parity ((i / S) & 1)
     __device__ __forceinline__ void init(int u0, int u1, const Params &prm) {
-        du = 0;
-        du1 = u1 - u0;
-        rb = (int)((uint32_t)u0 / (uint32_t)prm.KG);
-        gc = u0 - rb * prm.KG;
+        const int KG = prm.KG;
+        const int a_end = (u0 % KG) ? min(u1, (u0 / KG + 1) * KG) : u0;          // A = [u0, a_end)
+        const int c_beg = (u1 % KG) ? max(a_end, (u1 / KG) * KG) : u1;           // C = [c_beg, u1)
+        // parts in order A, C, M = [a_end, c_beg); empty ones dropped (no arrays: no local memory)
+        int q0s = u1, q0e = u1, q1s = u1, q1e = u1, q2s = u1, q2e = u1, k = 0;
+        auto push = [&](int s_, int e_) {
+            if (s_ >= e_) return;
+            if (k == 0) { q0s = s_; q0e = e_; } else if (k == 1) { q1s = s_; q1e = e_; } else { q2s = s_; q2e = e_; }
+            ++k;
+        };
+        push(u0, a_end);
+        push(c_beg, u1);
+        push(a_end, c_beg);
+        ns0 = q1s; ne0 = q1e; ns1 = q2s; ne1 = q2e;
         i = 0; slot = 0; ph = 0;
+        part(q0s, q0e, prm);
+    }
+    __device__ __forceinline__ void part(int s0, int e0, const Params &prm) {
+        u = s0; us = s0; ue = e0;
+        rb = (int)((uint32_t)u / (uint32_t)prm.KG);
+        gc = u - rb * prm.KG;
         shape(prm);
     }
     __device__ __forceinline__ void shape(const Params &prm) {
-        g = min(min(prm.G, prm.KG - gc), du1 - du);
+        g = min(min(prm.G, prm.KG - gc), ue - u);
         rows = min(kR, prm.MG - kR * rb);
     }
-    __device__ __forceinline__ bool valid() const { return du < du1; }
+    __device__ __forceinline__ bool valid() const { return u < ue; }
     __device__ __forceinline__ uint32_t par() const { return ph; }
+    __device__ __forceinline__ bool seg_first() const { return u == us || gc == 0; }
+    __device__ __forceinline__ bool seg_last(const Params &prm) const { return gc + g == prm.KG || u + g == ue; }
     __device__ __forceinline__ void next(const Params &prm) {
-        du += g;
+        u += g;
         gc += g;
         if (gc == prm.KG) { gc = 0; ++rb; }
         ++i;
         if (++slot == prm.S) { slot = 0; ph ^= 1u; }
-        shape(prm);
+        if (u == ue && ns0 < ne0) {
+            const int s0 = ns0, e0 = ne0;
+            ns0 = ns1; ne0 = ne1; ns1 = ne1;
+            part(s0, e0, prm);
+        } else {
+            shape(prm);
+        }
     }
 };
 
@@ -226,11 +257,40 @@ __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const 
         }
 }
 
+// Last contributor of a split rowblock: sum every contributor's fp32 partial in CTA order
+// (deterministic; its own partial included), write Y, re-zero the counter.
+template <int NT>
+__device__ __forceinline__ void fixup_sum(const Params &prm, int rb, int r, int pf, int pl, int lane) {
+    constexpr int N = NT * 8;
+    __threadfence();
+    float acc[4][NT][4];
+#pragma unroll
+    for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[tr][nt][e] = 0.f;
+    for (int qq = pf; qq <= pl; ++qq) {
+        const int sl = (rb == unit_start(qq, prm.U, prm.P) / prm.KG) ? 0 : 1;
+        const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part) + (((size_t)qq * 2 + sl) * kR + r) * (64 * N / 4);
+#pragma unroll
+        for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) {
+                float4 v = ldg_cg_f4(pp + (tr * NT + nt) * 32 + lane);
+                acc[tr][nt][0] += v.x; acc[tr][nt][1] += v.y; acc[tr][nt][2] += v.z; acc[tr][nt][3] += v.w;
+            }
+    }
+    const int grow = kR * rb + r;
+    store_y<NT>(prm.Y, N, grow * 64, acc, lane);
+    if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed
+}
+
 template <int NT>
 __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_constant__ Params prm) {
     constexpr int N = NT * 8;
     constexpr int KQ = Cfg<NT>::KQ, kCW = Cfg<NT>::CW;
-    constexpr int kScanWarp = Cfg<NT>::ScanWarp, kProducerWarp = Cfg<NT>::ProducerWarp;
+    constexpr int kScanWarp = Cfg<NT>::ScanWarp, kProducerWarp = Cfg<NT>::ProducerWarp, kFixWarp = Cfg<NT>::FixWarp;
     // named barriers: 0 = __syncthreads, 1..kR = epilogue (per GT row), kDescBar = descriptors ready
     constexpr uint32_t kDescBar = 1 + kR;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -249,6 +309,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     // barriers: full[S] (data landed), empty[S] (consumers done), scanned[S] (table written;
     // the scan warps acquired full[s] first, so consumers wait on scanned[s] only)
     const uint32_t bar_scan = sbase + 16 * kMaxStages;
+    const uint32_t bar_fix = sbase + 208;   // [split segment A/C][GT row]: partial parked (32 lanes)
 
     if (lane == 0) trace_k(prm, p, warp, 0);
     if (threadIdx.x == 0) {
@@ -257,13 +318,13 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             mbar_init(bar_empty + 8 * s, kCW);
         }
         for (int s = 0; s < S; ++s) mbar_init(bar_scan + 8 * s, kScanWarps);   // one elected arrive per scan warp
+        for (int k = 0; k < 2 * kR; ++k) mbar_init(bar_fix + 8 * k, 32);
         fence_barrier_init();
         // SMBD selector-table constants, read back into registers by every consumer thread so
         // ptxas keeps them live in registers instead of re-materialising them per PRMT.
         reinterpret_cast<uint32_t *>(smem)[kConstWord] = kSelA;
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = kSelB;
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 2] = kSelC;
-        for (int k = 0; k < 2 * kR; ++k) reinterpret_cast<int *>(smem)[kPendWord + k] = -1;
     }
     // The producer's first GTileOffset reads go out before the block barrier (no shared state).
     StageIter pit;
@@ -321,6 +382,33 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         return;
     }
 
+    if (warp == kFixWarp) {
+        // ------------------------------------------------------------ split-K fix-up
+        // At most two split segments per CTA (A: tail of the first rowblock, C: head of the
+        // last), processed first in StageIter order; for each and each GT row the reducing
+        // consumer parks its partial and arrives on bar_fix[seg][row].
+        const int a_rb = u0 / KG, c_rb = (u1 - 1) / KG;
+        const bool has_a = (u0 % KG) != 0;
+        const bool has_c = (u1 % KG) != 0 && !(has_a && c_rb == a_rb);
+        for (int sgi = 0; sgi < 2; ++sgi) {
+            if (!(sgi == 0 ? has_a : has_c)) continue;
+            const int rb = sgi == 0 ? a_rb : c_rb;
+            const int myslot = (rb == u0 / KG) ? 0 : 1;
+            const int rows = min(kR, prm.MG - kR * rb);
+            for (int r = 0; r < rows; ++r) {
+                mbar_wait_sleep(bar_fix + 8u * (uint32_t)(2 * myslot + r), 0u);
+                __threadfence();   // cumulative: the consumer's partial stores before the count
+                const int pf = unit_owner(rb * KG, U, prm.P);
+                const int pl = unit_owner((rb + 1) * KG - 1, U, prm.P);
+                int old = 0;
+                if (lane == 0) old = atomicAdd(prm.ws_cnt + kR * rb + r, 1);
+                old = __shfl_sync(0xffffffffu, old, 0);
+                if (old == pl - pf) fixup_sum<NT>(prm, rb, r, pf, pl, lane);   // last contributor
+            }
+        }
+        return;
+    }
+
     if (warp >= kScanWarp && warp < kScanWarp + kScanWarps) {
         // ------------------------------------------------------------ scan
         // Table per staged GT (r, j), 1024 B: [lane-half h][BT in GT storage order] {w, A},
@@ -338,9 +426,9 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                 int n = 0;
                 bool full_start = false;
                 for (d.init(u0, u1, prm); d.valid(); d.next(prm), ++n) {
-                    const bool zero = (d.gc == 0 || d.du == 0);
+                    const bool zero = d.seg_first();
                     if (zero) full_start = (d.gc == 0);
-                    const bool seg_end = (d.gc + d.g == KG) || (d.du + d.g == d.du1);
+                    const bool seg_end = d.seg_last(prm);
                     const bool complete = seg_end && full_start && (d.gc + d.g == KG);
                     const uint32_t w0 = (uint32_t)d.rb | ((uint32_t)d.slot << 20) | (d.ph << 24) | ((uint32_t)zero << 25) |
                                         ((uint32_t)seg_end << 26) | ((uint32_t)complete << 27) |
@@ -536,7 +624,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         }
     };
     named_bar_sync(kDescBar, 32u * (kCW + 1));
-    const int nst = (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3];
+    const int nst = (dbg_mode(prm) & 16) ? 0 : (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3];
     if (kPipe && nst > 0) begin_stage(rd(0), 0);
     // the next stage's descriptor is fetched during the current stage's decode (a shared load
     // at a stage boundary waits behind the decode traffic in the MIO queue)
@@ -597,7 +685,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         if (lane == 0) trace_ev(prm, p, i, cw, 2);   // decode done
         const StageDesc e = d;
         const int rb = e.rb(), rows = e.rows();
-        if (e.seg_end() && r < rows) {
+        if (e.seg_end() && r < rows && !(dbg_mode(prm) & 8)) {   // experiment bit 8: no epilogue
             // -------------------------------------------------------- epilogue
             // (1) reduce the 4*KQ partials of GT row r into warp (c = 0, q = 0), tree via smem.
             // Scratch = this stage's value region of GT row r: only row r's consumer warps read
@@ -643,9 +731,11 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                 if (e.complete()) {
                     store_y<NT>(prm.Y, N, row_base, acc, lane);
                 } else {
-                    // split rowblock: park the fp32 partial in the workspace now (plain stores) and
-                    // combine after the main loop, so the fence/atomic/partial-load latency of the
-                    // fix-up never holds a ring slot (it used to stall the producer for ~us)
+                    // split rowblock (split-K fix-up, the paper's ReductionWorkspace P:231): park the
+                    // fp32 partial; the fix-up warp counts it and the last contributor sums all
+                    // partials in CTA order (deterministic), writes Y and re-zeroes the counter.
+                    // Split segments are a CTA's first stages (StageIter order), so the fix-up
+                    // latency hides behind the full rowblocks.
                     const int myslot = (rb == u0 / KG) ? 0 : 1;
                     float4 *part = reinterpret_cast<float4 *>(prm.ws_part) + (((size_t)p * 2 + myslot) * kR + r) * (64 * N / 4);
 #pragma unroll
@@ -654,7 +744,8 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                         for (int nt = 0; nt < NT; ++nt)
                             part[(tr * NT + nt) * 32 + lane] =
                                 make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]);
-                    if (lane == 0) reinterpret_cast<volatile int *>(smem)[kPendWord + 2 * r + myslot] = rb;
+                    // hand the rest (fence, count, last-contributor sum) to the fix-up warp
+                    mbar_arrive(bar_fix + 8u * (uint32_t)(2 * myslot + r));
                 }
             }
         }
@@ -666,52 +757,6 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     }
 
     if (lane == 0) trace_k(prm, p, warp, 2);
-    // ---------------------------------------------------------------- split-K fix-up
-    // (the paper's ReductionWorkspace): for each split rowblock this CTA contributed
-    // to, count the contribution; the last contributor sums all partials in CTA order
-    // (deterministic) and writes Y, then re-zeroes the counter.
-    {
-        if (c == 0 && q == 0) {
-            const int pend[2] = {reinterpret_cast<volatile int *>(smem)[kPendWord + 2 * r],
-                                 reinterpret_cast<volatile int *>(smem)[kPendWord + 2 * r + 1]};
-            if (pend[0] >= 0 || pend[1] >= 0) __threadfence();   // partial stores before the counts
-#pragma unroll
-            for (int k = 0; k < 2; ++k) {
-                const int rb = pend[k];
-                if (rb < 0) continue;
-                const int grow = kR * rb + r;
-                const int pf = unit_owner(rb * KG, U, prm.P);
-                const int pl = unit_owner((rb + 1) * KG - 1, U, prm.P);
-                __syncwarp();
-                int old = 0;
-                if (lane == 0) old = atomicAdd(prm.ws_cnt + grow, 1);
-                old = __shfl_sync(0xffffffffu, old, 0);
-                if (old == pl - pf) {   // last contributor: sum all partials in CTA order
-                    __threadfence();
-                    float acc2[4][NT][4];
-#pragma unroll
-                    for (int tr = 0; tr < 4; ++tr)
-#pragma unroll
-                        for (int nt = 0; nt < NT; ++nt)
-#pragma unroll
-                            for (int e = 0; e < 4; ++e) acc2[tr][nt][e] = 0.f;
-                    for (int qq = pf; qq <= pl; ++qq) {
-                        const int sl = (rb == unit_start(qq, U, prm.P) / KG) ? 0 : 1;
-                        const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part) + (((size_t)qq * 2 + sl) * kR + r) * (64 * N / 4);
-#pragma unroll
-                        for (int tr = 0; tr < 4; ++tr)
-#pragma unroll
-                            for (int nt = 0; nt < NT; ++nt) {
-                                float4 v = ldg_cg_f4(pp + (tr * NT + nt) * 32 + lane);
-                                acc2[tr][nt][0] += v.x; acc2[tr][nt][1] += v.y; acc2[tr][nt][2] += v.z; acc2[tr][nt][3] += v.w;
-                            }
-                    }
-                    store_y<NT>(prm.Y, N, grow * 64, acc2, lane);
-                    if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed
-                }
-            }
-        }
-    }
     if (lane == 0) trace_k(prm, p, warp, 3);
 }
 
