@@ -52,7 +52,9 @@ for p in range(2):
         a = tr[p, :nst, w, :]
         wait = int(np.sum(a[:, 1] - a[:, 0]))
         busy = int(np.sum(a[:, 3] - a[:, 1]))
-        print(f"scan {w}: wait {wait} scan {busy} per-stage scan {busy / max(nst, 1):.0f}")
+        pre = int(np.sum(a[:, 2] - a[:, 1]))
+        print(f"scan {w}: wait {wait} scan {busy} per-stage scan {busy / max(nst, 1):.0f} "
+              f"(load+prefix {pre / max(nst, 1):.0f}, stores+publish {(busy - pre) / max(nst, 1):.0f})")
     a = tr[p, :nst, 18, :]
     print(f"producer: first issue {rel(a[0,1])}, wait-on-empty sum {int(np.sum(a[:,1]-a[:,0]))}")
     print("stage  prod_issued  scan_full(16)  scan_done(16)  cons_wait_end(min..max over warps)  rel(max)")
@@ -60,3 +62,16 @@ for p in range(2):
         c1 = tr[p, i, :NCW, 1]
         print(f"{i:4d} {rel(tr[p,i,18,1]):10d} {rel(tr[p,i,16,1]):10d} {rel(tr[p,i,16,3]):10d} "
               f"{rel(c1.min()):10d}..{rel(c1.max()):<10d} {rel(tr[p,i,:NCW,3].max()):10d}")
+
+# per-stage release latency (decode done -> slot released) of a few consumer warps: segment
+# ends (epilogue) stand out
+for p in range(1):
+    k = tr[p, 63]
+    t0 = k[:, 0][k[:, 0] > 0].min()
+    nst = int(max(np.count_nonzero(tr[p, :63, w, 3]) for w in range(NCW)))
+    print(f"=== CTA {p} epilogue scan (ev3-ev2 per stage, cycles) for warps 0, 1, 8, 15")
+    for i in range(nst):
+        v = [int(tr[p, i, w, 3] - tr[p, i, w, 2]) for w in (0, 1, 8, 15)]
+        if max(v) > 1500:
+            print(f"stage {i:3d} start {int(tr[p, i, 0, 0] - t0):7d}  epi {v}  decode-done w0..w15 spread "
+                  f"{int(tr[p, i, :NCW, 2].max() - tr[p, i, :NCW, 2].min())}")
