@@ -86,6 +86,7 @@ struct Params {
     float *ws_part;
     int32_t *ws_cnt;
     int KG, MG;
+    int N;                                      // real N (the tcgen05 path pads X to NB via TMA OOB fill)
     uint32_t U;                                 // units (rowblock x GT column); U * P < 2^32
     int P;
     int G, S;
@@ -760,6 +761,442 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     if (lane == 0) trace_k(prm, p, warp, 3);
 }
 
+// ================================================================ tcgen05 path
+// Same producer / scan / stage sequence as k_spmm; what changes is where the SMBD output goes
+// and who multiplies:
+//   * 16 decode warps: warp w owns TMEM lane quarter q = w & 3 (TCTile rows 2q, 2q+1 of the
+//     128-row rowblock; a warp may only touch its own lane quarter) and k-team kt = w >> 2
+//     (GroupTile column kt of the stage). Per stage it decodes 8 TCTiles (32 BitmapTiles) with
+//     the same SMBD as k_spmm and writes each TCTile's four A-fragment registers to TMEM with
+//     one tcgen05.st.16x128b.x2 (A operand of the MMA, Fig. 6 step 5 on tcgen05).
+//   * 1 MMA warp (one thread): per stage and k-team, 4 x tcgen05.mma kind::f16, M = 128,
+//     N = NB, K = 16, A from TMEM, B = the TMA-staged X slab (MN-major, 32B/64B swizzle),
+//     D fp32 in TMEM (two buffers). The accumulation over K happens in the tensor core, so
+//     the consumer-side cross-warp reduction of k_spmm disappears.
+//   * 4 epilogue warps (lane quarters): tcgen05.ld of D at a rowblock end, one RNE to fp16,
+//     Y stores, or the split-K partial + "last contributor sums" fix-up.
+// Pipelines: afull/aempty[k-team][2] (A buffers), dfull/dempty[2] (D buffers), empty[slot]
+// counts the 16 decode warps + the MMA warp's commit (X is read by the tensor core).
+struct CfgTC {
+    static constexpr int CW = 16;
+    static constexpr int EpiWarp = 16;       // 16..19 (lane quarter = warp & 3)
+    static constexpr int MmaWarp = 20;
+    static constexpr int ScanWarp = 21;      // 21, 22
+    static constexpr int ProducerWarp = 23;
+    static constexpr int Threads = 24 * 32;
+    static constexpr uint32_t TmemCols = 512;
+    static constexpr int ABufs = 3;          // A buffers per k-team (TMEM columns [0, 384))
+    static constexpr uint32_t DCol = 384;    // D buffers: columns [384, 384 + 2 NB)
+};
+// barrier / scalar region (bytes from the aligned smem base)
+constexpr uint32_t kTcFull = 0, kTcEmpty = 64, kTcScan = 128, kTcTmemSlot = 208, kTcFlag = 212;
+constexpr uint32_t kTcAFull = 256, kTcAEmpty = 352, kTcDFull = 448, kTcDEmpty = 464;   // afull/aempty [4][3]
+// ring position of a 3-deep A buffer: buffer index and phase parity, advanced once per stage
+struct ARing {
+    uint32_t b = 0, ph = 0;
+    __device__ __forceinline__ void next() { if (++b == CfgTC::ABufs) { b = 0; ph ^= 1u; } }
+};
+
+template <int NB>
+__global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_constant__ Params prm) {
+    constexpr int kCW = CfgTC::CW;
+    constexpr uint32_t kDescBar = 1, kEpiBar = 2, kEndBar = 3;
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *const smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+    const uint32_t sbase = smem_u32(smem);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int p = blockIdx.x;
+    const uint32_t U = prm.U;
+    const int KG = prm.KG, G = prm.G, S = prm.S;
+    const int u0 = unit_start(p, U, prm.P), u1 = unit_start(p + 1, U, prm.P);
+    const uint32_t bar_full = sbase + kTcFull, bar_empty = sbase + kTcEmpty, bar_scan = sbase + kTcScan;
+    const uint32_t bar_af = sbase + kTcAFull, bar_ae = sbase + kTcAEmpty, bar_df = sbase + kTcDFull,
+                   bar_de = sbase + kTcDEmpty;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(bar_full + 8 * s, 1);
+            mbar_init(bar_empty + 8 * s, kCW + 1);          // decode warps + the MMA commit
+            mbar_init(bar_scan + 8 * s, kScanWarps);
+        }
+        for (int k = 0; k < 4 * CfgTC::ABufs; ++k) {
+            mbar_init(bar_af + 8 * k, 4);                  // the 4 lane-quarter warps of a k-team
+            mbar_init(bar_ae + 8 * k, 1);                  // MMA commit
+        }
+        for (int k = 0; k < 2; ++k) {
+            mbar_init(bar_df + 8 * k, 1);                  // MMA commit
+            mbar_init(bar_de + 8 * k, 4);                  // the 4 epilogue warps
+        }
+        fence_barrier_init();
+        reinterpret_cast<uint32_t *>(smem)[kConstWord] = kSelA;
+        reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = kSelB;
+        reinterpret_cast<uint32_t *>(smem)[kConstWord + 2] = kSelC;
+    }
+    if (warp == CfgTC::MmaWarp) tm_alloc(sbase + kTcTmemSlot, CfgTC::TmemCols);
+    StageIter pit;
+    int4 poff = make_int4(0, 0, 0, 0);
+    auto load_off = [&](const StageIter &sg) {
+        const int g0 = kR * sg.rb * KG + sg.gc;
+        int4 v;
+        v.x = __ldg(prm.off + g0);
+        v.y = __ldg(prm.off + g0 + sg.g);
+        v.z = sg.rows > 1 ? __ldg(prm.off + g0 + KG) : 0;
+        v.w = sg.rows > 1 ? __ldg(prm.off + g0 + KG + sg.g) : 0;
+        return v;
+    };
+    if (warp == CfgTC::ProducerWarp && lane == 0) {
+        pit.init(u0, u1, prm);
+        if (pit.valid()) poff = load_off(pit);
+    }
+    tm_fence_before();
+    __syncthreads();
+    tm_fence_after();
+    const uint32_t tmem = *reinterpret_cast<volatile uint32_t *>(smem + kTcTmemSlot);
+
+    if (warp == CfgTC::ProducerWarp) {
+        // ------------------------------------------------------------ producer (as k_spmm)
+        if (lane != 0) return;
+        const uint64_t pol_w = policy_evict_first();
+        const uint32_t xbytes = 64u * NB * 2u;         // one GroupTile column of X (box {NB, 64})
+        for (; pit.valid();) {
+            const StageIter sg = pit;
+            const int i = sg.i, slot = sg.slot;
+            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, sg.par() ^ 1u);
+            const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
+            const uint32_t fb = bar_full + 8 * slot;
+            const uint32_t bmb = (uint32_t)sg.g * 512u;
+            mbar_expect_tx(fb, (uint32_t)sg.rows * bmb + (uint32_t)sg.g * xbytes);
+            for (int r = 0; r < sg.rows; ++r)
+                bulk_g2s(st + prm.st_bm + (uint32_t)(r * G) * 512u,
+                         prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc) * 64, bmb, fb, pol_w);
+            for (int j = 0; j < sg.g; ++j) tma_2d_g2s(st + (uint32_t)j * xbytes, &prm.tmap_x, 0, 64 * (sg.gc + j), fb);
+            const int4 o = poff;
+            const uint32_t vb0 = 2u * (uint32_t)(o.y - o.x);
+            const uint32_t vb1 = sg.rows > 1 ? 2u * (uint32_t)(o.w - o.z) : 0u;
+            if (vb0) bulk_g2s(st + prm.st_v0, prm.vals + o.x, vb0, fb, pol_w);
+            if (vb1) bulk_g2s(st + prm.st_v1, prm.vals + o.z, vb1, fb, pol_w);
+            mbar_arrive_expect_tx(fb, vb0 + vb1);
+            pit.next(prm);
+            if (pit.valid()) poff = load_off(pit);
+        }
+        return;
+    }
+
+    if (warp >= CfgTC::ScanWarp && warp < CfgTC::ScanWarp + kScanWarps) {
+        // ------------------------------------------------------------ scan (as k_spmm)
+        constexpr int Q = kMaxG;
+        const int r = warp - CfgTC::ScanWarp;
+        if (r == 0) {
+            if (lane == 0) {
+                StageIter d;
+                int n = 0;
+                bool full_start = false;
+                for (d.init(u0, u1, prm); d.valid(); d.next(prm), ++n) {
+                    const bool zero = d.seg_first();
+                    if (zero) full_start = (d.gc == 0);
+                    const bool seg_end = d.seg_last(prm);
+                    const bool complete = seg_end && full_start && (d.gc + d.g == KG);
+                    const uint32_t w0 = (uint32_t)d.rb | ((uint32_t)d.slot << 20) | (d.ph << 24) | ((uint32_t)zero << 25) |
+                                        ((uint32_t)seg_end << 26) | ((uint32_t)complete << 27) |
+                                        ((uint32_t)(d.rows - 1) << 28);
+                    sts_v4(sbase + prm.o_desc + 16u * (uint32_t)n,
+                           make_uint4(w0, (uint32_t)d.gc | ((uint32_t)d.g << 16), prm.o_tbl + (uint32_t)d.slot * prm.tbl_bytes,
+                                      prm.o_stage + (uint32_t)d.slot * prm.stage_bytes));
+                }
+                reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3] = (uint32_t)n;
+            }
+            __syncwarp();
+            named_bar_arrive(kDescBar, 32u * (kCW + 4 + 1 + 1));
+        }
+        StageIter it;
+        for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
+            const StageIter &sg = it;
+            const int slot = it.slot;
+            mbar_wait_sleep(bar_full + 8 * slot, it.par());
+            uint2 ba[Q], bb[Q];
+#pragma unroll
+            for (int qq = 0; qq < Q; ++qq) {
+                const uint32_t bmsm = sbase + prm.o_stage + slot * prm.stage_bytes + prm.st_bm + (uint32_t)(r * G + qq) * 512u;
+                if (r < sg.rows && qq < sg.g) {
+                    ba[qq] = lds_v2(bmsm + 8u * lane);
+                    bb[qq] = lds_v2(bmsm + 256u + 8u * lane);
+                } else {
+                    ba[qq] = make_uint2(0u, 0u);
+                    bb[qq] = make_uint2(0u, 0u);
+                }
+            }
+            const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
+            const uint32_t tb = sbase + prm.o_tbl + slot * prm.tbl_bytes;
+            uint32_t packed[Q], incl[Q];
+#pragma unroll
+            for (int qq = 0; qq < Q; ++qq) {
+                packed[qq] = (__popc(ba[qq].x) + __popc(ba[qq].y)) | ((__popc(bb[qq].x) + __popc(bb[qq].y)) << 16);
+                incl[qq] = packed[qq];
+            }
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                uint32_t y[Q];
+#pragma unroll
+                for (int qq = 0; qq < Q; ++qq) y[qq] = __shfl_up_sync(0xffffffffu, incl[qq], o);
+#pragma unroll
+                for (int qq = 0; qq < Q; ++qq) incl[qq] += (lane >= o) ? y[qq] : 0u;
+            }
+            int rel = 0;
+#pragma unroll
+            for (int qq = 0; qq < Q; ++qq) {
+                const uint32_t t = __shfl_sync(0xffffffffu, incl[qq], 31);
+                if (r < sg.rows && qq < sg.g) {
+                    const uint32_t vsm = st + (r ? prm.st_v1 : prm.st_v0);
+                    const uint32_t excl = incl[qq] - packed[qq];
+                    const uint32_t ea = excl & 0xFFFFu, eb = (t & 0xFFFFu) + (excl >> 16);
+                    const uint32_t Aa = vsm + 2u * (uint32_t)(rel + (int)ea);
+                    const uint32_t Ab = vsm + 2u * (uint32_t)(rel + (int)eb);
+                    const uint32_t te = tb + (uint32_t)(r * G + qq) * 1024u + 8u * lane;
+                    sts_v2(te, ba[qq].x, Aa - 4u);
+                    sts_v2(te + 512u, ba[qq].y, Aa - 4u + 2u * __popc(ba[qq].x));
+                    sts_v2(te + 256u, bb[qq].x, Ab - 4u);
+                    sts_v2(te + 768u, bb[qq].y, Ab - 4u + 2u * __popc(bb[qq].x));
+                }
+                rel += (int)(((t & 0xFFFFu) + (t >> 16) + 7u) & ~7u);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar_scan + 8 * slot);
+        }
+        return;
+    }
+
+    const uint32_t desc = sbase + prm.o_desc;
+    auto rd = [&](int si) {
+        const uint4 v = lds_v4(desc + 16u * (uint32_t)si);
+        return StageDesc{v.x, v.y, v.z, v.w};
+    };
+    named_bar_sync(kDescBar, 32u * (kCW + 4 + 1 + 1));
+    const int nst = (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3];
+
+    if (warp == CfgTC::MmaWarp) {
+        // ------------------------------------------------------------ MMA issuer
+        // The whole warp runs the loop (warp-uniform operands stay in uniform registers);
+        // one elected lane issues each tcgen05.mma / commit.
+        {
+            // instruction descriptor: D fp32 (bit 4), A/B fp16, A K-major, B MN-major (bit 16),
+            // N >> 3 at [17, 23), M >> 4 at [24, 29) (verified by tools/tc_probe.cu)
+            constexpr uint32_t idesc = (1u << 4) | (1u << 16) | ((uint32_t)(NB >> 3) << 17) | ((128u >> 4) << 24);
+            // B (X slab) smem descriptor: MN-major canonical layout with the 32B (NB = 16) / 64B
+            // (NB = 32) swizzle, SBO = 8 k-rows, version 1 (sm_100)
+            constexpr uint64_t kDescHi = ((uint64_t)((8 * NB * 2) >> 4) << 32) | (1ull << 46) |
+                                         ((uint64_t)(NB == 16 ? 6 : 4) << 61) | (1ull << 16);
+            int seg = -1;
+            uint32_t first = 0;
+            ARing ar;
+            for (int i = 0; i < nst; ++i, ar.next()) {
+                const StageDesc d = rd(i);
+                if (d.zero()) {
+                    ++seg;
+                    if (seg >= 2) mbar_wait(bar_de + 8u * (uint32_t)(seg & 1), (((uint32_t)seg >> 1) & 1u) ^ 1u);
+                    first = 1;
+                }
+                mbar_wait(bar_full + 8 * d.slot(), d.par());     // X slab landed (async proxy)
+                const uint32_t dcol = CfgTC::DCol + (uint32_t)(seg & 1) * NB;
+                const uint32_t xs = sbase + d.stg;
+                const int g = d.g();
+#pragma unroll 1
+                for (int kt = 0; kt < 4; ++kt) {
+                    const uint32_t ab = (uint32_t)(kt * CfgTC::ABufs) + ar.b;
+                    mbar_wait(bar_af + 8u * ab, ar.ph);
+                    tm_fence_after();
+                    if (kt < g) {
+#pragma unroll
+                        for (int tc = 0; tc < 4; ++tc) {
+                            const uint32_t xa = xs + (uint32_t)kt * (64u * NB * 2u) + (uint32_t)tc * (16u * NB * 2u);
+                            const uint64_t bdesc = kDescHi | (uint64_t)((xa >> 4) & 0x3FFFu);
+                            umma_f16_ts_elect(tmem + dcol, tmem + ab * 32u + 8u * (uint32_t)tc, bdesc, idesc, first ^ 1u);
+                            first = 0;
+                        }
+                    }
+                    umma_commit_elect(bar_ae + 8u * ab);
+                }
+                umma_commit_elect(bar_empty + 8 * d.slot());
+                if (d.seg_end()) umma_commit_elect(bar_df + 8u * (uint32_t)(seg & 1));
+            }
+        }
+        __syncwarp();
+        named_bar_sync(kEndBar, 32u * (kCW + 4 + 1));
+        tm_fence_after();
+        tm_dealloc(tmem, CfgTC::TmemCols);
+        return;
+    }
+
+    if (warp >= CfgTC::EpiWarp && warp < CfgTC::EpiWarp + 4) {
+        // ------------------------------------------------------------ epilogue
+        const int q = warp & 3;
+        const int N = prm.N;
+        const int row_in = 32 * q + lane;               // row within the 128-row rowblock (= TMEM lane)
+        int seg = -1;
+        for (int i = 0; i < nst; ++i) {
+            const StageDesc d = rd(i);
+            if (d.zero()) ++seg;
+            if (!d.seg_end()) continue;
+            const uint32_t db = (uint32_t)(seg & 1);
+            // timed back-off, not the hinted sleep: a hinted try_wait wakes on every mbarrier
+            // event of the CTA (measured: ~2.6 M wake-ups per launch, 15 % of all instructions)
+            mbar_wait_backoff(bar_df + 8u * db, ((uint32_t)seg >> 1) & 1u, 256u, 2048u);
+            tm_fence_after();
+            float v[NB];
+            {
+                float t[16];
+                tm_ld_32x32b_x16(tmem + ((uint32_t)(32 * q) << 16) + CfgTC::DCol + db * NB, t);
+#pragma unroll
+                for (int j = 0; j < 16; ++j) v[j] = t[j];
+                if constexpr (NB == 32) {
+                    tm_ld_32x32b_x16(tmem + ((uint32_t)(32 * q) << 16) + CfgTC::DCol + db * NB + 16u, t);
+#pragma unroll
+                    for (int j = 0; j < 16; ++j) v[16 + j] = t[j];
+                }
+            }
+            tm_wait_ld();
+            tm_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar_de + 8u * db);
+            const int rb = d.rb();
+            const bool valid = row_in < 64 * d.rows();
+            const size_t grow = (size_t)rb * 128 + (size_t)row_in;
+            if (d.complete()) {
+                if (valid) {
+                    uint4 *yp = reinterpret_cast<uint4 *>(prm.Y + grow * (size_t)N);
+#pragma unroll
+                    for (int c8 = 0; c8 < NB / 8; ++c8)
+                        if (c8 * 8 < N) {
+                            __half2 h0 = __floats2half2_rn(v[8 * c8 + 0], v[8 * c8 + 1]);   // one RNE per output (A11)
+                            __half2 h1 = __floats2half2_rn(v[8 * c8 + 2], v[8 * c8 + 3]);
+                            __half2 h2 = __floats2half2_rn(v[8 * c8 + 4], v[8 * c8 + 5]);
+                            __half2 h3 = __floats2half2_rn(v[8 * c8 + 6], v[8 * c8 + 7]);
+                            yp[c8] = make_uint4(*reinterpret_cast<uint32_t *>(&h0), *reinterpret_cast<uint32_t *>(&h1),
+                                                *reinterpret_cast<uint32_t *>(&h2), *reinterpret_cast<uint32_t *>(&h3));
+                        }
+                }
+            } else {
+                // split rowblock: park the fp32 partial, count, the last contributor sums all
+                // partials in CTA order (deterministic), writes Y and re-zeroes the counter
+                const int myslot = (rb == u0 / KG) ? 0 : 1;
+                if (valid) {
+                    float4 *pp = reinterpret_cast<float4 *>(prm.ws_part + (((size_t)p * 2 + myslot) * 128 + row_in) * N);
+#pragma unroll
+                    for (int c4 = 0; c4 < NB / 4; ++c4)
+                        if (c4 * 4 < N) pp[c4] = make_float4(v[4 * c4], v[4 * c4 + 1], v[4 * c4 + 2], v[4 * c4 + 3]);
+                }
+                __threadfence();
+                named_bar_sync(kEpiBar, 128);
+                const int pf = unit_owner(rb * KG, U, prm.P);
+                const int pl = unit_owner((rb + 1) * KG - 1, U, prm.P);
+                if (warp == CfgTC::EpiWarp && lane == 0) {
+                    const int old = atomicAdd(prm.ws_cnt + rb, 1);
+                    *reinterpret_cast<volatile uint32_t *>(smem + kTcFlag) = (old == pl - pf) ? 1u : 0u;
+                }
+                named_bar_sync(kEpiBar, 128);
+                if (*reinterpret_cast<volatile uint32_t *>(smem + kTcFlag)) {
+                    __threadfence();
+                    if (valid) {
+#pragma unroll
+                        for (int j = 0; j < NB; ++j) v[j] = 0.f;
+                        for (int qq = pf; qq <= pl; ++qq) {
+                            const int sl = (rb == unit_start(qq, U, prm.P) / KG) ? 0 : 1;
+                            const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part + (((size_t)qq * 2 + sl) * 128 + row_in) * N);
+#pragma unroll
+                            for (int c4 = 0; c4 < NB / 4; ++c4)
+                                if (c4 * 4 < N) {
+                                    const float4 x = ldg_cg_f4(pp + c4);
+                                    v[4 * c4] += x.x; v[4 * c4 + 1] += x.y; v[4 * c4 + 2] += x.z; v[4 * c4 + 3] += x.w;
+                                }
+                        }
+                        uint4 *yp = reinterpret_cast<uint4 *>(prm.Y + grow * (size_t)N);
+#pragma unroll
+                        for (int c8 = 0; c8 < NB / 8; ++c8)
+                            if (c8 * 8 < N) {
+                                __half2 h0 = __floats2half2_rn(v[8 * c8 + 0], v[8 * c8 + 1]);
+                                __half2 h1 = __floats2half2_rn(v[8 * c8 + 2], v[8 * c8 + 3]);
+                                __half2 h2 = __floats2half2_rn(v[8 * c8 + 4], v[8 * c8 + 5]);
+                                __half2 h3 = __floats2half2_rn(v[8 * c8 + 6], v[8 * c8 + 7]);
+                                yp[c8] = make_uint4(*reinterpret_cast<uint32_t *>(&h0), *reinterpret_cast<uint32_t *>(&h1),
+                                                    *reinterpret_cast<uint32_t *>(&h2), *reinterpret_cast<uint32_t *>(&h3));
+                            }
+                    }
+                    if (warp == CfgTC::EpiWarp && lane == 0) prm.ws_cnt[rb] = 0;   // leave the workspace zeroed
+                }
+            }
+        }
+        tm_fence_before();
+        named_bar_sync(kEndBar, 32u * (kCW + 4 + 1));
+        return;
+    }
+
+    // ---------------------------------------------------------------- decode warps
+    const int q = warp & 3, kt = warp >> 2, r = q >> 1;
+    uint32_t mulc = opaque_u32(1u << (30u - 2u * (uint32_t)(lane & 15)));
+    const uint32_t tbl_lane = (uint32_t)(lane >> 4) * 512u + (uint32_t)(q & 1) * 64u;   // + GT * 1024 + tc * 128
+    const uint32_t t_q = tmem + ((uint32_t)(32 * q) << 16);
+    const uint32_t selA = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];
+    const uint32_t selB = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];
+    const uint32_t selC = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 2];
+    uint4 E[4];
+    uint32_t tA0[8], tA1[8], sA[8], tB0[8], tB1[8], sB[8];
+    auto load_E = [&](uint32_t tb, int tc) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) E[k] = lds_v4(tb + (uint32_t)tc * 128u + 16u * k);
+    };
+    auto issue = [&](uint32_t (&t0)[8], uint32_t (&t1)[8], uint32_t (&s1)[8]) {
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
+            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;
+            const uint32_t z = w * mulc;
+            const uint32_t a = A + 2u * __popc(z);
+            const uint32_t y = z >> 30;
+            s1[k] = y * (y * selB + selA) + selC;
+            t0[k] = lds_u16(a);
+            t1[k] = lds_u16(a + 2u);
+        }
+    };
+    auto assemble = [&](const uint32_t (&t0)[8], const uint32_t (&t1)[8], const uint32_t (&s1)[8], uint32_t tcol) {
+        uint32_t a[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) a[k] = prmt(t0[k], t1[k], s1[k]);
+        tm_st_16x128b_x2(t_q + tcol, a[0], a[1], a[2], a[3]);                    // TCTile row 2q
+        tm_st_16x128b_x2(t_q + (16u << 16) + tcol, a[4], a[5], a[6], a[7]);      // TCTile row 2q + 1
+    };
+    ARing ar;
+    for (int i = 0; i < nst; ++i, ar.next()) {
+        const StageDesc d = rd(i);
+        const uint32_t ab = (uint32_t)(kt * CfgTC::ABufs) + ar.b;
+        mbar_wait_sleep(bar_scan + 8 * d.slot(), d.par());
+        if (i >= CfgTC::ABufs) mbar_wait(bar_ae + 8u * ab, ar.ph ^ 1u);
+        tm_fence_after();
+        if (r < d.rows() && kt < d.g()) {
+            const uint32_t tb = sbase + d.tbl + (uint32_t)(r * G + kt) * 1024u + tbl_lane;
+            const uint32_t acol = ab * 32u;
+            load_E(tb, 0);
+            issue(tA0, tA1, sA);
+            load_E(tb, 1);
+            issue(tB0, tB1, sB);
+            load_E(tb, 2);
+            assemble(tA0, tA1, sA, acol + 0u);
+            issue(tA0, tA1, sA);
+            load_E(tb, 3);
+            assemble(tB0, tB1, sB, acol + 8u);
+            issue(tB0, tB1, sB);
+            assemble(tA0, tA1, sA, acol + 16u);
+            assemble(tB0, tB1, sB, acol + 24u);
+            tm_wait_st();
+        }
+        tm_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+            mbar_arrive(bar_af + 8u * ab);
+            mbar_arrive(bar_empty + 8 * d.slot());
+        }
+    }
+    named_bar_sync(kEndBar, 32u * (kCW + 4 + 1));
+}
+
 struct Plan {
     int P, G, S;
     long long U;
@@ -791,7 +1228,7 @@ using EncodeTiledFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_
                                    const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
-int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N) {
+int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N, int NX) {
     static EncodeTiledFn fn = nullptr;
     if (!fn) {
         void *f = nullptr;
@@ -805,17 +1242,19 @@ int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N) {
     }
     const cuuint64_t dims[2] = {(cuuint64_t)N, (cuuint64_t)K};
     const cuuint64_t strides[1] = {(cuuint64_t)N * 2};
-    const cuuint32_t box[2] = {(cuuint32_t)N, 64u};
+    // box {NX, 64}: NX > N (tcgen05 path, N = 8 / 24) reads past the tensor's columns, which the
+    // TMA fills with zeros (X padded to the MMA's N = 16 / 32 without a copy)
+    const cuuint32_t box[2] = {(cuuint32_t)NX, 64u};
     const cuuint32_t estr[2] = {1u, 1u};
-    const CUtensorMapSwizzle sw = N == 16 ? CU_TENSOR_MAP_SWIZZLE_32B : N == 32 ? CU_TENSOR_MAP_SWIZZLE_64B
-                                                                               : CU_TENSOR_MAP_SWIZZLE_NONE;
+    const CUtensorMapSwizzle sw = NX == 16 ? CU_TENSOR_MAP_SWIZZLE_32B : NX == 32 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                                                 : CU_TENSOR_MAP_SWIZZLE_NONE;
     CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, const_cast<uint16_t *>(X), dims, strides, box, estr,
                     CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS ? SPINFER_OK : SPINFER_EINVAL;
 }
 
-bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
+bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl, bool tc) {
     const int MG = M / kGT, KG = K / kGT;
     const int nRB = (MG + kR - 1) / kR;
     const long long U = (long long)nRB * KG;
@@ -829,14 +1268,15 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl) {
     cudaGetLastError();
     int maxv = max_gt_values > 0 ? max_gt_values : 4096;
     maxv = std::min(4096, (maxv + 7) & ~7);
-    const uint32_t o_desc = 256;
+    const uint32_t o_desc = 512;
+    const int NX = tc ? (N <= 16 ? 16 : 32) : N;   // X slab columns
     int gmax = kMaxG, smax = kMaxStages;
     if (const char *e = getenv("SPINFER_G")) gmax = std::max(1, std::min(kMaxG, atoi(e)));
     if (const char *e = getenv("SPINFER_S")) smax = std::max(2, std::min(kMaxStages, atoi(e)));
     for (int G = gmax; G >= 1; --G) {
         uint32_t tbl = (uint32_t)kR * G * 64 * 16;
-        const uint32_t scr_row = (uint32_t)(N <= 16 ? 4 : 2) * 64 * N * 4;   // 2*KQ fp32 partials: the epilogue scratch per GT row
-        uint32_t st_bm = (uint32_t)G * 64 * N * 2;            // X slab first, then bitmaps
+        const uint32_t scr_row = tc ? 0u : (uint32_t)(N <= 16 ? 4 : 2) * 64 * N * 4;   // k_spmm: epilogue scratch per GT row
+        uint32_t st_bm = (uint32_t)G * 64 * NX * 2;           // X slab first, then bitmaps
         uint32_t st_v0 = st_bm + (uint32_t)kR * G * 512;
         uint32_t vcap = align_up(std::max((uint32_t)G * maxv * 2, scr_row), 16);   // also the epilogue scratch
         uint32_t st_v1 = st_v0 + vcap;
@@ -879,6 +1319,21 @@ int launch_nt(const Plan &pl, cudaStream_t st) {
     return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
 }
 
+template <int NB>
+int launch_tc(const Plan &pl, cudaStream_t st) {
+    static int configured_smem[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if ((int)pl.smem > configured_smem[dev]) {
+        if (cudaFuncSetAttribute(k_spmm_tc<NB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem) != cudaSuccess)
+            return SPINFER_ECUDA;
+        configured_smem[dev] = (int)pl.smem;
+    }
+    k_spmm_tc<NB><<<pl.P, CfgTC::Threads, pl.smem, st>>>(pl.prm);
+    return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
+}
+
 }  // namespace
 
 size_t spmm_workspace_bytes(int M, int K, int N) {
@@ -893,12 +1348,16 @@ size_t spmm_workspace_bytes(int M, int K, int N) {
 int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *ws, size_t ws_bytes,
                 cudaStream_t st) {
     Plan pl;
-    if (!make_plan(M, K, N, T->max_gt_values, &pl)) return SPINFER_EINVAL;
+    // tcgen05 path by default; SPINFER_KERNEL=mma selects the mma.sync kernel (A/B experiments)
+    const char *ke = getenv("SPINFER_KERNEL");
+    const bool tc = !(ke && ke[0] == 'm');
+    if (!make_plan(M, K, N, T->max_gt_values, &pl, tc)) return SPINFER_EINVAL;
     const size_t need = spmm_workspace_bytes(M, K, N);
     if (need == 0) return SPINFER_EINVAL;
     if (ws_bytes < need || ws == nullptr) return SPINFER_ENOSPC;
     Params &q = pl.prm;
-    if (int rc = encode_x_map(&q.tmap_x, X, K, N)) return rc;
+    if (int rc = encode_x_map(&q.tmap_x, X, K, N, tc ? (N <= 16 ? 16 : 32) : N)) return rc;
+    q.N = N;
     q.off = T->gtile_offset;
     q.bm = T->bitmap;
     q.vals = T->values;
@@ -918,7 +1377,9 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
         q.trace = trace_buf;
     }
     int rc = SPINFER_EINVAL;
-    switch (N) {
+    if (tc) {
+        rc = N <= 16 ? launch_tc<16>(pl, st) : launch_tc<32>(pl, st);
+    } else switch (N) {
         case 8: rc = launch_nt<1>(pl, st); break;
         case 16: rc = launch_nt<2>(pl, st); break;
         case 24: rc = launch_nt<3>(pl, st); break;

@@ -122,7 +122,22 @@ __global__ void k_mma(const __grid_constant__ Args args, const __half *A /*[128]
             uint64_t d = (uint64_t)((start >> 4) & 0x3FFF) | (lbo << 16) | (sbo << 32) | (1ull << 46) | ((uint64_t)swz_type << 61);
             mma_f16_ts(tb + 0u, tb + 32u + 8u * s, d, idesc, s > 0 ? 1u : 0u);
         }
+        const long long t0 = clock64();
         mma_commit(smem_u32(&bars[1]));
+        mbar_wait(smem_u32(&bars[1]), 0);
+        const long long t1 = clock64();
+        // second round: 16 MMAs back to back (a stage's worth), then commit
+        for (int s = 0; s < 16; ++s) {
+            const uint32_t start = xs + (uint32_t)(s & 3) * 16u * NB * 2u;
+            const uint64_t sbo = (uint64_t)(8 * NB * 2) >> 4;
+            uint64_t d = (uint64_t)((start >> 4) & 0x3FFF) | (1ull << 16) | (sbo << 32) | (1ull << 46) | ((uint64_t)swz_type << 61);
+            mma_f16_ts(tb + 64u, tb + 32u + 8u * (s & 3), d, (1u << 4) | (1u << 16) | ((uint32_t)(NB >> 3) << 17) | ((128u >> 4) << 24), s > 0 ? 1u : 0u);
+        }
+        const long long t2 = clock64();
+        mma_commit(smem_u32(&bars[1]));
+        mbar_wait(smem_u32(&bars[1]), 1);
+        const long long t3 = clock64();
+        printf("NB=%d: 4 MMAs issue+commit->arrive %lld cycles (issue part incl. above); 16 MMAs issue %lld, commit->arrive %lld cycles\n", NB, t1 - t0, t2 - t1, t3 - t2);
     }
     __syncwarp();
     mbar_wait(smem_u32(&bars[1]), 0);
