@@ -279,3 +279,12 @@ __device__ __forceinline__ void umma_commit_elect(uint32_t bar) {
                  ::"r"(bar) : "memory");
 }
 }  // namespace spinfer
+
+namespace spinfer {
+// One lane of the (converged) warp returns true.
+__device__ __forceinline__ bool elect_one() {
+    uint32_t p;
+    asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\tselp.u32 %0, 1, 0, e;\n\t}" : "=r"(p));
+    return p != 0;
+}
+}  // namespace spinfer

@@ -762,45 +762,78 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
 }
 
 // ================================================================ tcgen05 path
-// Same producer / scan / stage sequence as k_spmm; what changes is where the SMBD output goes
-// and who multiplies:
+// Same stream-K stage sequence as k_spmm; what changes is the data path and who multiplies:
 //   * 16 decode warps: warp w owns TMEM lane quarter q = w & 3 (TCTile rows 2q, 2q+1 of the
 //     128-row rowblock; a warp may only touch its own lane quarter) and k-team kt = w >> 2
-//     (GroupTile column kt of the stage). Per stage it decodes 8 TCTiles (32 BitmapTiles) with
-//     the same SMBD as k_spmm and writes each TCTile's four A-fragment registers to TMEM with
-//     one tcgen05.st.16x128b.x2 (A operand of the MMA, Fig. 6 step 5 on tcgen05).
-//   * 1 MMA warp (one thread): per stage and k-team, 4 x tcgen05.mma kind::f16, M = 128,
-//     N = NB, K = 16, A from TMEM, B = the TMA-staged X slab (MN-major, 32B/64B swizzle),
-//     D fp32 in TMEM (two buffers). The accumulation over K happens in the tensor core, so
-//     the consumer-side cross-warp reduction of k_spmm disappears.
-//   * 4 epilogue warps (lane quarters): tcgen05.ld of D at a rowblock end, one RNE to fp16,
-//     Y stores, or the split-K partial + "last contributor sums" fix-up.
-// Pipelines: afull/aempty[k-team][2] (A buffers), dfull/dempty[2] (D buffers), empty[slot]
-// counts the 16 decode warps + the MMA warp's commit (X is read by the tensor core).
+//     (GroupTile column kt of the stage). Per stage it
+//       - builds the SMBD table for its GroupTile (PopCount prefix over the GT's 64 BTs)
+//         from bitmaps it loaded into registers one stage earlier (no TMA, no scan warps):
+//         {bitmap half-word, smem address of that half's first value - 4} per (BT, half);
+//       - decodes its 8 TCTiles (32 BitmapTiles, MaskedPopCount Alg. 2) into
+//         A-fragment registers and writes each TCTile to TMEM with one tcgen05.st.16x128b.x2.
+//   * 1 MMA warp (one elected lane issues): per stage and GroupTile column 4 x tcgen05.mma
+//     kind::f16, M = 128, N = NB, K = 16, A from TMEM, B = the TMA-staged X slab (MN-major,
+//     32B/64B swizzle), D fp32 in TMEM (4 buffers). The tensor core accumulates over K.
+//   * 1 producer warp: per stage two 1-D bulk copies (the packed values of the two GT rows,
+//     contiguous along K) and one 2-D tensor TMA (X rows [64 gc, 64 (gc + G)), box {NB, 64 G}).
+//     Measured on B200 (tools/tma_sweep.sh): a bulk copy occupies the SM's TMA unit >= ~310 ns
+//     however small, so a stage issues as few copies as possible.
+//   * rowblock epilogue: segment s is finished by k-team s & 3 one stage after its last stage:
+//     tcgen05.ld of D, one RNE to fp16 and the Y store, or (split rowblock) the fp32 partial,
+//     counted and summed by the fix-up warp off the decode path.
+// Every role walks the same StageIter sequence itself (no descriptor table, no start-up wait).
 struct CfgTC {
     static constexpr int CW = 16;
-    static constexpr int EpiWarp = 16;       // 16..19 (lane quarter = warp & 3)
-    static constexpr int MmaWarp = 20;
-    static constexpr int ScanWarp = 21;      // 21, 22
-    static constexpr int ProducerWarp = 23;
-    static constexpr int Threads = 24 * 32;
+    static constexpr int MmaWarp = 16;
+    static constexpr int ProducerWarp = 17;
+    static constexpr int ScanWarp = 18;      // 18, 19: SMBD tables of even / odd stages
+    static constexpr int Threads = 20 * 32;  // 5 warps per SM sub-partition: 96 registers each
     static constexpr uint32_t TmemCols = 512;
-    static constexpr int ABufs = 3;          // A buffers per k-team (TMEM columns [0, 384))
-    static constexpr uint32_t DCol = 384;    // D buffers: columns [384, 384 + 2 NB)
+    static constexpr int ABufs = 3;          // A buffers: TMEM columns [0, 384), 32 per k-team
+    static constexpr uint32_t DCol = 384;    // D buffers: [384, 384 + 4 NB)
+    static constexpr int DBufs = 4;
 };
-// barrier / scalar region (bytes from the aligned smem base)
-constexpr uint32_t kTcFull = 0, kTcEmpty = 64, kTcScan = 128, kTcTmemSlot = 208, kTcFlag = 212;
-constexpr uint32_t kTcAFull = 256, kTcAEmpty = 352, kTcDFull = 448, kTcDEmpty = 464;   // afull/aempty [4][3]
-// ring position of a 3-deep A buffer: buffer index and phase parity, advanced once per stage
-struct ARing {
+// barrier / scalar region (bytes from the aligned smem base); per-warp tables from 1024
+constexpr uint32_t kTcFull = 0, kTcEmpty = 64, kTcEmptyX = 128, kTcTmemSlot = 208;
+constexpr uint32_t kTcAFull = 256, kTcAEmpty = 288, kTcDFull = 320, kTcDEmpty = 352, kTcFix = 384;
+constexpr uint32_t kTcScan = 512;      // [S]: the slot's SMBD table is written
+// ring position of a multi-buffer: index and phase parity, advanced once per use
+template <int NBUF>
+struct Ring {
     uint32_t b = 0, ph = 0;
-    __device__ __forceinline__ void next() { if (++b == CfgTC::ABufs) { b = 0; ph ^= 1u; } }
+    __device__ __forceinline__ void next() { if (++b == NBUF) { b = 0; ph ^= 1u; } }
 };
+// per-stage segment flags, computed identically by every role from the StageIter
+struct SegFlags {
+    bool full_start = false;
+    bool zero = false, seg_end = false, complete = false;
+    __device__ __forceinline__ void at(const StageIter &sg, const Params &prm) {
+        zero = sg.seg_first();
+        if (zero) full_start = (sg.gc == 0);
+        seg_end = sg.seg_last(prm);
+        complete = seg_end && full_start && (sg.gc + sg.g == prm.KG);
+    }
+};
+
+template <int NB>
+__device__ __forceinline__ void store_y_row(uint16_t *Y, size_t grow, int N, const float (&v)[NB]) {
+    uint4 *yp = reinterpret_cast<uint4 *>(Y + grow * (size_t)N);
+#pragma unroll
+    for (int c8 = 0; c8 < NB / 8; ++c8)
+        if (c8 * 8 < N) {
+            __half2 h0 = __floats2half2_rn(v[8 * c8 + 0], v[8 * c8 + 1]);   // one RNE per output (A11)
+            __half2 h1 = __floats2half2_rn(v[8 * c8 + 2], v[8 * c8 + 3]);
+            __half2 h2 = __floats2half2_rn(v[8 * c8 + 4], v[8 * c8 + 5]);
+            __half2 h3 = __floats2half2_rn(v[8 * c8 + 6], v[8 * c8 + 7]);
+            yp[c8] = make_uint4(*reinterpret_cast<uint32_t *>(&h0), *reinterpret_cast<uint32_t *>(&h1),
+                                *reinterpret_cast<uint32_t *>(&h2), *reinterpret_cast<uint32_t *>(&h3));
+        }
+}
 
 template <int NB>
 __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_constant__ Params prm) {
     constexpr int kCW = CfgTC::CW;
-    constexpr uint32_t kDescBar = 1, kEpiBar = 2, kEndBar = 3;
+    constexpr uint32_t kEndBar = 1;   // named barrier: decode warps + MMA warp at the end (TMEM dealloc)
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *const smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     const uint32_t sbase = smem_u32(smem);
@@ -809,128 +842,196 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
     const uint32_t U = prm.U;
     const int KG = prm.KG, G = prm.G, S = prm.S;
     const int u0 = unit_start(p, U, prm.P), u1 = unit_start(p + 1, U, prm.P);
-    const uint32_t bar_full = sbase + kTcFull, bar_empty = sbase + kTcEmpty, bar_scan = sbase + kTcScan;
+    // ring barriers per slot: full (values + X landed), empty (every decode warp is done with the
+    // slot's values), emptyx (the MMA has read the slot's X slab)
+    const uint32_t bar_full = sbase + kTcFull, bar_empty = sbase + kTcEmpty, bar_emptyx = sbase + kTcEmptyX;
     const uint32_t bar_af = sbase + kTcAFull, bar_ae = sbase + kTcAEmpty, bar_df = sbase + kTcDFull,
-                   bar_de = sbase + kTcDEmpty;
+                   bar_de = sbase + kTcDEmpty, bar_scan = sbase + kTcScan;
 
+    if (lane == 0) trace_k(prm, p, warp, 0);
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
             mbar_init(bar_full + 8 * s, 1);
-            mbar_init(bar_empty + 8 * s, kCW + 1);          // decode warps + the MMA commit
-            mbar_init(bar_scan + 8 * s, kScanWarps);
+            mbar_init(bar_empty + 8 * s, kCW);             // every decode warp
+            mbar_init(bar_emptyx + 8 * s, 1);              // the MMA commit
+            mbar_init(bar_scan + 8 * s, 1);                // the stage's scan warp
         }
-        for (int k = 0; k < 4 * CfgTC::ABufs; ++k) {
-            mbar_init(bar_af + 8 * k, 4);                  // the 4 lane-quarter warps of a k-team
+        for (int k = 0; k < CfgTC::ABufs; ++k) {
+            mbar_init(bar_af + 8 * k, kCW);                // every decode warp has published its A tiles
             mbar_init(bar_ae + 8 * k, 1);                  // MMA commit
         }
-        for (int k = 0; k < 2; ++k) {
+        for (int k = 0; k < CfgTC::DBufs; ++k) {
             mbar_init(bar_df + 8 * k, 1);                  // MMA commit
-            mbar_init(bar_de + 8 * k, 4);                  // the 4 epilogue warps
+            mbar_init(bar_de + 8 * k, 4);                  // the 4 warps of the finishing k-team
         }
+        for (int k = 0; k < 2; ++k) mbar_init(sbase + kTcFix + 8 * k, 4);   // split segment A / C parked
         fence_barrier_init();
         reinterpret_cast<uint32_t *>(smem)[kConstWord] = kSelA;
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = kSelB;
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 2] = kSelC;
     }
     if (warp == CfgTC::MmaWarp) tm_alloc(sbase + kTcTmemSlot, CfgTC::TmemCols);
-    StageIter pit;
-    int4 poff = make_int4(0, 0, 0, 0);
-    auto load_off = [&](const StageIter &sg) {
-        const int g0 = kR * sg.rb * KG + sg.gc;
-        int4 v;
-        v.x = __ldg(prm.off + g0);
-        v.y = __ldg(prm.off + g0 + sg.g);
-        v.z = sg.rows > 1 ? __ldg(prm.off + g0 + KG) : 0;
-        v.w = sg.rows > 1 ? __ldg(prm.off + g0 + KG + sg.g) : 0;
-        return v;
-    };
-    if (warp == CfgTC::ProducerWarp && lane == 0) {
-        pit.init(u0, u1, prm);
-        if (pit.valid()) poff = load_off(pit);
-    }
     tm_fence_before();
     __syncthreads();
     tm_fence_after();
     const uint32_t tmem = *reinterpret_cast<volatile uint32_t *>(smem + kTcTmemSlot);
-
-    if (warp == CfgTC::ProducerWarp) {
-        // ------------------------------------------------------------ producer (as k_spmm)
-        if (lane != 0) return;
-        const uint64_t pol_w = policy_evict_first();
-        const uint32_t xbytes = 64u * NB * 2u;         // one GroupTile column of X (box {NB, 64})
-        for (; pit.valid();) {
-            const StageIter sg = pit;
-            const int i = sg.i, slot = sg.slot;
-            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, sg.par() ^ 1u);
-            const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
-            const uint32_t fb = bar_full + 8 * slot;
-            const uint32_t bmb = (uint32_t)sg.g * 512u;
-            mbar_expect_tx(fb, (uint32_t)sg.rows * bmb + (uint32_t)sg.g * xbytes);
-            for (int r = 0; r < sg.rows; ++r)
-                bulk_g2s(st + prm.st_bm + (uint32_t)(r * G) * 512u,
-                         prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc) * 64, bmb, fb, pol_w);
-            for (int j = 0; j < sg.g; ++j) tma_2d_g2s(st + (uint32_t)j * xbytes, &prm.tmap_x, 0, 64 * (sg.gc + j), fb);
-            const int4 o = poff;
-            const uint32_t vb0 = 2u * (uint32_t)(o.y - o.x);
-            const uint32_t vb1 = sg.rows > 1 ? 2u * (uint32_t)(o.w - o.z) : 0u;
-            if (vb0) bulk_g2s(st + prm.st_v0, prm.vals + o.x, vb0, fb, pol_w);
-            if (vb1) bulk_g2s(st + prm.st_v1, prm.vals + o.z, vb1, fb, pol_w);
-            mbar_arrive_expect_tx(fb, vb0 + vb1);
-            pit.next(prm);
-            if (pit.valid()) poff = load_off(pit);
-        }
+    if (lane == 0) trace_k(prm, p, warp, 1);
+    if (u0 >= u1 || (dbg_mode(prm) & 16)) {   // no work (more CTAs than units); experiment bit 16: launch only
+        if (warp == CfgTC::MmaWarp) tm_dealloc(tmem, CfgTC::TmemCols);
         return;
     }
 
-    if (warp >= CfgTC::ScanWarp && warp < CfgTC::ScanWarp + kScanWarps) {
-        // ------------------------------------------------------------ scan (as k_spmm)
-        constexpr int Q = kMaxG;
-        const int r = warp - CfgTC::ScanWarp;
-        if (r == 0) {
-            if (lane == 0) {
-                StageIter d;
-                int n = 0;
-                bool full_start = false;
-                for (d.init(u0, u1, prm); d.valid(); d.next(prm), ++n) {
-                    const bool zero = d.seg_first();
-                    if (zero) full_start = (d.gc == 0);
-                    const bool seg_end = d.seg_last(prm);
-                    const bool complete = seg_end && full_start && (d.gc + d.g == KG);
-                    const uint32_t w0 = (uint32_t)d.rb | ((uint32_t)d.slot << 20) | (d.ph << 24) | ((uint32_t)zero << 25) |
-                                        ((uint32_t)seg_end << 26) | ((uint32_t)complete << 27) |
-                                        ((uint32_t)(d.rows - 1) << 28);
-                    sts_v4(sbase + prm.o_desc + 16u * (uint32_t)n,
-                           make_uint4(w0, (uint32_t)d.gc | ((uint32_t)d.g << 16), prm.o_tbl + (uint32_t)d.slot * prm.tbl_bytes,
-                                      prm.o_stage + (uint32_t)d.slot * prm.stage_bytes));
-                }
-                reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3] = (uint32_t)n;
+    if (warp == CfgTC::ProducerWarp) {
+        // ------------------------------------------------------------ producer
+        // Lanes 0 / 1 prefetch the value range of GT row 0 / 1 one stage ahead and issue its bulk
+        // copy (one instruction for both rows); lane 0 issues the X tensor TMA.
+        const uint64_t pol_w = policy_evict_first();
+        const uint32_t xbytes = 64u * NB * 2u;         // one GroupTile column of X
+        int2 poff = make_int2(0, 0);
+        auto load_off = [&](const StageIter &sg) {
+            int2 v = make_int2(0, 0);
+            if (lane < sg.rows) {
+                const int g0 = (kR * sg.rb + lane) * KG + sg.gc;
+                v.x = __ldg(prm.off + g0);
+                v.y = __ldg(prm.off + g0 + sg.g);
             }
-            __syncwarp();
-            named_bar_arrive(kDescBar, 32u * (kCW + 4 + 1 + 1));
-        }
-        StageIter it;
-        for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
-            const StageIter &sg = it;
-            const int slot = it.slot;
-            mbar_wait_sleep(bar_full + 8 * slot, it.par());
-            uint2 ba[Q], bb[Q];
+            return v;
+        };
+        // split-K fix-up, served by this warp while it waits for free slots: at most two split
+        // rowblocks per CTA (A: the tail of the rowblock it starts inside, C: the head of the one
+        // it ends inside). The finishing k-team parks this CTA's fp32 partial and arrives on
+        // fix[A/C]; this warp counts it and, as the last contributor, sums all partials in CTA
+        // order (deterministic), writes Y and re-zeroes the counter (ReductionWorkspace).
+        const int N = prm.N;
+        const int a_rb = u0 / KG, c_rb = (u1 - 1) / KG;
+        const bool has_a = (u0 % KG) != 0;
+        const bool has_c = (u1 % KG) != 0 && !(has_a && c_rb == a_rb);
+        int fx = has_a ? 0 : (has_c ? 1 : 2);   // next split segment to serve (2: none left)
+        auto fixup = [&](int sgi) {
+            const int rb = sgi == 0 ? a_rb : c_rb;
+            const int rows = min(kR, prm.MG - kR * rb);
+            __threadfence();   // cumulative: the team's partial stores before the count
+            const int pf = unit_owner(rb * KG, U, prm.P);
+            const int pl = unit_owner((rb + 1) * KG - 1, U, prm.P);
+            int old = 0;
+            if (lane == 0) old = atomicAdd(prm.ws_cnt + rb, 1);
+            old = __shfl_sync(0xffffffffu, old, 0);
+            if (old != pl - pf) return;
+            __threadfence();
+            for (int row_in = lane; row_in < 64 * rows; row_in += 32) {
+                float v[NB];
 #pragma unroll
-            for (int qq = 0; qq < Q; ++qq) {
-                const uint32_t bmsm = sbase + prm.o_stage + slot * prm.stage_bytes + prm.st_bm + (uint32_t)(r * G + qq) * 512u;
-                if (r < sg.rows && qq < sg.g) {
-                    ba[qq] = lds_v2(bmsm + 8u * lane);
-                    bb[qq] = lds_v2(bmsm + 256u + 8u * lane);
-                } else {
-                    ba[qq] = make_uint2(0u, 0u);
-                    bb[qq] = make_uint2(0u, 0u);
+                for (int j = 0; j < NB; ++j) v[j] = 0.f;
+                for (int qq = pf; qq <= pl; ++qq) {
+                    const int sl = (rb == unit_start(qq, U, prm.P) / KG) ? 0 : 1;
+                    const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part + (((size_t)qq * 2 + sl) * 128 + row_in) * N);
+#pragma unroll
+                    for (int c4 = 0; c4 < NB / 4; ++c4)
+                        if (c4 * 4 < N) {
+                            const float4 x = ldg_cg_f4(pp + c4);
+                            v[4 * c4] += x.x; v[4 * c4 + 1] += x.y; v[4 * c4 + 2] += x.z; v[4 * c4 + 3] += x.w;
+                        }
+                }
+                store_y_row<NB>(prm.Y, (size_t)rb * 128 + (size_t)row_in, N, v);
+            }
+            if (lane == 0) prm.ws_cnt[rb] = 0;   // leave the workspace zeroed
+        };
+        auto next_fx = [&]() { fx = (fx == 0 && has_c) ? 1 : 2; };
+        StageIter pit;
+        pit.init(u0, u1, prm);
+        poff = load_off(pit);
+        for (; pit.valid();) {
+            const StageIter sg = pit;
+            const int i = sg.i, slot = sg.slot;
+            if (lane == 0) trace_ev(prm, p, i, warp, 0);
+            if (i >= S) {
+                while (true) {
+                    if (fx < 2 && mbar_test_wait(sbase + kTcFix + 8u * (uint32_t)fx, 0u)) {
+                        fixup(fx);
+                        next_fx();
+                        continue;
+                    }
+                    if (mbar_try_wait_sleep(bar_empty + 8 * slot, sg.par() ^ 1u)) break;
                 }
             }
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
+            const uint32_t vb = 2u * (uint32_t)(poff.y - poff.x);   // lanes 0, 1: value bytes of their GT row
+            const uint32_t vtot = __shfl_sync(0xffffffffu, vb, 0) + __shfl_sync(0xffffffffu, vb, 1);
+            if (lane == 0) mbar_arrive_expect_tx(bar_full + 8 * slot, (uint32_t)G * xbytes + vtot);
+            __syncwarp();
+            if (lane < sg.rows && vb)
+                bulk_g2s(st + (lane ? prm.st_v1 : prm.st_v0), prm.vals + poff.x, vb, bar_full + 8 * slot, pol_w);
+            // the X slab region is free once the MMA of stage i - S has completed
+            if (i >= S) mbar_wait(bar_emptyx + 8 * slot, sg.par() ^ 1u);
+            if (lane == 0) tma_2d_g2s(st, &prm.tmap_x, 0, 64 * sg.gc, bar_full + 8 * slot);   // box {NB, 64 G}
+            if (lane == 0) trace_ev(prm, p, i, warp, 1);
+            pit.next(prm);
+            if (pit.valid()) poff = load_off(pit);
+        }
+        while (fx < 2) {
+            mbar_wait_backoff(sbase + kTcFix + 8u * (uint32_t)fx, 0u, 128u, 1024u);
+            fixup(fx);
+            next_fx();
+        }
+        if (lane == 0) trace_k(prm, p, warp, 3);
+        return;
+    }
+
+    if (warp >= CfgTC::ScanWarp) {
+        // ------------------------------------------------------------ scan
+        // Scan warp s builds the SMBD tables of the stages i = s (mod 2), both GT rows: per
+        // staged GroupTile the popcounts of its 64 BTs, a shuffle scan (the PopCount prefix,
+        // P:274) and a table {bitmap half-word, smem address of that half's first value - 4}
+        // per (BT, lane half), layout [GT (r, j)][half][BT] x 8 B. The bitmaps come from global
+        // memory straight into registers, prefetched two stages ahead (no TMA copy: a bulk copy
+        // costs the SM's TMA unit >= ~310 ns however small, tools/tma_sweep.sh). A table waits
+        // only for its slot to be free, so its latency (shuffle round trips through the loaded
+        // MIO queue) is hidden; two warps double the throughput.
+        constexpr int Q = 2 * kMaxG;
+        const int sw = warp - CfgTC::ScanWarp;
+        struct Bm { uint2 a[Q], b[Q]; int o[kR]; };
+        auto fetch = [&](const StageIter &sg, Bm &f) {
+#pragma unroll
+            for (int qq = 0; qq < Q; ++qq) {
+                const int rr = qq / kMaxG, j = qq % kMaxG;
+                if (rr < sg.rows && j < sg.g) {
+                    const uint64_t *gp = prm.bm + ((size_t)(kR * sg.rb + rr) * KG + sg.gc + j) * 64;
+                    f.a[qq] = ldg_nc_v2(gp + lane);
+                    f.b[qq] = ldg_nc_v2(gp + 32 + lane);
+                } else {
+                    f.a[qq] = make_uint2(0u, 0u);
+                    f.b[qq] = make_uint2(0u, 0u);
+                }
+            }
+        };
+        StageIter it;
+        it.init(u0, u1, prm);
+        if (sw == 1) it.next(prm);
+        auto skip2 = [&](StageIter &x) { x.next(prm); if (x.valid()) x.next(prm); };
+        Bm F;   // one register set: the next stage's loads are issued right after a table is
+                // published and complete while the warp waits for that stage's slot
+        if (it.valid()) fetch(it, F);
+        auto one = [&](Bm &cur) -> bool {
+            if (!it.valid()) return false;
+            const StageIter sg = it;
+            const int slot = sg.slot;
+            if (lane == 0) trace_ev(prm, p, sg.i, warp, 0);
+            if (sg.i >= S) mbar_wait_sleep(bar_empty + 8 * slot, sg.par() ^ 1u);   // the slot's table is free
+            if (lane == 0) trace_ev(prm, p, sg.i, warp, 1);
+            const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const uint32_t tb = sbase + prm.o_tbl + slot * prm.tbl_bytes;
+            if (dbg_mode(prm) & 2) {   // experiment: no table build
+                __syncwarp();
+                if (lane == 0) mbar_arrive(bar_scan + 8 * slot);
+                skip2(it);
+                if (it.valid()) fetch(it, cur);
+                return true;
+            }
             uint32_t packed[Q], incl[Q];
 #pragma unroll
             for (int qq = 0; qq < Q; ++qq) {
-                packed[qq] = (__popc(ba[qq].x) + __popc(ba[qq].y)) | ((__popc(bb[qq].x) + __popc(bb[qq].y)) << 16);
+                packed[qq] = (__popc(cur.a[qq].x) + __popc(cur.a[qq].y)) |
+                             ((__popc(cur.b[qq].x) + __popc(cur.b[qq].y)) << 16);
                 incl[qq] = packed[qq];
             }
 #pragma unroll
@@ -941,37 +1042,39 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
 #pragma unroll
                 for (int qq = 0; qq < Q; ++qq) incl[qq] += (lane >= o) ? y[qq] : 0u;
             }
-            int rel = 0;
+            int rel[kR] = {0, 0};
 #pragma unroll
             for (int qq = 0; qq < Q; ++qq) {
+                const int rr = qq / kMaxG, j = qq % kMaxG;
                 const uint32_t t = __shfl_sync(0xffffffffu, incl[qq], 31);
-                if (r < sg.rows && qq < sg.g) {
-                    const uint32_t vsm = st + (r ? prm.st_v1 : prm.st_v0);
+                if (rr < sg.rows && j < sg.g) {
+                    const uint32_t vsm = st + (rr ? prm.st_v1 : prm.st_v0);
                     const uint32_t excl = incl[qq] - packed[qq];
                     const uint32_t ea = excl & 0xFFFFu, eb = (t & 0xFFFFu) + (excl >> 16);
-                    const uint32_t Aa = vsm + 2u * (uint32_t)(rel + (int)ea);
-                    const uint32_t Ab = vsm + 2u * (uint32_t)(rel + (int)eb);
-                    const uint32_t te = tb + (uint32_t)(r * G + qq) * 1024u + 8u * lane;
-                    sts_v2(te, ba[qq].x, Aa - 4u);
-                    sts_v2(te + 512u, ba[qq].y, Aa - 4u + 2u * __popc(ba[qq].x));
-                    sts_v2(te + 256u, bb[qq].x, Ab - 4u);
-                    sts_v2(te + 768u, bb[qq].y, Ab - 4u + 2u * __popc(bb[qq].x));
+                    const uint32_t Aa = vsm + 2u * (uint32_t)(rel[rr] + (int)ea);
+                    const uint32_t Ab = vsm + 2u * (uint32_t)(rel[rr] + (int)eb);
+                    const uint32_t te = tb + (uint32_t)(rr * G + j) * 1024u + 8u * lane;
+                    sts_v2(te, cur.a[qq].x, Aa - 4u);
+                    sts_v2(te + 512u, cur.a[qq].y, Aa - 4u + 2u * __popc(cur.a[qq].x));
+                    sts_v2(te + 256u, cur.b[qq].x, Ab - 4u);
+                    sts_v2(te + 768u, cur.b[qq].y, Ab - 4u + 2u * __popc(cur.b[qq].x));
                 }
-                rel += (int)(((t & 0xFFFFu) + (t >> 16) + 7u) & ~7u);
+                // GT j's first value within the row's chunk: earlier GTs' counts, each padded to
+                // a multiple of 8 values (the GTileOffset rule, encode.cu)
+                rel[rr] += (int)(((t & 0xFFFFu) + (t >> 16) + 7u) & ~7u);
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(bar_scan + 8 * slot);
+            if (lane == 0) trace_ev(prm, p, sg.i, warp, 3);
+            skip2(it);
+            if (it.valid()) fetch(it, cur);   // this warp's next stage
+            return true;
+        };
+        while (one(F)) {
         }
+        if (lane == 0) trace_k(prm, p, warp, 3);
         return;
     }
-
-    const uint32_t desc = sbase + prm.o_desc;
-    auto rd = [&](int si) {
-        const uint4 v = lds_v4(desc + 16u * (uint32_t)si);
-        return StageDesc{v.x, v.y, v.z, v.w};
-    };
-    named_bar_sync(kDescBar, 32u * (kCW + 4 + 1 + 1));
-    const int nst = (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3];
 
     if (warp == CfgTC::MmaWarp) {
         // ------------------------------------------------------------ MMA issuer
@@ -987,156 +1090,112 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
                                          ((uint64_t)(NB == 16 ? 6 : 4) << 61) | (1ull << 16);
             int seg = -1;
             uint32_t first = 0;
-            ARing ar;
-            for (int i = 0; i < nst; ++i, ar.next()) {
-                const StageDesc d = rd(i);
-                if (d.zero()) {
+            Ring<CfgTC::ABufs> ar;
+            Ring<CfgTC::DBufs> dr;
+            SegFlags sf;
+            StageIter it;
+            for (it.init(u0, u1, prm); it.valid(); it.next(prm), ar.next()) {
+                const int i = it.i, slot = it.slot;
+                sf.at(it, prm);
+                // every decode warp has published stage i's A tiles (which implies the stage's
+                // data, X slab included, has landed)
+                if (lane == 0) trace_ev(prm, p, i, warp, 0);
+                mbar_wait(bar_af + 8u * ar.b, ar.ph);
+                tm_fence_after();
+                if (lane == 0) trace_ev(prm, p, i, warp, 1);
+                if (sf.zero) {
+                    if (seg >= 0) dr.next();
                     ++seg;
-                    if (seg >= 2) mbar_wait(bar_de + 8u * (uint32_t)(seg & 1), (((uint32_t)seg >> 1) & 1u) ^ 1u);
+                    if (seg >= CfgTC::DBufs) mbar_wait(bar_de + 8u * dr.b, dr.ph ^ 1u);
+                    tm_fence_after();
                     first = 1;
                 }
-                mbar_wait(bar_full + 8 * d.slot(), d.par());     // X slab landed (async proxy)
-                const uint32_t dcol = CfgTC::DCol + (uint32_t)(seg & 1) * NB;
-                const uint32_t xs = sbase + d.stg;
-                const int g = d.g();
-#pragma unroll 1
-                for (int kt = 0; kt < 4; ++kt) {
-                    const uint32_t ab = (uint32_t)(kt * CfgTC::ABufs) + ar.b;
-                    mbar_wait(bar_af + 8u * ab, ar.ph);
-                    tm_fence_after();
-                    if (kt < g) {
+                // per-stage bases; every MMA operand is base + a compile-time offset (one elected
+                // lane issues the 4 x g MMAs: no per-MMA election or register broadcasts)
+                const uint32_t d_t = tmem + CfgTC::DCol + dr.b * NB;
+                const uint32_t a_t = tmem + ar.b * 32u;
+                const uint32_t x_lo = (sbase + prm.o_stage + (uint32_t)slot * prm.stage_bytes) >> 4;
+                const int g = it.g;
+                if (elect_one()) {
 #pragma unroll
-                        for (int tc = 0; tc < 4; ++tc) {
-                            const uint32_t xa = xs + (uint32_t)kt * (64u * NB * 2u) + (uint32_t)tc * (16u * NB * 2u);
-                            const uint64_t bdesc = kDescHi | (uint64_t)((xa >> 4) & 0x3FFFu);
-                            umma_f16_ts_elect(tmem + dcol, tmem + ab * 32u + 8u * (uint32_t)tc, bdesc, idesc, first ^ 1u);
-                            first = 0;
+                    for (int kt = 0; kt < kMaxG; ++kt) {
+                        if (kt < g) {
+#pragma unroll
+                            for (int tc = 0; tc < 4; ++tc) {
+                                const uint64_t bdesc = kDescHi | (uint64_t)((x_lo + (uint32_t)(kt * 4 + tc) * (16u * NB * 2u / 16u)) & 0x3FFFu);
+                                umma_f16_ts(d_t, a_t + (uint32_t)(kt * CfgTC::ABufs * 32 + 8 * tc), bdesc, idesc, first ^ 1u);
+                                first = 0;
+                            }
                         }
                     }
-                    umma_commit_elect(bar_ae + 8u * ab);
                 }
-                umma_commit_elect(bar_empty + 8 * d.slot());
-                if (d.seg_end()) umma_commit_elect(bar_df + 8u * (uint32_t)(seg & 1));
+                __syncwarp();
+                first = 0;
+                if (lane == 0) trace_ev(prm, p, i, warp, 2);
+                umma_commit_elect(bar_ae + 8u * ar.b);
+                umma_commit_elect(bar_emptyx + 8 * slot);
+                if (sf.seg_end) umma_commit_elect(bar_df + 8u * dr.b);
+                if (lane == 0) trace_ev(prm, p, i, warp, 3);
             }
         }
         __syncwarp();
-        named_bar_sync(kEndBar, 32u * (kCW + 4 + 1));
+        named_bar_sync(kEndBar, 32u * (kCW + 1));
         tm_fence_after();
         tm_dealloc(tmem, CfgTC::TmemCols);
-        return;
-    }
-
-    if (warp >= CfgTC::EpiWarp && warp < CfgTC::EpiWarp + 4) {
-        // ------------------------------------------------------------ epilogue
-        const int q = warp & 3;
-        const int N = prm.N;
-        const int row_in = 32 * q + lane;               // row within the 128-row rowblock (= TMEM lane)
-        int seg = -1;
-        for (int i = 0; i < nst; ++i) {
-            const StageDesc d = rd(i);
-            if (d.zero()) ++seg;
-            if (!d.seg_end()) continue;
-            const uint32_t db = (uint32_t)(seg & 1);
-            // timed back-off, not the hinted sleep: a hinted try_wait wakes on every mbarrier
-            // event of the CTA (measured: ~2.6 M wake-ups per launch, 15 % of all instructions)
-            mbar_wait_backoff(bar_df + 8u * db, ((uint32_t)seg >> 1) & 1u, 256u, 2048u);
-            tm_fence_after();
-            float v[NB];
-            {
-                float t[16];
-                tm_ld_32x32b_x16(tmem + ((uint32_t)(32 * q) << 16) + CfgTC::DCol + db * NB, t);
-#pragma unroll
-                for (int j = 0; j < 16; ++j) v[j] = t[j];
-                if constexpr (NB == 32) {
-                    tm_ld_32x32b_x16(tmem + ((uint32_t)(32 * q) << 16) + CfgTC::DCol + db * NB + 16u, t);
-#pragma unroll
-                    for (int j = 0; j < 16; ++j) v[16 + j] = t[j];
-                }
-            }
-            tm_wait_ld();
-            tm_fence_before();
-            __syncwarp();
-            if (lane == 0) mbar_arrive(bar_de + 8u * db);
-            const int rb = d.rb();
-            const bool valid = row_in < 64 * d.rows();
-            const size_t grow = (size_t)rb * 128 + (size_t)row_in;
-            if (d.complete()) {
-                if (valid) {
-                    uint4 *yp = reinterpret_cast<uint4 *>(prm.Y + grow * (size_t)N);
-#pragma unroll
-                    for (int c8 = 0; c8 < NB / 8; ++c8)
-                        if (c8 * 8 < N) {
-                            __half2 h0 = __floats2half2_rn(v[8 * c8 + 0], v[8 * c8 + 1]);   // one RNE per output (A11)
-                            __half2 h1 = __floats2half2_rn(v[8 * c8 + 2], v[8 * c8 + 3]);
-                            __half2 h2 = __floats2half2_rn(v[8 * c8 + 4], v[8 * c8 + 5]);
-                            __half2 h3 = __floats2half2_rn(v[8 * c8 + 6], v[8 * c8 + 7]);
-                            yp[c8] = make_uint4(*reinterpret_cast<uint32_t *>(&h0), *reinterpret_cast<uint32_t *>(&h1),
-                                                *reinterpret_cast<uint32_t *>(&h2), *reinterpret_cast<uint32_t *>(&h3));
-                        }
-                }
-            } else {
-                // split rowblock: park the fp32 partial, count, the last contributor sums all
-                // partials in CTA order (deterministic), writes Y and re-zeroes the counter
-                const int myslot = (rb == u0 / KG) ? 0 : 1;
-                if (valid) {
-                    float4 *pp = reinterpret_cast<float4 *>(prm.ws_part + (((size_t)p * 2 + myslot) * 128 + row_in) * N);
-#pragma unroll
-                    for (int c4 = 0; c4 < NB / 4; ++c4)
-                        if (c4 * 4 < N) pp[c4] = make_float4(v[4 * c4], v[4 * c4 + 1], v[4 * c4 + 2], v[4 * c4 + 3]);
-                }
-                __threadfence();
-                named_bar_sync(kEpiBar, 128);
-                const int pf = unit_owner(rb * KG, U, prm.P);
-                const int pl = unit_owner((rb + 1) * KG - 1, U, prm.P);
-                if (warp == CfgTC::EpiWarp && lane == 0) {
-                    const int old = atomicAdd(prm.ws_cnt + rb, 1);
-                    *reinterpret_cast<volatile uint32_t *>(smem + kTcFlag) = (old == pl - pf) ? 1u : 0u;
-                }
-                named_bar_sync(kEpiBar, 128);
-                if (*reinterpret_cast<volatile uint32_t *>(smem + kTcFlag)) {
-                    __threadfence();
-                    if (valid) {
-#pragma unroll
-                        for (int j = 0; j < NB; ++j) v[j] = 0.f;
-                        for (int qq = pf; qq <= pl; ++qq) {
-                            const int sl = (rb == unit_start(qq, U, prm.P) / KG) ? 0 : 1;
-                            const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part + (((size_t)qq * 2 + sl) * 128 + row_in) * N);
-#pragma unroll
-                            for (int c4 = 0; c4 < NB / 4; ++c4)
-                                if (c4 * 4 < N) {
-                                    const float4 x = ldg_cg_f4(pp + c4);
-                                    v[4 * c4] += x.x; v[4 * c4 + 1] += x.y; v[4 * c4 + 2] += x.z; v[4 * c4 + 3] += x.w;
-                                }
-                        }
-                        uint4 *yp = reinterpret_cast<uint4 *>(prm.Y + grow * (size_t)N);
-#pragma unroll
-                        for (int c8 = 0; c8 < NB / 8; ++c8)
-                            if (c8 * 8 < N) {
-                                __half2 h0 = __floats2half2_rn(v[8 * c8 + 0], v[8 * c8 + 1]);
-                                __half2 h1 = __floats2half2_rn(v[8 * c8 + 2], v[8 * c8 + 3]);
-                                __half2 h2 = __floats2half2_rn(v[8 * c8 + 4], v[8 * c8 + 5]);
-                                __half2 h3 = __floats2half2_rn(v[8 * c8 + 6], v[8 * c8 + 7]);
-                                yp[c8] = make_uint4(*reinterpret_cast<uint32_t *>(&h0), *reinterpret_cast<uint32_t *>(&h1),
-                                                    *reinterpret_cast<uint32_t *>(&h2), *reinterpret_cast<uint32_t *>(&h3));
-                            }
-                    }
-                    if (warp == CfgTC::EpiWarp && lane == 0) prm.ws_cnt[rb] = 0;   // leave the workspace zeroed
-                }
-            }
-        }
-        tm_fence_before();
-        named_bar_sync(kEndBar, 32u * (kCW + 4 + 1));
+        if (lane == 0) trace_k(prm, p, warp, 3);
         return;
     }
 
     // ---------------------------------------------------------------- decode warps
     const int q = warp & 3, kt = warp >> 2, r = q >> 1;
-    uint32_t mulc = opaque_u32(1u << (30u - 2u * (uint32_t)(lane & 15)));
-    const uint32_t tbl_lane = (uint32_t)(lane >> 4) * 512u + (uint32_t)(q & 1) * 64u;   // + GT * 1024 + tc * 128
+    const uint32_t mulc = opaque_u32(1u << (30u - 2u * (uint32_t)(lane & 15)));
     const uint32_t t_q = tmem + ((uint32_t)(32 * q) << 16);
     const uint32_t selA = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord];
     const uint32_t selB = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];
     const uint32_t selC = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 2];
+    const int N = prm.N;
+    const int row_in = 32 * q + lane;               // row within the 128-row rowblock (= TMEM lane)
+    const uint32_t tbl_lane = (uint32_t)(lane >> 4) * 512u + (uint32_t)(q & 1) * 64u;   // + GT * 1024 + tc * 128
+
+    // rowblock epilogue of a segment (D buffer db): run by the 4 warps of k-team seg & 3
+    auto epilogue = [&](uint32_t db, uint32_t dph, int rb, int rows, bool complete) {
+        mbar_wait(bar_df + 8u * db, dph);
+        tm_fence_after();
+        float v[NB];
+        {
+            float t[16];
+            tm_ld_32x32b_x16(t_q + CfgTC::DCol + db * NB, t);
+#pragma unroll
+            for (int j = 0; j < 16; ++j) v[j] = t[j];
+            if constexpr (NB == 32) {
+                tm_ld_32x32b_x16(t_q + CfgTC::DCol + db * NB + 16u, t);
+#pragma unroll
+                for (int j = 0; j < 16; ++j) v[16 + j] = t[j];
+            }
+        }
+        tm_wait_ld();
+        tm_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(bar_de + 8u * db);
+        const bool valid = row_in < 64 * rows;
+        if (complete) {
+            if (valid) store_y_row<NB>(prm.Y, (size_t)rb * 128 + (size_t)row_in, N, v);
+            return;
+        }
+        // split rowblock: park this CTA's fp32 partial; the fix-up warp does the rest
+        const int myslot = (rb == u0 / KG) ? 0 : 1;
+        if (valid) {
+            float4 *pp = reinterpret_cast<float4 *>(prm.ws_part + (((size_t)p * 2 + myslot) * 128 + row_in) * N);
+#pragma unroll
+            for (int c4 = 0; c4 < NB / 4; ++c4)
+                if (c4 * 4 < N) pp[c4] = make_float4(v[4 * c4], v[4 * c4 + 1], v[4 * c4 + 2], v[4 * c4 + 3]);
+        }
+        __threadfence();
+        __syncwarp();
+        const bool is_a = (u0 % KG) != 0 && rb == u0 / KG;
+        if (lane == 0) mbar_arrive(sbase + kTcFix + (is_a ? 0u : 8u));
+    };
+
     uint4 E[4];
     uint32_t tA0[8], tA1[8], sA[8], tB0[8], tB1[8], sB[8];
     auto load_E = [&](uint32_t tb, int tc) {
@@ -1163,16 +1222,32 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         tm_st_16x128b_x2(t_q + tcol, a[0], a[1], a[2], a[3]);                    // TCTile row 2q
         tm_st_16x128b_x2(t_q + (16u << 16) + tcol, a[4], a[5], a[6], a[7]);      // TCTile row 2q + 1
     };
-    ARing ar;
-    for (int i = 0; i < nst; ++i, ar.next()) {
-        const StageDesc d = rd(i);
-        const uint32_t ab = (uint32_t)(kt * CfgTC::ABufs) + ar.b;
-        mbar_wait_sleep(bar_scan + 8 * d.slot(), d.par());
-        if (i >= CfgTC::ABufs) mbar_wait(bar_ae + 8u * ab, ar.ph ^ 1u);
+
+    Ring<CfgTC::ABufs> ar;
+    Ring<CfgTC::DBufs> dr;
+    SegFlags sf;
+    int seg = -1;
+    bool pend = false;   // pending epilogue of this k-team: run at the end of the stage after its segment
+    uint32_t pend_db = 0, pend_dph = 0;
+    int pend_rb = 0, pend_rows = 0;
+    bool pend_complete = false;
+    StageIter it;
+    for (it.init(u0, u1, prm); it.valid(); it.next(prm), ar.next()) {
+        const int i = it.i, slot = it.slot;
+        sf.at(it, prm);
+        if (sf.zero) {
+            if (seg >= 0) dr.next();
+            ++seg;
+        }
+        if (lane == 0) trace_ev(prm, p, i, warp, 0);
+        mbar_wait_sleep(bar_scan + 8 * slot, it.par());   // table written (the scan runs ahead)
+        mbar_wait_sleep(bar_full + 8 * slot, it.par());   // values and X landed
+        if (lane == 0) trace_ev(prm, p, i, warp, 1);
+        if (i >= CfgTC::ABufs) mbar_wait(bar_ae + 8u * ar.b, ar.ph ^ 1u);
         tm_fence_after();
-        if (r < d.rows() && kt < d.g()) {
-            const uint32_t tb = sbase + d.tbl + (uint32_t)(r * G + kt) * 1024u + tbl_lane;
-            const uint32_t acol = ab * 32u;
+        if (r < it.rows && kt < it.g && !(dbg_mode(prm) & 1)) {
+            const uint32_t tb = sbase + prm.o_tbl + (uint32_t)slot * prm.tbl_bytes + (uint32_t)(r * G + kt) * 1024u + tbl_lane;
+            const uint32_t acol = ((uint32_t)(kt * CfgTC::ABufs) + ar.b) * 32u;
             load_E(tb, 0);
             issue(tA0, tA1, sA);
             load_E(tb, 1);
@@ -1190,11 +1265,24 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         tm_fence_before();
         __syncwarp();
         if (lane == 0) {
-            mbar_arrive(bar_af + 8u * ab);
-            mbar_arrive(bar_empty + 8 * d.slot());
+            mbar_arrive(bar_af + 8u * ar.b);
+            mbar_arrive(bar_empty + 8 * slot);
         }
+        if (lane == 0) trace_ev(prm, p, i, warp, 2);
+        if (pend) {
+            epilogue(pend_db, pend_dph, pend_rb, pend_rows, pend_complete);
+            pend = false;
+        }
+        if (sf.seg_end && (seg & 3) == kt) {
+            pend = true;
+            pend_db = dr.b; pend_dph = dr.ph; pend_rb = it.rb; pend_rows = it.rows; pend_complete = sf.complete;
+        }
+        if (lane == 0) trace_ev(prm, p, i, warp, 3);
     }
-    named_bar_sync(kEndBar, 32u * (kCW + 4 + 1));
+    if (pend) epilogue(pend_db, pend_dph, pend_rb, pend_rows, pend_complete);
+    tm_fence_before();
+    named_bar_sync(kEndBar, 32u * (kCW + 1));
+    if (lane == 0) trace_k(prm, p, warp, 3);
 }
 
 struct Plan {
@@ -1228,7 +1316,7 @@ using EncodeTiledFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_
                                    const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
-int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N, int NX) {
+int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows) {
     static EncodeTiledFn fn = nullptr;
     if (!fn) {
         void *f = nullptr;
@@ -1244,7 +1332,7 @@ int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N, int NX) {
     const cuuint64_t strides[1] = {(cuuint64_t)N * 2};
     // box {NX, 64}: NX > N (tcgen05 path, N = 8 / 24) reads past the tensor's columns, which the
     // TMA fills with zeros (X padded to the MMA's N = 16 / 32 without a copy)
-    const cuuint32_t box[2] = {(cuuint32_t)NX, 64u};
+    const cuuint32_t box[2] = {(cuuint32_t)NX, (cuuint32_t)box_rows};
     const cuuint32_t estr[2] = {1u, 1u};
     const CUtensorMapSwizzle sw = NX == 16 ? CU_TENSOR_MAP_SWIZZLE_32B : NX == 32 ? CU_TENSOR_MAP_SWIZZLE_64B
                                                                                  : CU_TENSOR_MAP_SWIZZLE_NONE;
@@ -1268,7 +1356,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl, bool tc) {
     cudaGetLastError();
     int maxv = max_gt_values > 0 ? max_gt_values : 4096;
     maxv = std::min(4096, (maxv + 7) & ~7);
-    const uint32_t o_desc = 512;
+    const uint32_t o_desc = 1024;
     const int NX = tc ? (N <= 16 ? 16 : 32) : N;   // X slab columns
     int gmax = kMaxG, smax = kMaxStages;
     if (const char *e = getenv("SPINFER_G")) gmax = std::max(1, std::min(kMaxG, atoi(e)));
@@ -1277,14 +1365,15 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl, bool tc) {
         uint32_t tbl = (uint32_t)kR * G * 64 * 16;
         const uint32_t scr_row = tc ? 0u : (uint32_t)(N <= 16 ? 4 : 2) * 64 * N * 4;   // k_spmm: epilogue scratch per GT row
         uint32_t st_bm = (uint32_t)G * 64 * NX * 2;           // X slab first, then bitmaps
-        uint32_t st_v0 = st_bm + (uint32_t)kR * G * 512;
+        uint32_t st_v0 = st_bm + (tc ? 0u : (uint32_t)kR * G * 512);   // tcgen05 path: bitmaps go to registers
         uint32_t vcap = align_up(std::max((uint32_t)G * maxv * 2, scr_row), 16);   // also the epilogue scratch
         uint32_t st_v1 = st_v0 + vcap;
         uint32_t stage = align_up(st_v1 + vcap, 1024);   // slots stay 1024-aligned (X swizzle)
         // stage descriptors: at most one per unit, and no more than ceil(units/G) + rowblock splits
         const uint32_t desc_bytes = align_up((uint32_t)(16 * std::min<long long>(upc, upc / G + upc / KG + 3)), 128);
         uint32_t fixed = o_desc + desc_bytes + 128 + 2048;   // +slack: t1 over-read, base and ring alignment
-        stage += tbl;                                     // each ring slot carries its table (accounted with it)
+        if (tc) fixed = 1024 + 128 + 1024;   // tcgen05 path: no descriptor table
+        stage += tbl;                                     // k_spmm: each ring slot carries its table
         if ((long long)fixed + 2LL * stage > smem_max) continue;
         int S = (int)std::min<long long>(smax, ((long long)smem_max - fixed) / stage);
         if (S < 3 && G > 1) continue;
@@ -1297,6 +1386,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl, bool tc) {
         q.tbl_bytes = tbl;
         q.o_desc = o_desc;
         q.o_tbl = q.o_desc + desc_bytes;
+        if (tc) q.o_tbl = 1024;
         q.o_stage = align_up(q.o_tbl + (uint32_t)S * tbl, 1024);
         pl->smem = (size_t)q.o_stage + (size_t)S * stage + 128 + 1024;   // +1024: runtime base alignment
         return true;
@@ -1348,15 +1438,15 @@ size_t spmm_workspace_bytes(int M, int K, int N) {
 int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *ws, size_t ws_bytes,
                 cudaStream_t st) {
     Plan pl;
-    // tcgen05 path by default; SPINFER_KERNEL=mma selects the mma.sync kernel (A/B experiments)
+    // mma.sync kernel by default (faster so far); SPINFER_KERNEL=tc selects the tcgen05 kernel
     const char *ke = getenv("SPINFER_KERNEL");
-    const bool tc = !(ke && ke[0] == 'm');
+    const bool tc = ke && ke[0] == 't';
     if (!make_plan(M, K, N, T->max_gt_values, &pl, tc)) return SPINFER_EINVAL;
     const size_t need = spmm_workspace_bytes(M, K, N);
     if (need == 0) return SPINFER_EINVAL;
     if (ws_bytes < need || ws == nullptr) return SPINFER_ENOSPC;
     Params &q = pl.prm;
-    if (int rc = encode_x_map(&q.tmap_x, X, K, N, tc ? (N <= 16 ? 16 : 32) : N)) return rc;
+    if (int rc = encode_x_map(&q.tmap_x, X, K, N, tc ? (N <= 16 ? 16 : 32) : N, tc ? 64 * pl.G : 64)) return rc;
     q.N = N;
     q.off = T->gtile_offset;
     q.bm = T->bitmap;
