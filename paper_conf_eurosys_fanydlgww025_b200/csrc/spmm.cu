@@ -362,12 +362,13 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             const uint32_t bmb = (uint32_t)sg.g * 512u;
             // X and bitmaps first (no offsets needed); the arrive comes with the value bytes last,
             // so the phase cannot complete before every transaction is registered
-            mbar_expect_tx(fb, (uint32_t)sg.rows * bmb + (uint32_t)sg.g * xbytes);
+            mbar_expect_tx(fb, (uint32_t)sg.rows * bmb + (uint32_t)G * xbytes);
             for (int r = 0; r < sg.rows; ++r)
                 bulk_g2s(st + prm.st_bm + (uint32_t)(r * G) * 512u,
                          prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc) * 64, bmb, fb, pol_w);
-            // X slab rows [64 gc, 64 (gc + g)): L2-resident (every CTA reads X), default policy
-            for (int j = 0; j < sg.g; ++j) tma_2d_g2s(st + (uint32_t)j * xbytes, &prm.tmap_x, 0, 64 * (sg.gc + j), fb);
+            // X slab rows [64 gc, 64 (gc + G)) in one tensor TMA (box {N, 64 G}; rows past K are
+            // zero-filled): L2-resident (every CTA reads X), default policy
+            tma_2d_g2s(st, &prm.tmap_x, 0, 64 * sg.gc, fb);
             const int4 o = poff;
             const uint32_t vb0 = 2u * (uint32_t)(o.y - o.x);
             const uint32_t vb1 = sg.rows > 1 ? 2u * (uint32_t)(o.w - o.z) : 0u;
@@ -771,9 +772,12 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
 //         {bitmap half-word, smem address of that half's first value - 4} per (BT, half);
 //       - decodes its 8 TCTiles (32 BitmapTiles, MaskedPopCount Alg. 2) into
 //         A-fragment registers and writes each TCTile to TMEM with one tcgen05.st.16x128b.x2.
-//   * 1 MMA warp (one elected lane issues): per stage and GroupTile column 4 x tcgen05.mma
+//   * the k-team multiplies its own GroupTile column: once its 4 lane-quarter warps have written
+//     their A tiles (named barrier), one elected lane of the team's warp 0 issues 4 x tcgen05.mma
 //     kind::f16, M = 128, N = NB, K = 16, A from TMEM, B = the TMA-staged X slab (MN-major,
-//     32B/64B swizzle), D fp32 in TMEM (4 buffers). The tensor core accumulates over K.
+//     32B/64B swizzle), into the team's own fp32 accumulator in TMEM (2 per team: segment parity).
+//     Four issuers in parallel (a single MMA warp issuing 16 tiny MMAs per stage was the
+//     pipeline's slowest link); the epilogue sums the team accumulators in team order.
 //   * 1 producer warp: per stage two 1-D bulk copies (the packed values of the two GT rows,
 //     contiguous along K) and one 2-D tensor TMA (X rows [64 gc, 64 (gc + G)), box {NB, 64 G}).
 //     Measured on B200 (tools/tma_sweep.sh): a bulk copy occupies the SM's TMA unit >= ~310 ns
@@ -784,18 +788,21 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
 // Every role walks the same StageIter sequence itself (no descriptor table, no start-up wait).
 struct CfgTC {
     static constexpr int CW = 16;
-    static constexpr int MmaWarp = 16;
-    static constexpr int ProducerWarp = 17;
-    static constexpr int ScanWarp = 18;      // 18, 19: SMBD tables of even / odd stages
-    static constexpr int Threads = 20 * 32;  // 5 warps per SM sub-partition: 96 registers each
+    static constexpr int ProducerWarp = 16;
+    static constexpr int ScanWarp = 17;      // 17, 18: SMBD tables of even / odd stages
+    static constexpr int Threads = 19 * 32;  // <= 5 warps per SM sub-partition: 96 registers each
     static constexpr uint32_t TmemCols = 512;
-    static constexpr int ABufs = 3;          // A buffers: TMEM columns [0, 384), 32 per k-team
-    static constexpr uint32_t DCol = 384;    // D buffers: [384, 384 + 4 NB)
-    static constexpr int DBufs = 4;
+};
+// TMEM columns: A buffers [k-team][ABufs] x 32 columns, then D [k-team][segment parity] x NB
+template <int NB>
+struct TmemTC {
+    static constexpr int ABufs = NB == 16 ? 3 : 2;
+    static constexpr uint32_t DCol = 4u * ABufs * 32u;
+    static_assert(DCol + 8u * NB <= CfgTC::TmemCols, "TMEM budget");
 };
 // barrier / scalar region (bytes from the aligned smem base); per-warp tables from 1024
 constexpr uint32_t kTcFull = 0, kTcEmpty = 64, kTcEmptyX = 128, kTcTmemSlot = 208;
-constexpr uint32_t kTcAFull = 256, kTcAEmpty = 288, kTcDFull = 320, kTcDEmpty = 352, kTcFix = 384;
+constexpr uint32_t kTcAEmpty = 256, kTcDFull = 352, kTcDEmpty = 368, kTcFix = 384;   // aempty [4][3]
 constexpr uint32_t kTcScan = 512;      // [S]: the slot's SMBD table is written
 // ring position of a multi-buffer: index and phase parity, advanced once per use
 template <int NBUF>
@@ -833,7 +840,9 @@ __device__ __forceinline__ void store_y_row(uint16_t *Y, size_t grow, int N, con
 template <int NB>
 __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_constant__ Params prm) {
     constexpr int kCW = CfgTC::CW;
-    constexpr uint32_t kEndBar = 1;   // named barrier: decode warps + MMA warp at the end (TMEM dealloc)
+    constexpr int ABufs = TmemTC<NB>::ABufs;
+    constexpr uint32_t DCol = TmemTC<NB>::DCol;
+    constexpr uint32_t kEndBar = 1, kTeamBar = 2;   // named barriers: decode warps at the end; 2 + kt: k-team kt
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *const smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     const uint32_t sbase = smem_u32(smem);
@@ -845,23 +854,20 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
     // ring barriers per slot: full (values + X landed), empty (every decode warp is done with the
     // slot's values), emptyx (the MMA has read the slot's X slab)
     const uint32_t bar_full = sbase + kTcFull, bar_empty = sbase + kTcEmpty, bar_emptyx = sbase + kTcEmptyX;
-    const uint32_t bar_af = sbase + kTcAFull, bar_ae = sbase + kTcAEmpty, bar_df = sbase + kTcDFull,
-                   bar_de = sbase + kTcDEmpty, bar_scan = sbase + kTcScan;
+    const uint32_t bar_ae = sbase + kTcAEmpty, bar_df = sbase + kTcDFull, bar_de = sbase + kTcDEmpty,
+                   bar_scan = sbase + kTcScan;
 
     if (lane == 0) trace_k(prm, p, warp, 0);
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
             mbar_init(bar_full + 8 * s, 1);
             mbar_init(bar_empty + 8 * s, kCW);             // every decode warp
-            mbar_init(bar_emptyx + 8 * s, 1);              // the MMA commit
+            mbar_init(bar_emptyx + 8 * s, 4);              // the 4 k-teams' MMA commits
             mbar_init(bar_scan + 8 * s, 1);                // the stage's scan warp
         }
-        for (int k = 0; k < CfgTC::ABufs; ++k) {
-            mbar_init(bar_af + 8 * k, kCW);                // every decode warp has published its A tiles
-            mbar_init(bar_ae + 8 * k, 1);                  // MMA commit
-        }
-        for (int k = 0; k < CfgTC::DBufs; ++k) {
-            mbar_init(bar_df + 8 * k, 1);                  // MMA commit
+        for (int k = 0; k < 4 * ABufs; ++k) mbar_init(bar_ae + 8 * k, 1);   // [k-team][buffer]: team MMA commit
+        for (int k = 0; k < 2; ++k) {
+            mbar_init(bar_df + 8 * k, 4);                  // [segment parity]: the 4 k-teams' commits
             mbar_init(bar_de + 8 * k, 4);                  // the 4 warps of the finishing k-team
         }
         for (int k = 0; k < 2; ++k) mbar_init(sbase + kTcFix + 8 * k, 4);   // split segment A / C parked
@@ -870,14 +876,14 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = kSelB;
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 2] = kSelC;
     }
-    if (warp == CfgTC::MmaWarp) tm_alloc(sbase + kTcTmemSlot, CfgTC::TmemCols);
+    if (warp == 0) tm_alloc(sbase + kTcTmemSlot, CfgTC::TmemCols);
     tm_fence_before();
     __syncthreads();
     tm_fence_after();
     const uint32_t tmem = *reinterpret_cast<volatile uint32_t *>(smem + kTcTmemSlot);
     if (lane == 0) trace_k(prm, p, warp, 1);
     if (u0 >= u1 || (dbg_mode(prm) & 16)) {   // no work (more CTAs than units); experiment bit 16: launch only
-        if (warp == CfgTC::MmaWarp) tm_dealloc(tmem, CfgTC::TmemCols);
+        if (warp == 0) tm_dealloc(tmem, CfgTC::TmemCols);
         return;
     }
 
@@ -1076,76 +1082,6 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         return;
     }
 
-    if (warp == CfgTC::MmaWarp) {
-        // ------------------------------------------------------------ MMA issuer
-        // The whole warp runs the loop (warp-uniform operands stay in uniform registers);
-        // one elected lane issues each tcgen05.mma / commit.
-        {
-            // instruction descriptor: D fp32 (bit 4), A/B fp16, A K-major, B MN-major (bit 16),
-            // N >> 3 at [17, 23), M >> 4 at [24, 29) (verified by tools/tc_probe.cu)
-            constexpr uint32_t idesc = (1u << 4) | (1u << 16) | ((uint32_t)(NB >> 3) << 17) | ((128u >> 4) << 24);
-            // B (X slab) smem descriptor: MN-major canonical layout with the 32B (NB = 16) / 64B
-            // (NB = 32) swizzle, SBO = 8 k-rows, version 1 (sm_100)
-            constexpr uint64_t kDescHi = ((uint64_t)((8 * NB * 2) >> 4) << 32) | (1ull << 46) |
-                                         ((uint64_t)(NB == 16 ? 6 : 4) << 61) | (1ull << 16);
-            int seg = -1;
-            uint32_t first = 0;
-            Ring<CfgTC::ABufs> ar;
-            Ring<CfgTC::DBufs> dr;
-            SegFlags sf;
-            StageIter it;
-            for (it.init(u0, u1, prm); it.valid(); it.next(prm), ar.next()) {
-                const int i = it.i, slot = it.slot;
-                sf.at(it, prm);
-                // every decode warp has published stage i's A tiles (which implies the stage's
-                // data, X slab included, has landed)
-                if (lane == 0) trace_ev(prm, p, i, warp, 0);
-                mbar_wait(bar_af + 8u * ar.b, ar.ph);
-                tm_fence_after();
-                if (lane == 0) trace_ev(prm, p, i, warp, 1);
-                if (sf.zero) {
-                    if (seg >= 0) dr.next();
-                    ++seg;
-                    if (seg >= CfgTC::DBufs) mbar_wait(bar_de + 8u * dr.b, dr.ph ^ 1u);
-                    tm_fence_after();
-                    first = 1;
-                }
-                // per-stage bases; every MMA operand is base + a compile-time offset (one elected
-                // lane issues the 4 x g MMAs: no per-MMA election or register broadcasts)
-                const uint32_t d_t = tmem + CfgTC::DCol + dr.b * NB;
-                const uint32_t a_t = tmem + ar.b * 32u;
-                const uint32_t x_lo = (sbase + prm.o_stage + (uint32_t)slot * prm.stage_bytes) >> 4;
-                const int g = it.g;
-                if (elect_one()) {
-#pragma unroll
-                    for (int kt = 0; kt < kMaxG; ++kt) {
-                        if (kt < g) {
-#pragma unroll
-                            for (int tc = 0; tc < 4; ++tc) {
-                                const uint64_t bdesc = kDescHi | (uint64_t)((x_lo + (uint32_t)(kt * 4 + tc) * (16u * NB * 2u / 16u)) & 0x3FFFu);
-                                umma_f16_ts(d_t, a_t + (uint32_t)(kt * CfgTC::ABufs * 32 + 8 * tc), bdesc, idesc, first ^ 1u);
-                                first = 0;
-                            }
-                        }
-                    }
-                }
-                __syncwarp();
-                first = 0;
-                if (lane == 0) trace_ev(prm, p, i, warp, 2);
-                umma_commit_elect(bar_ae + 8u * ar.b);
-                umma_commit_elect(bar_emptyx + 8 * slot);
-                if (sf.seg_end) umma_commit_elect(bar_df + 8u * dr.b);
-                if (lane == 0) trace_ev(prm, p, i, warp, 3);
-            }
-        }
-        __syncwarp();
-        named_bar_sync(kEndBar, 32u * (kCW + 1));
-        tm_fence_after();
-        tm_dealloc(tmem, CfgTC::TmemCols);
-        if (lane == 0) trace_k(prm, p, warp, 3);
-        return;
-    }
-
     // ---------------------------------------------------------------- decode warps
     const int q = warp & 3, kt = warp >> 2, r = q >> 1;
     const uint32_t mulc = opaque_u32(1u << (30u - 2u * (uint32_t)(lane & 15)));
@@ -1157,23 +1093,28 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
     const int row_in = 32 * q + lane;               // row within the 128-row rowblock (= TMEM lane)
     const uint32_t tbl_lane = (uint32_t)(lane >> 4) * 512u + (uint32_t)(q & 1) * 64u;   // + GT * 1024 + tc * 128
 
-    // rowblock epilogue of a segment (D buffer db): run by the 4 warps of k-team seg & 3
-    auto epilogue = [&](uint32_t db, uint32_t dph, int rb, int rows, bool complete) {
-        mbar_wait(bar_df + 8u * db, dph);
+    // rowblock epilogue of a segment (D parity db): run by the 4 warps of k-team seg & 3 one stage
+    // after the segment's last stage. Sums the k-teams' accumulators in team order
+    // (deterministic; nteams = the teams that issued MMAs in the segment).
+    auto epilogue = [&](uint32_t db, uint32_t dph_, int rb, int rows, bool complete, int nteams) {
+        mbar_wait(bar_df + 8u * db, dph_);
         tm_fence_after();
         float v[NB];
-        {
-            float t[16];
-            tm_ld_32x32b_x16(t_q + CfgTC::DCol + db * NB, t);
 #pragma unroll
-            for (int j = 0; j < 16; ++j) v[j] = t[j];
-            if constexpr (NB == 32) {
-                tm_ld_32x32b_x16(t_q + CfgTC::DCol + db * NB + 16u, t);
+        for (int j = 0; j < NB; ++j) v[j] = 0.f;
 #pragma unroll
-                for (int j = 0; j < 16; ++j) v[16 + j] = t[j];
+        for (int tt = 0; tt < 4; ++tt) {
+            if (tt < nteams) {
+#pragma unroll
+                for (int h = 0; h < NB / 16; ++h) {
+                    float x[16];
+                    tm_ld_32x32b_x16(t_q + DCol + ((uint32_t)tt * 2u + db) * NB + 16u * h, x);
+                    tm_wait_ld();
+#pragma unroll
+                    for (int j = 0; j < 16; ++j) v[16 * h + j] += x[j];
+                }
             }
         }
-        tm_wait_ld();
         tm_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(bar_de + 8u * db);
@@ -1182,7 +1123,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
             if (valid) store_y_row<NB>(prm.Y, (size_t)rb * 128 + (size_t)row_in, N, v);
             return;
         }
-        // split rowblock: park this CTA's fp32 partial; the fix-up warp does the rest
+        // split rowblock: park this CTA's fp32 partial; the producer warp does the fix-up
         const int myslot = (rb == u0 / KG) ? 0 : 1;
         if (valid) {
             float4 *pp = reinterpret_cast<float4 *>(prm.ws_part + (((size_t)p * 2 + myslot) * 128 + row_in) * N);
@@ -1223,31 +1164,49 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         tm_st_16x128b_x2(t_q + (16u << 16) + tcol, a[4], a[5], a[6], a[7]);      // TCTile row 2q + 1
     };
 
-    Ring<CfgTC::ABufs> ar;
-    Ring<CfgTC::DBufs> dr;
+    // k-team MMA issue (warp q = 0 of the team, one elected lane): tcgen05.mma kind::f16,
+    // M = 128, N = NB, K = 16; A = the team's TMEM buffer, B = the TMA-staged X slab (MN-major
+    // canonical layout, 32B / 64B swizzle, SBO = 8 k-rows, version 1; verified by
+    // tools/tc_probe.cu), D = the team's accumulator of the segment's parity.
+    constexpr uint32_t idesc = (1u << 4) | (1u << 16) | ((uint32_t)(NB >> 3) << 17) | ((128u >> 4) << 24);
+    constexpr uint64_t kDescHi = ((uint64_t)((8 * NB * 2) >> 4) << 32) | (1ull << 46) |
+                                 ((uint64_t)(NB == 16 ? 6 : 4) << 61) | (1ull << 16);
+    Ring<ABufs> ar;
     SegFlags sf;
     int seg = -1;
-    bool pend = false;   // pending epilogue of this k-team: run at the end of the stage after its segment
+    uint32_t dpar = 1, dph = 1;     // D parity of the current segment and its phase (advanced at segment start)
+    bool first = false;             // team: the next MMA starts the segment's accumulation
+    int maxg = 0;                   // GT columns of the segment's widest stage (teams kt < maxg multiply)
+    bool pend = false;              // pending epilogue of this k-team: run at the end of the stage after its segment
     uint32_t pend_db = 0, pend_dph = 0;
-    int pend_rb = 0, pend_rows = 0;
+    int pend_rb = 0, pend_rows = 0, pend_nt = 0;
     bool pend_complete = false;
     StageIter it;
     for (it.init(u0, u1, prm); it.valid(); it.next(prm), ar.next()) {
         const int i = it.i, slot = it.slot;
         sf.at(it, prm);
         if (sf.zero) {
-            if (seg >= 0) dr.next();
             ++seg;
+            dpar ^= 1u;
+            if (dpar == 0) dph ^= 1u;
+            first = true;
+            maxg = 0;
         }
+        maxg = max(maxg, it.g);
         if (lane == 0) trace_ev(prm, p, i, warp, 0);
-        mbar_wait_sleep(bar_scan + 8 * slot, it.par());   // table written (the scan runs ahead)
-        mbar_wait_sleep(bar_full + 8 * slot, it.par());   // values and X landed
+        const bool reuse0 = (dbg_mode(prm) & 4) != 0;   // experiment: stage 0's data for every stage
+        if (!reuse0 || i == 0) {
+            mbar_wait_sleep(bar_scan + 8 * slot, it.par());   // table written (the scan runs ahead)
+            mbar_wait_sleep(bar_full + 8 * slot, it.par());   // values and X landed
+        }
         if (lane == 0) trace_ev(prm, p, i, warp, 1);
-        if (i >= CfgTC::ABufs) mbar_wait(bar_ae + 8u * ar.b, ar.ph ^ 1u);
+        const uint32_t ab = (uint32_t)(kt * ABufs) + ar.b;
+        if (i >= ABufs) mbar_wait(bar_ae + 8u * ab, ar.ph ^ 1u);
         tm_fence_after();
         if (r < it.rows && kt < it.g && !(dbg_mode(prm) & 1)) {
-            const uint32_t tb = sbase + prm.o_tbl + (uint32_t)slot * prm.tbl_bytes + (uint32_t)(r * G + kt) * 1024u + tbl_lane;
-            const uint32_t acol = ((uint32_t)(kt * CfgTC::ABufs) + ar.b) * 32u;
+            const uint32_t tb = sbase + prm.o_tbl + (uint32_t)(reuse0 ? 0 : slot) * prm.tbl_bytes +
+                                (uint32_t)(r * G + kt) * 1024u + tbl_lane;
+            const uint32_t acol = ab * 32u;
             load_E(tb, 0);
             issue(tA0, tA1, sA);
             load_E(tb, 1);
@@ -1264,24 +1223,52 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         }
         tm_fence_before();
         __syncwarp();
-        if (lane == 0) {
-            mbar_arrive(bar_af + 8u * ar.b);
-            mbar_arrive(bar_empty + 8 * slot);
+        if (lane == 0) mbar_arrive(bar_empty + 8 * slot);   // this warp is done with the slot's values/table
+        // the team's 4 lane-quarter warps have written their A tiles: the team leader multiplies
+        named_bar_sync(kTeamBar + (uint32_t)kt, 128);
+        const bool mm = kt < it.g;
+        if (q == 0) {
+            tm_fence_after();
+            if (sf.zero && seg >= 2) {   // the D buffer's previous segment has been read out
+                mbar_wait(bar_de + 8u * dpar, dph ^ 1u);
+                tm_fence_after();
+            }
+            const uint32_t d_t = tmem + DCol + ((uint32_t)kt * 2u + dpar) * NB;
+            const uint32_t a_t = tmem + ab * 32u;
+            const uint32_t x_lo = (sbase + prm.o_stage + (uint32_t)(reuse0 ? 0 : slot) * prm.stage_bytes) >> 4;
+            const uint32_t acc0 = first ? 0u : 1u;
+            if (elect_one()) {
+                if (mm) {
+#pragma unroll
+                    for (int tc = 0; tc < 4; ++tc) {
+                        const uint64_t bdesc = kDescHi | (uint64_t)((x_lo + (uint32_t)(kt * 4 + tc) * (16u * NB * 2u / 16u)) & 0x3FFFu);
+                        umma_f16_ts(d_t, a_t + 8u * (uint32_t)tc, bdesc, idesc, tc == 0 ? acc0 : 1u);
+                    }
+                }
+                umma_commit(bar_ae + 8u * ab);
+                umma_commit(bar_emptyx + 8 * slot);
+                if (sf.seg_end) umma_commit(bar_df + 8u * dpar);
+            }
+            __syncwarp();
         }
+        if (mm) first = false;
         if (lane == 0) trace_ev(prm, p, i, warp, 2);
         if (pend) {
-            epilogue(pend_db, pend_dph, pend_rb, pend_rows, pend_complete);
+            epilogue(pend_db, pend_dph, pend_rb, pend_rows, pend_complete, pend_nt);
             pend = false;
         }
         if (sf.seg_end && (seg & 3) == kt) {
             pend = true;
-            pend_db = dr.b; pend_dph = dr.ph; pend_rb = it.rb; pend_rows = it.rows; pend_complete = sf.complete;
+            pend_db = dpar; pend_dph = dph; pend_rb = it.rb; pend_rows = it.rows; pend_complete = sf.complete;
+            pend_nt = min(maxg, 4);
         }
         if (lane == 0) trace_ev(prm, p, i, warp, 3);
     }
-    if (pend) epilogue(pend_db, pend_dph, pend_rb, pend_rows, pend_complete);
+    if (pend) epilogue(pend_db, pend_dph, pend_rb, pend_rows, pend_complete, pend_nt);
     tm_fence_before();
-    named_bar_sync(kEndBar, 32u * (kCW + 1));
+    named_bar_sync(kEndBar, 32u * kCW);   // every MMA has completed (the last epilogues waited on them)
+    tm_fence_after();
+    if (warp == 0) tm_dealloc(tmem, CfgTC::TmemCols);
     if (lane == 0) trace_k(prm, p, warp, 3);
 }
 
@@ -1446,7 +1433,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     if (need == 0) return SPINFER_EINVAL;
     if (ws_bytes < need || ws == nullptr) return SPINFER_ENOSPC;
     Params &q = pl.prm;
-    if (int rc = encode_x_map(&q.tmap_x, X, K, N, tc ? (N <= 16 ? 16 : 32) : N, tc ? 64 * pl.G : 64)) return rc;
+    if (int rc = encode_x_map(&q.tmap_x, X, K, N, tc ? (N <= 16 ? 16 : 32) : N, 64 * pl.G)) return rc;
     q.N = N;
     q.off = T->gtile_offset;
     q.bm = T->bitmap;

@@ -35,19 +35,18 @@ sp.spmm(T, Xd)
 torch.cuda.synchronize()
 tr = np.fromfile(os.environ["SPINFER_TRACE"], dtype=np.int64).reshape(4, 64, 20, 4)
 
-PW, MW = 17, 16   # producer, MMA warps (decode warps 0-15)
+PW = 16   # producer warp (decode warps 0-15; k-team leaders issue the MMAs)
 for p in range(2):
     k = tr[p, 63]
     t0 = k[:, 0][k[:, 0] > 0].min()
     R = lambda v: int(v - t0) if v > 0 else -1  # noqa: E731
     nst = int(np.count_nonzero(tr[p, :63, PW, 1]))
     print(f"=== CTA {p}: {nst} stages; entry..sync {R(k[:,1].max())}, exit max {max(R(v) for v in k[:, 3])}")
-    print(" st  prodW  issued  dataSeen(min..max)  Apub(min..max)   mmaAseen mmaIssued commit")
+    print(" st  prodW  issued  dataSeen(min..max)  MMAissued(min..max)")
     for i in range(nst):
         c = tr[p, i]
         cw1 = c[:16, 1]; cw2 = c[:16, 2]
-        print(f"{i:3d} {R(c[PW,0]):7d} {R(c[PW,1]):7d} {R(cw1.min()):8d}..{R(cw1.max()):<8d} {R(cw2.min()):7d}..{R(cw2.max()):<7d} "
-              f"{R(c[MW,1]):8d} {R(c[MW,2]):8d} {R(c[MW,3]):7d}")
+        print(f"{i:3d} {R(c[PW,0]):7d} {R(c[PW,1]):7d} {R(cw1.min()):8d}..{R(cw1.max()):<8d} {R(cw2.min()):7d}..{R(cw2.max()):<7d}")
     a = tr[p, :nst, :16, :]
     wait = (a[:, :, 1] - a[:, :, 0]).sum(0)
     work = (a[:, :, 2] - a[:, :, 1]).sum(0)
