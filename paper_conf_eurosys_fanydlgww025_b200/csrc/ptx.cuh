@@ -113,6 +113,11 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t
 // cp.async.mbarrier.arrive.noinc makes the barrier observe one arrival when all of
 // this thread's prior cp.async operations have completed.
 // 2-D TMA tile load (tensor map in param/const space, coordinates innermost first).
+// Pulls a tensor map (here: a __grid_constant__ kernel parameter) into the TMA unit's
+// descriptor cache ahead of its first use.
+__device__ __forceinline__ void prefetch_tmap(const void *tmap) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(tmap)) : "memory");
+}
 __device__ __forceinline__ void tma_2d_g2s(uint32_t dst, const void *tmap, int c0, int c1, uint32_t bar) {
     asm volatile(
         "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
@@ -282,6 +287,12 @@ __device__ __forceinline__ void umma_commit_elect(uint32_t bar) {
 
 namespace spinfer {
 // One lane of the (converged) warp returns true.
+template <uint32_t R> __device__ __forceinline__ void setmaxnreg_inc() {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;\n" ::"n"(R));
+}
+template <uint32_t R> __device__ __forceinline__ void setmaxnreg_dec() {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;\n" ::"n"(R));
+}
 __device__ __forceinline__ bool elect_one() {
     uint32_t p;
     asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\tselp.u32 %0, 1, 0, e;\n\t}" : "=r"(p));

@@ -67,6 +67,22 @@ constexpr int kMaxStages = 8;
 #ifndef SPINFER_MAXG
 #define SPINFER_MAXG 4
 #endif
+// register split between the warp roles (setmaxnreg, per warpgroup): the consumer warpgroups
+// grow to SPINFER_MAXNREG registers, the role warpgroup (fix-up, scan, producer) shrinks to
+// SPINFER_ROLEREG; 0 = one budget for all warps
+#ifndef SPINFER_MAXNREG
+#define SPINFER_MAXNREG 0
+#endif
+#ifndef SPINFER_ROLEREG
+#define SPINFER_ROLEREG 56
+#endif
+// software-pipelined consumer loop also for the 16-warp (KQ = 2) variant
+#ifndef SPINFER_EPREF
+#define SPINFER_EPREF 0
+#endif
+#ifndef SPINFER_PIPE2
+#define SPINFER_PIPE2 0
+#endif
 constexpr int kMaxG = SPINFER_MAXG;  // max GroupTile columns per stage (the scan unrolls over it)
 constexpr int kConstWord = 48;      // smem word index (byte 192) of the SMBD selector-table constants
 constexpr int kTraceCTAs = 4, kTraceStages = 64, kTraceW = 20, kTraceEv = 4;   // stage 63 = kernel-level events
@@ -340,11 +356,16 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         return v;
     };
     if (warp == kProducerWarp && lane == 0) {
+        prefetch_tmap(&prm.tmap_x);
         pit.init(u0, u1, prm);
         if (pit.valid()) poff = load_off(pit);
     }
     __syncthreads();
     if (lane == 0) trace_k(prm, p, warp, 1);
+#if SPINFER_MAXNREG
+    if (warp >= kCW) setmaxnreg_dec<SPINFER_ROLEREG>();
+    else setmaxnreg_inc<SPINFER_MAXNREG>();
+#endif
 
     if (warp == kProducerWarp) {
         // ------------------------------------------------------------ producer
@@ -587,7 +608,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         }
     };
     const bool compute = !(dbg_mode(prm) & 1);
-    constexpr bool kPipe = (KQ == 1);          // explicit cross-step software pipeline (8 consumer warps)
+    constexpr bool kPipe = (KQ == 1) || SPINFER_PIPE2;          // explicit cross-step software pipeline (8 consumer warps)
     const bool reuse0 = (dbg_mode(prm) & 4) != 0;   // experiment: pure consumer throughput on stage 0's data
     auto load_x = [&](uint32_t xs, int j, uint32_t (&bfr)[NT][2]) {   // B fragments of GT j, TCTile column c
         const uint32_t xk = xs + (uint32_t)(64 * j) * cpr * 16u;     // xs includes this lane's x_lane
@@ -651,6 +672,21 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             // KQ = 2: 4 consumer warps per scheduler hide the latencies; one register set.
             const uint32_t xs = sbase + d.stg + x_lane;
             const uint32_t tb = sbase + d.tbl + tbl_lane;
+#if SPINFER_EPREF
+            // the next step's table entries are loaded as soon as the current step has consumed
+            // E (issue), so their latency hides behind the current step's assembly and MMAs
+            load_E(tb, 2 * q);
+            for (int j = q; j < g; j += KQ) {
+                uint32_t bfr[NT][2];
+                load_x(xs, j, bfr);
+                issue(tA0, tA1, sA);
+                load_E(tb, 2 * j + 1);
+                assemble(tA0, tA1, sA, 0, bfr);
+                issue(tA0, tA1, sA);
+                if (j + KQ < g) load_E(tb, 2 * (j + KQ));
+                assemble(tA0, tA1, sA, 2, bfr);
+            }
+#else
             for (int j = q; j < g; j += KQ) {
                 uint32_t bfr[NT][2];
                 load_x(xs, j, bfr);
@@ -661,6 +697,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                     assemble(tA0, tA1, sA, 2 * h, bfr);
                 }
             }
+#endif
         } else if (d.rows() > r && compute && q < g) {
             const uint32_t xs = sbase + d.stg + x_lane;
             const uint32_t tb = sbase + d.tbl + tbl_lane;
@@ -876,6 +913,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = kSelB;
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 2] = kSelC;
     }
+    if (warp == CfgTC::ProducerWarp && lane == 0) prefetch_tmap(&prm.tmap_x);
     if (warp == 0) tm_alloc(sbase + kTcTmemSlot, CfgTC::TmemCols);
     tm_fence_before();
     __syncthreads();
@@ -1425,9 +1463,14 @@ size_t spmm_workspace_bytes(int M, int K, int N) {
 int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *ws, size_t ws_bytes,
                 cudaStream_t st) {
     Plan pl;
-    // mma.sync kernel by default (faster so far); SPINFER_KERNEL=tc selects the tcgen05 kernel
+    // Kernel choice by N, from the B200 measurements: the mma.sync kernel for
+    // N <= 16, the tcgen05 kernel (accumulators in TMEM) for N >= 24, where mma.sync needs twice
+    // the HMMAs and accumulator registers (config 2 shape, mean us: N=24 114.9 vs 112.1, N=32
+    // 126.8 vs 111.0). SPINFER_KERNEL=mma|tc overrides (tests and experiments).
     const char *ke = getenv("SPINFER_KERNEL");
-    const bool tc = ke && ke[0] == 't';
+    bool tc = N >= 24;
+    if (ke && ke[0] == 't') tc = true;
+    if (ke && ke[0] == 'm') tc = false;
     if (!make_plan(M, K, N, T->max_gt_values, &pl, tc)) return SPINFER_EINVAL;
     const size_t need = spmm_workspace_bytes(M, K, N);
     if (need == 0) return SPINFER_EINVAL;

@@ -36,11 +36,38 @@ def run_case(M, K, N, s, seed=1, mode="uniform"):
 SHAPES = [(64, 64), (256, 256), (128, 4096), (192, 320), (1024, 1024), (4096, 2048), (320, 1472)]
 
 
+@pytest.mark.parametrize("kernel", ["default", "mma", "tc"])
 @pytest.mark.parametrize("M,K", SHAPES)
 @pytest.mark.parametrize("N", [8, 16, 24, 32])
-def test_spmm_shapes(M, K, N):
+def test_spmm_shapes(M, K, N, kernel, monkeypatch):
+    """Both sm_100a kernels (mma.sync and tcgen05; the library picks by N) on every shape."""
+    if kernel != "default":
+        monkeypatch.setenv("SPINFER_KERNEL", kernel)
     W, X, Y, Yref = run_case(M, K, N, 0.5, seed=M + K + N)
-    assert_within(Y, Yref, north_star_bound(oracle.decode(oracle.encode(W)), X), f"{M}x{K}x{N}")
+    assert_within(Y, Yref, north_star_bound(oracle.decode(oracle.encode(W)), X), f"{M}x{K}x{N} {kernel}")
+
+
+@pytest.mark.parametrize("kernel", ["mma", "tc"])
+@pytest.mark.parametrize("N", [8, 16, 24, 32])
+def test_spmm_integer_exact_both_kernels(N, kernel, monkeypatch):
+    """P-S2 bit-exactness for each kernel explicitly (split-K fix-up included: 4 CTAs on a
+    long K force rowblocks split across CTAs)."""
+    monkeypatch.setenv("SPINFER_KERNEL", kernel)
+    monkeypatch.setenv("SPINFER_MAX_CTAS", "4")
+    M, K = 384, 2048
+    for seed in range(100, 200):
+        W = synth.weight(M, K, 0.5, seed=seed, mode="int")
+        X = synth.activation(K, N, seed=seed + 1, mode="int")
+        R = oracle.encode(W)
+        Yref = oracle.spmm_f64(R, X)
+        if np.abs(Yref).max() <= 2048:
+            break
+    import torch
+    sp = _sp()
+    Y = f16_bits(sp.spmm(sp.encode(to_dev(W)), to_dev(X)))
+    torch.cuda.synchronize()
+    exp = Yref.astype(np.float16).view(np.uint16)
+    assert np.array_equal(Y, exp), f"{kernel} N={N}: {int(np.count_nonzero(Y != exp))} mismatches"
 
 
 @pytest.mark.parametrize("s", [0.0, 0.3, 0.4, 0.6, 0.7, 0.95])
