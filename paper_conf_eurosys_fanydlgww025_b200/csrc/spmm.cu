@@ -77,6 +77,20 @@ constexpr int kMaxStages = 8;
 #define SPINFER_ROLEREG 56
 #endif
 // software-pipelined consumer loop also for the 16-warp (KQ = 2) variant
+// asynchronous rowblock epilogue: at a segment end that is not the CTA's last, every consumer
+// warp parks its fp32 partial in the workspace (L2) and moves on; the fix-up warp sums the
+// partials in warp order (deterministic) and writes Y / joins the split-K fix-up
+#ifndef SPINFER_AEPI
+#define SPINFER_AEPI 0
+#endif
+// waits of the fix-up warp / the producer: timed back-off (not woken by the CTA's other barrier
+// traffic) instead of the event-woken suspend of mbar_wait_sleep; 0 = suspend
+#ifndef SPINFER_FIXBO
+#define SPINFER_FIXBO 0
+#endif
+#ifndef SPINFER_PRODBO
+#define SPINFER_PRODBO 0
+#endif
 #ifndef SPINFER_EPREF
 #define SPINFER_EPREF 0
 #endif
@@ -100,6 +114,7 @@ struct Params {
     const uint16_t *X;
     uint16_t *Y;
     float *ws_part;
+    float *ws_epi;      // [P][2 buffers][kR][8 warps][64 x N] fp32 partials of the asynchronous epilogue
     int32_t *ws_cnt;
     int KG, MG;
     int N;                                      // real N (the tcgen05 path pads X to NB via TMA OOB fill)
@@ -327,6 +342,8 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     // the scan warps acquired full[s] first, so consumers wait on scanned[s] only)
     const uint32_t bar_scan = sbase + 16 * kMaxStages;
     const uint32_t bar_fix = sbase + 208;   // [split segment A/C][GT row]: partial parked (32 lanes)
+    const uint32_t bar_epi = sbase + 256;   // [buffer][GT row]: the row's consumer warps parked their partials
+    const uint32_t bar_epifree = sbase + 288;   // [buffer]: the fix-up warp has read the buffer
 
     if (lane == 0) trace_k(prm, p, warp, 0);
     if (threadIdx.x == 0) {
@@ -336,6 +353,8 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         }
         for (int s = 0; s < S; ++s) mbar_init(bar_scan + 8 * s, kScanWarps);   // one elected arrive per scan warp
         for (int k = 0; k < 2 * kR; ++k) mbar_init(bar_fix + 8 * k, 32);
+        for (int k = 0; k < 2 * kR; ++k) mbar_init(bar_epi + 8 * k, 4 * KQ);
+        for (int k = 0; k < 2; ++k) mbar_init(bar_epifree + 8 * k, 1);
         fence_barrier_init();
         // SMBD selector-table constants, read back into registers by every consumer thread so
         // ptxas keeps them live in registers instead of re-materialising them per PRMT.
@@ -377,7 +396,11 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             const int i = sg.i, slot = sg.slot;
             if ((dbg_mode(prm) & 4) && i > 0) break;   // experiment: consumers reuse stage 0 forever
             trace_ev(prm, p, i, warp, 0);
+#if SPINFER_PRODBO
+            if (i >= S) mbar_wait_backoff(bar_empty + 8 * slot, sg.par() ^ 1u, 32u, SPINFER_PRODBO);
+#else
             if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, sg.par() ^ 1u);
+#endif
             const uint32_t st = sbase + prm.o_stage + slot * prm.stage_bytes;
             const uint32_t fb = bar_full + 8 * slot;
             const uint32_t bmb = (uint32_t)sg.g * 512u;
@@ -406,6 +429,93 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     }
 
     if (warp == kFixWarp) {
+#if SPINFER_AEPI
+        // ------------------------------------------------------------ epilogue + split-K fix-up
+        // Walks the CTA's stage sequence. At every segment end except the last: waits for the
+        // row's 4*KQ consumer partials (workspace, L2), sums them in warp order, and writes Y
+        // (complete rowblock) or parks the CTA partial and joins the cross-CTA count; the last
+        // contributor sums all partials in CTA order. The CTA's last segment is reduced
+        // by the consumers themselves (nothing left to overlap); if it is split, its leader
+        // parks the partial on bar_fix as before.
+        {
+            StageIter d;
+            bool full_start = false;
+            int segi = 0;
+            for (d.init(u0, u1, prm); d.valid();) {
+                const bool zero = d.seg_first();
+                if (zero) full_start = (d.gc == 0);
+                const bool seg_end = d.seg_last(prm);
+                const bool complete = seg_end && full_start && (d.gc + d.g == KG);
+                const int rb = d.rb, rows = d.rows;
+                d.next(prm);
+                if (!seg_end) continue;
+                const bool last = !d.valid();
+                const int myslot = (rb == u0 / KG) ? 0 : 1;
+                const int pf = unit_owner(rb * KG, U, prm.P);
+                const int pl = unit_owner((rb + 1) * KG - 1, U, prm.P);
+                auto count_and_sum = [&](int r) {
+                    int old = 0;
+                    if (lane == 0) old = atomicAdd(prm.ws_cnt + kR * rb + r, 1);
+                    old = __shfl_sync(0xffffffffu, old, 0);
+                    if (old == pl - pf) fixup_sum<NT>(prm, rb, r, pf, pl, lane);   // last contributor
+                };
+                if (last) {
+                    if (!complete)
+                        for (int r = 0; r < rows; ++r) {
+                            mbar_wait_sleep(bar_fix + 8u * (uint32_t)(2 * myslot + r), 0u);
+                            __threadfence();   // cumulative: the consumer's partial stores before the count
+                            count_and_sum(r);
+                        }
+                    break;
+                }
+                const uint32_t buf = (uint32_t)segi & 1u, ph = ((uint32_t)segi >> 1) & 1u;
+                for (int r = 0; r < rows; ++r) {
+                    mbar_wait_sleep(bar_epi + 8u * (buf * kR + (uint32_t)r), ph);
+                    float acc[4][NT][4];
+#pragma unroll
+                    for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                        for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) acc[tr][nt][e] = 0.f;
+                    const float4 *src = reinterpret_cast<const float4 *>(prm.ws_epi) +
+                                        (((size_t)p * 2 + buf) * kR + r) * 8 * (64 * N / 4);
+                    for (int w = 0; w < 4 * KQ; ++w)
+#pragma unroll
+                        for (int tr = 0; tr < 4; ++tr) {
+                            float4 v[NT];
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt)
+                                v[nt] = ldg_cg_f4(src + (size_t)w * (64 * N / 4) + (tr * NT + nt) * 32 + lane);
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt) {
+                                acc[tr][nt][0] += v[nt].x; acc[tr][nt][1] += v[nt].y;
+                                acc[tr][nt][2] += v[nt].z; acc[tr][nt][3] += v[nt].w;
+                            }
+                        }
+                    const int grow = kR * rb + r;
+                    if (complete) {
+                        store_y<NT>(prm.Y, N, grow * 64, acc, lane);
+                    } else {
+                        float4 *part = reinterpret_cast<float4 *>(prm.ws_part) + (((size_t)p * 2 + myslot) * kR + r) * (64 * N / 4);
+#pragma unroll
+                        for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt)
+                                part[(tr * NT + nt) * 32 + lane] =
+                                    make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]);
+                        __threadfence();
+                        __syncwarp();
+                        count_and_sum(r);
+                    }
+                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(bar_epifree + 8u * buf);   // the buffer may be overwritten
+                ++segi;
+            }
+        }
+        return;
+#endif
         // ------------------------------------------------------------ split-K fix-up
         // At most two split segments per CTA (A: tail of the first rowblock, C: head of the
         // last), processed first in StageIter order; for each and each GT row the reducing
@@ -419,7 +529,13 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             const int myslot = (rb == u0 / KG) ? 0 : 1;
             const int rows = min(kR, prm.MG - kR * rb);
             for (int r = 0; r < rows; ++r) {
+#if SPINFER_FIXBO
+                // the parked partial is not urgent: poll every few microseconds at most instead of
+                // waking on each of the CTA's ~30 barrier events per stage
+                mbar_wait_backoff(bar_fix + 8u * (uint32_t)(2 * myslot + r), 0u, 256u, 2048u);
+#else
                 mbar_wait_sleep(bar_fix + 8u * (uint32_t)(2 * myslot + r), 0u);
+#endif
                 __threadfence();   // cumulative: the consumer's partial stores before the count
                 const int pf = unit_owner(rb * KG, U, prm.P);
                 const int pl = unit_owner((rb + 1) * KG - 1, U, prm.P);
@@ -652,6 +768,8 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     // the next stage's descriptor is fetched during the current stage's decode (a shared load
     // at a stage boundary waits behind the decode traffic in the MIO queue)
     StageDesc dn = rd(0);
+    int segi = 0;   // segment ends seen (asynchronous epilogue buffer / phase)
+    (void)segi;
     for (int i = 0; i < nst; ++i) {
         const int cw = warp;
         const StageDesc d = dn;
@@ -724,6 +842,25 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         if (lane == 0) trace_ev(prm, p, i, cw, 2);   // decode done
         const StageDesc e = d;
         const int rb = e.rb(), rows = e.rows();
+#if SPINFER_AEPI
+        if (e.seg_end() && i + 1 < nst) {
+            // asynchronous epilogue (not the CTA's last segment): park this warp's partial, move on
+            const uint32_t buf = (uint32_t)segi & 1u, use = (uint32_t)segi >> 1;
+            ++segi;
+            if (r < rows && !(dbg_mode(prm) & 8)) {
+                if (use > 0) mbar_wait_sleep(bar_epifree + 8u * buf, (use - 1u) & 1u);
+                float4 *dst = reinterpret_cast<float4 *>(prm.ws_epi) +
+                              ((((size_t)p * 2 + buf) * kR + r) * 8 + (size_t)(c * KQ + q)) * (64 * N / 4);
+#pragma unroll
+                for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                    for (int nt = 0; nt < NT; ++nt)
+                        dst[(tr * NT + nt) * 32 + lane] = make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]);
+                __syncwarp();
+                if (lane == 0) mbar_arrive(bar_epi + 8u * (buf * kR + (uint32_t)r));   // release: the stores above
+            }
+        } else
+#endif
         if (e.seg_end() && r < rows && !(dbg_mode(prm) & 8)) {   // experiment bit 8: no epilogue
             // -------------------------------------------------------- epilogue
             // (1) reduce the 4*KQ partials of GT row r into warp (c = 0, q = 0), tree via smem.
@@ -841,6 +978,12 @@ struct TmemTC {
 constexpr uint32_t kTcFull = 0, kTcEmpty = 64, kTcEmptyX = 128, kTcTmemSlot = 208;
 constexpr uint32_t kTcAEmpty = 256, kTcDFull = 352, kTcDEmpty = 368, kTcFix = 384;   // aempty [4][3]
 constexpr uint32_t kTcScan = 512;      // [S]: the slot's SMBD table is written
+constexpr uint32_t kTcTeamCnt = 960;   // int [k-team][A buffer]: A tiles written (last of 4 writers issues the MMA)
+// k-team MMA issue by the last of the team's 4 lane-quarter warps to finish its A tiles (a shared
+// atomic count per A buffer) instead of a named barrier of the 4 warps: no warp waits for another
+#ifndef SPINFER_TC_LAST
+#define SPINFER_TC_LAST 0
+#endif
 // ring position of a multi-buffer: index and phase parity, advanced once per use
 template <int NBUF>
 struct Ring {
@@ -908,6 +1051,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
             mbar_init(bar_de + 8 * k, 4);                  // the 4 warps of the finishing k-team
         }
         for (int k = 0; k < 2; ++k) mbar_init(sbase + kTcFix + 8 * k, 4);   // split segment A / C parked
+        for (int k = 0; k < 12; ++k) reinterpret_cast<int *>(smem + kTcTeamCnt)[k] = 0;
         fence_barrier_init();
         reinterpret_cast<uint32_t *>(smem)[kConstWord] = kSelA;
         reinterpret_cast<uint32_t *>(smem)[kConstWord + 1] = kSelB;
@@ -1262,10 +1406,25 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         tm_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(bar_empty + 8 * slot);   // this warp is done with the slot's values/table
+        const bool mm = kt < it.g;
+#if SPINFER_TC_LAST
+        // the last of the team's 4 lane-quarter warps to finish its A tiles multiplies
+        bool issuer = false;
+        {
+            int old = 0;
+            if (lane == 0) {
+                __threadfence_block();   // release: this warp's TMEM stores (fenced above) before the count
+                old = atomicAdd(reinterpret_cast<int *>(smem + kTcTeamCnt) + ab, 1);
+                __threadfence_block();   // acquire: the other warps' stores before the MMA
+            }
+            issuer = (__shfl_sync(0xffffffffu, old, 0) & 3) == 3;
+        }
+#else
         // the team's 4 lane-quarter warps have written their A tiles: the team leader multiplies
         named_bar_sync(kTeamBar + (uint32_t)kt, 128);
-        const bool mm = kt < it.g;
-        if (q == 0) {
+        const bool issuer = (q == 0);
+#endif
+        if (issuer) {
             tm_fence_after();
             if (sf.zero && seg >= 2) {   // the D buffer's previous segment has been read out
                 mbar_wait(bar_de + 8u * dpar, dph ^ 1u);
@@ -1457,7 +1616,8 @@ size_t spmm_workspace_bytes(int M, int K, int N) {
     const long long U = (long long)((MG + kR - 1) / kR) * KG;
     const int P = choose_P(U);
     size_t part = (size_t)P * 2 * kR * 64 * N * 4;
-    return kCounterBytes + part;
+    size_t epi = (size_t)P * 2 * kR * 8 * 64 * N * 4;   // asynchronous epilogue partials
+    return kCounterBytes + part + epi;
 }
 
 int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *ws, size_t ws_bytes,
@@ -1485,6 +1645,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     q.Y = Y;
     q.ws_cnt = reinterpret_cast<int32_t *>(ws);
     q.ws_part = reinterpret_cast<float *>(reinterpret_cast<uint8_t *>(ws) + kCounterBytes);
+    q.ws_epi = q.ws_part + (size_t)pl.P * 2 * kR * 64 * N;
     q.dbg = 0;
     if (const char *e = getenv("SPINFER_DEBUG_MODE")) q.dbg = atoi(e);
     q.trace = nullptr;
