@@ -124,12 +124,14 @@ def test_spmm_deterministic_and_workspace_reusable():
     assert int(cnt.abs().sum()) == 0
 
 
-def test_spmm_config2_sampled_rows():
-    """Full-size config 2 (M/K/N = 28672/8192/16, s = 0.5) in the launch bench.py times;
-    parity on sampled rows (incl. first/last rows and rowblock/CTA boundaries)."""
+@pytest.mark.parametrize("N", [16, 32])
+def test_spmm_config2_sampled_rows(N):
+    """Full-size config 2 (M/K = 28672/8192, s = 0.5) in the launch bench.py times (N = 16:
+    mma.sync kernel; N = 32: tcgen05 kernel); parity on sampled rows (incl. first/last rows
+    and rowblock/CTA boundaries)."""
     import torch
     sp = _sp()
-    M, K, N = 28672, 8192, 16
+    M, K = 28672, 8192
     W = synth.weight(M, K, 0.5)
     X = synth.activation(K, N)
     T = sp.encode(to_dev(W))
