@@ -216,6 +216,14 @@ def run_ours(a, rank, world, local_rank):
         evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
         barrier()
         torch.cuda.synchronize()
+        # ~1 ms of device-side spin ahead of the loop, outside every event pair: the host gets
+        # ahead of the device, so no step's events also time a host-side launch gap (without it
+        # the first timed step read 257-384 us against 84-86 us for the others, profiles/r1_steps)
+        torch.cuda._sleep(2_000_000)
+        for _ in range(2):   # untimed lead-in steps in the same burst (the first step after a host
+            if do_flush:     # synchronize also ran slow: profiles/r1_steps.txt)
+                flush_l2()
+            fn()
         for i in range(steps):
             if do_flush:
                 flush_l2()
@@ -336,7 +344,7 @@ def run_ours(a, rank, world, local_rank):
         "config": {"workload": workload_name(a), "M": M, "K": K, "N": N, "sparsity": a.sparsity,
                    "nnz": T.nnz, "n_values": T.n_values, "seed": a.seed, "l2": "flushed before each step: 256 MiB memset, then a 256 MiB read (cold, clean L2)",
                    "parallelism": f"row-partitioned x{world} (weak, no collective)" if world > 1 else "1 GPU"},
-        "us_per_spmm": kmax * 1e3, "us_median": kern_med * 1e3,
+        "us_per_spmm": kmax * 1e3, "us_median": kern_med * 1e3, "us_steps": [round(x * 1e3, 1) for x in t_ms],
         "tflops_dense_equiv": 2 * M * K * N / (kern_ms * 1e-3) / 1e12,
         "frac_of_8tbs": achieved / 8000.0,
         "cublas_fp16": cublas,

@@ -113,6 +113,9 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t
 // cp.async.mbarrier.arrive.noinc makes the barrier observe one arrival when all of
 // this thread's prior cp.async operations have completed.
 // 2-D TMA tile load (tensor map in param/const space, coordinates innermost first).
+__device__ __forceinline__ void prefetch_l2(const void *p) {
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
 // Pulls a tensor map (here: a __grid_constant__ kernel parameter) into the TMA unit's
 // descriptor cache ahead of its first use.
 __device__ __forceinline__ void prefetch_tmap(const void *tmap) {

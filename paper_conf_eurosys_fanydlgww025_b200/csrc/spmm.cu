@@ -91,6 +91,9 @@ constexpr int kMaxStages = 8;
 #ifndef SPINFER_PRODBO
 #define SPINFER_PRODBO 0
 #endif
+#ifndef SPINFER_PAGEPF
+#define SPINFER_PAGEPF 1
+#endif
 #ifndef SPINFER_EPREF
 #define SPINFER_EPREF 0
 #endif
@@ -125,6 +128,7 @@ struct Params {
     uint32_t tbl_bytes;
     uint32_t o_desc, o_tbl, o_stage;            // region offsets from the smem base
     long long *trace;   // experiments only (SPINFER_TRACE): [kTraceCTAs][kTraceStages][8] clock64 stamps
+    float avg_gt;       // n_values / NGT: predicts where a CTA's first value range lies (start-up page prefetch)
     int dbg;            // experiments only (SPINFER_DEBUG_MODE): bit0 = consumers skip decode/MMA, bit1 = scan skips work
 };
 
@@ -376,6 +380,18 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     };
     if (warp == kProducerWarp && lane == 0) {
         prefetch_tmap(&prm.tmap_x);
+#if SPINFER_PAGEPF
+        // Start-up: the first value copies wait for their GTileOffset entries; touching the
+        // predicted first value line of each GT row now overlaps that page's translation with
+        // the offset loads (a hint only: nothing depends on the prediction).
+        {
+            const int rb0 = u0 / KG, gc0 = u0 - rb0 * KG;
+            for (int r = 0; r < kR && kR * rb0 + r < prm.MG; ++r) {
+                const long long g = (long long)(kR * rb0 + r) * KG + gc0;
+                prefetch_l2(prm.vals + (long long)((double)g * prm.avg_gt));
+            }
+        }
+#endif
         pit.init(u0, u1, prm);
         if (pit.valid()) poff = load_off(pit);
     }
@@ -1616,7 +1632,7 @@ size_t spmm_workspace_bytes(int M, int K, int N) {
     const long long U = (long long)((MG + kR - 1) / kR) * KG;
     const int P = choose_P(U);
     size_t part = (size_t)P * 2 * kR * 64 * N * 4;
-    size_t epi = (size_t)P * 2 * kR * 8 * 64 * N * 4;   // asynchronous epilogue partials
+    size_t epi = SPINFER_AEPI ? (size_t)P * 2 * kR * 8 * 64 * N * 4 : 0;   // asynchronous epilogue partials
     return kCounterBytes + part + epi;
 }
 
@@ -1646,6 +1662,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     q.ws_cnt = reinterpret_cast<int32_t *>(ws);
     q.ws_part = reinterpret_cast<float *>(reinterpret_cast<uint8_t *>(ws) + kCounterBytes);
     q.ws_epi = q.ws_part + (size_t)pl.P * 2 * kR * 64 * N;
+    q.avg_gt = (float)((double)T->n_values / ((double)(M / kGT) * (double)(K / kGT)));
     q.dbg = 0;
     if (const char *e = getenv("SPINFER_DEBUG_MODE")) q.dbg = atoi(e);
     q.trace = nullptr;
