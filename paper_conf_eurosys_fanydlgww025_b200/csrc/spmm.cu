@@ -148,10 +148,23 @@ __device__ __forceinline__ void trace_ev(const Params &prm, int p, int i, int w,
         prm.trace[(((size_t)p * kTraceStages + i) * kTraceW + w) * kTraceEv + ev] = clock64();
 #endif
 }
+constexpr size_t kTraceBase2 = (size_t)kTraceCTAs * kTraceStages * kTraceW * kTraceEv;   // then [CTA][entry, exit] ns
+constexpr int kTraceMaxCTAs = 1024;
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
 __device__ __forceinline__ void trace_k(const Params &prm, int p, int w, int ev) {
 #if SPINFER_INSTRUMENT == 1
     if (prm.trace && p < kTraceCTAs && w < kTraceW)
         prm.trace[(((size_t)p * kTraceStages + kTraceStages - 1) * kTraceW + w) * kTraceEv + ev] = clock64();
+    // every CTA: entry (warp 0) and exit (last warp out) on the global ns timer
+    if (prm.trace && p < kTraceMaxCTAs) {
+        unsigned long long *g = reinterpret_cast<unsigned long long *>(prm.trace + kTraceBase2);
+        if (ev == 0 && w == 0) g[2 * p] = globaltimer_ns();
+        if (ev == 3) atomicMax(g + 2 * p + 1, globaltimer_ns());
+    }
 #endif
 }
 __device__ __forceinline__ int dbg_mode(const Params &prm) {
@@ -997,6 +1010,9 @@ constexpr uint32_t kTcScan = 512;      // [S]: the slot's SMBD table is written
 constexpr uint32_t kTcTeamCnt = 960;   // int [k-team][A buffer]: A tiles written (last of 4 writers issues the MMA)
 // k-team MMA issue by the last of the team's 4 lane-quarter warps to finish its A tiles (a shared
 // atomic count per A buffer) instead of a named barrier of the 4 warps: no warp waits for another
+#ifndef SPINFER_TC_WARPFIX
+#define SPINFER_TC_WARPFIX 1
+#endif
 #ifndef SPINFER_TC_LAST
 #define SPINFER_TC_LAST 0
 #endif
@@ -1111,6 +1127,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         const bool has_a = (u0 % KG) != 0;
         const bool has_c = (u1 % KG) != 0 && !(has_a && c_rb == a_rb);
         int fx = has_a ? 0 : (has_c ? 1 : 2);   // next split segment to serve (2: none left)
+        if (SPINFER_TC_WARPFIX) fx = 2;          // the epilogue warps do the fix-up themselves
         auto fixup = [&](int sgi) {
             const int rb = sgi == 0 ? a_rb : c_rb;
             const int rows = min(kR, prm.MG - kR * rb);
@@ -1329,10 +1346,44 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
             for (int c4 = 0; c4 < NB / 4; ++c4)
                 if (c4 * 4 < N) pp[c4] = make_float4(v[4 * c4], v[4 * c4 + 1], v[4 * c4 + 2], v[4 * c4 + 3]);
         }
+#if SPINFER_TC_WARPFIX
+        // split-K fix-up per lane quarter, by the warp that parked it (one counter per rowblock
+        // and quarter): the last contributor sums every contributor's partial of its 32 rows in
+        // CTA order (deterministic), writes Y and re-zeroes the counter. A lane owns one
+        // row, so all partials' loads of a row are in flight together (the single producer lane
+        // group serving it measured a 10-20 us tail on CTAs whose last segment is split).
+        __threadfence();
+        __syncwarp();
+        const int pf = unit_owner(rb * KG, U, prm.P);
+        const int pl = unit_owner((rb + 1) * KG - 1, U, prm.P);
+        int old = 0;
+        if (lane == 0) old = atomicAdd(prm.ws_cnt + 4 * rb + q, 1);
+        old = __shfl_sync(0xffffffffu, old, 0);
+        if (old != pl - pf) return;
+        __threadfence();
+        if (valid) {
+            // v (this CTA's partial, parked above) is re-used as the sum
+#pragma unroll
+            for (int j = 0; j < NB; ++j) v[j] = 0.f;
+            for (int qq = pf; qq <= pl; ++qq) {
+                const int sl = (rb == unit_start(qq, U, prm.P) / KG) ? 0 : 1;
+                const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part + (((size_t)qq * 2 + sl) * 128 + row_in) * N);
+#pragma unroll
+                for (int c4 = 0; c4 < NB / 4; ++c4)
+                    if (c4 * 4 < N) {
+                        const float4 x = ldg_cg_f4(pp + c4);
+                        v[4 * c4] += x.x; v[4 * c4 + 1] += x.y; v[4 * c4 + 2] += x.z; v[4 * c4 + 3] += x.w;
+                    }
+            }
+            store_y_row<NB>(prm.Y, (size_t)rb * 128 + (size_t)row_in, N, v);
+        }
+        if (lane == 0) prm.ws_cnt[4 * rb + q] = 0;   // leave the workspace zeroed
+#else
         __threadfence();
         __syncwarp();
         const bool is_a = (u0 % KG) != 0 && rb == u0 / KG;
         if (lane == 0) mbar_arrive(sbase + kTcFix + (is_a ? 0u : 8u));
+#endif
     };
 
     uint4 E[4];
@@ -1647,6 +1698,8 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     bool tc = N >= 24;
     if (ke && ke[0] == 't') tc = true;
     if (ke && ke[0] == 'm') tc = false;
+    // the tcgen05 kernel's fix-up keeps one counter per rowblock and TMEM lane quarter
+    if (tc && 4LL * ((M / kGT + kR - 1) / kR) > kMaxCounters) tc = false;
     if (!make_plan(M, K, N, T->max_gt_values, &pl, tc)) return SPINFER_EINVAL;
     const size_t need = spmm_workspace_bytes(M, K, N);
     if (need == 0) return SPINFER_EINVAL;
@@ -1668,7 +1721,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     q.trace = nullptr;
     static long long *trace_buf = nullptr;
     const char *trace_path = getenv("SPINFER_TRACE");
-    const size_t trace_n = (size_t)kTraceCTAs * kTraceStages * kTraceW * kTraceEv;
+    const size_t trace_n = kTraceBase2 + 2 * kTraceMaxCTAs;
     if (trace_path) {
         if (!trace_buf && cudaMalloc(&trace_buf, trace_n * 8) != cudaSuccess) return SPINFER_ECUDA;
         cudaMemsetAsync(trace_buf, 0, trace_n * 8, st);
@@ -1685,7 +1738,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
         default: break;
     }
     if (trace_path && rc == SPINFER_OK) {   // debug only: synchronous dump of the stage timeline
-        static long long host[kTraceCTAs * kTraceStages * kTraceW * kTraceEv];
+        static long long host[kTraceBase2 + 2 * kTraceMaxCTAs];
         cudaMemcpyAsync(host, trace_buf, sizeof(host), cudaMemcpyDeviceToHost, st);
         cudaStreamSynchronize(st);
         if (FILE *f = fopen(trace_path, "wb")) { fwrite(host, 1, sizeof(host), f); fclose(f); }

@@ -1,1 +1,3 @@
-timeout 200 python bench.py --steps 40 --warmup 5 --no-cpu-baseline --no-e2e --json-out gpurun_out/st.json > /dev/null 2>&1; python -c "import json;d=json.load(open('gpurun_out/st.json'));print(d['us_steps']); print(d['us_per_spmm'], d['us_median'], 'cublas', d['cublas_fp16']['us'])"
+SPINFER_KERNEL=tc timeout 600 python -m pytest tests/test_spmm_gpu.py -x -q --timeout 120 2>&1 | tail -2
+BENCH_ARGS="--N 32" bash tools/ab.sh "tcnowf:libspinfer_tcnowf.so:" "tcwf:libspinfer_tcwf.so:"
+timeout 200 env SPINFER_KERNEL=tc python tools/cta_times.py 32
