@@ -148,7 +148,7 @@ __device__ __forceinline__ void trace_ev(const Params &prm, int p, int i, int w,
         prm.trace[(((size_t)p * kTraceStages + i) * kTraceW + w) * kTraceEv + ev] = clock64();
 #endif
 }
-constexpr size_t kTraceBase2 = (size_t)kTraceCTAs * kTraceStages * kTraceW * kTraceEv;   // then [CTA][entry, exit] ns
+constexpr size_t kTraceBase2 = (size_t)kTraceCTAs * kTraceStages * kTraceW * kTraceEv;   // then [CTA][entry, exit] ns, [CTA] smid
 constexpr int kTraceMaxCTAs = 1024;
 __device__ __forceinline__ unsigned long long globaltimer_ns() {
     unsigned long long t;
@@ -162,7 +162,12 @@ __device__ __forceinline__ void trace_k(const Params &prm, int p, int w, int ev)
     // every CTA: entry (warp 0) and exit (last warp out) on the global ns timer
     if (prm.trace && p < kTraceMaxCTAs) {
         unsigned long long *g = reinterpret_cast<unsigned long long *>(prm.trace + kTraceBase2);
-        if (ev == 0 && w == 0) g[2 * p] = globaltimer_ns();
+        if (ev == 0 && w == 0) {
+            uint32_t smid;
+            asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+            g[2 * p] = globaltimer_ns();
+            g[2 * kTraceMaxCTAs + p] = smid;
+        }
         if (ev == 3) atomicMax(g + 2 * p + 1, globaltimer_ns());
     }
 #endif
@@ -1721,7 +1726,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     q.trace = nullptr;
     static long long *trace_buf = nullptr;
     const char *trace_path = getenv("SPINFER_TRACE");
-    const size_t trace_n = kTraceBase2 + 2 * kTraceMaxCTAs;
+    const size_t trace_n = kTraceBase2 + 3 * kTraceMaxCTAs;
     if (trace_path) {
         if (!trace_buf && cudaMalloc(&trace_buf, trace_n * 8) != cudaSuccess) return SPINFER_ECUDA;
         cudaMemsetAsync(trace_buf, 0, trace_n * 8, st);
@@ -1738,7 +1743,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
         default: break;
     }
     if (trace_path && rc == SPINFER_OK) {   // debug only: synchronous dump of the stage timeline
-        static long long host[kTraceBase2 + 2 * kTraceMaxCTAs];
+        static long long host[kTraceBase2 + 3 * kTraceMaxCTAs];
         cudaMemcpyAsync(host, trace_buf, sizeof(host), cudaMemcpyDeviceToHost, st);
         cudaStreamSynchronize(st);
         if (FILE *f = fopen(trace_path, "wb")) { fwrite(host, 1, sizeof(host), f); fclose(f); }

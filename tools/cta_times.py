@@ -31,9 +31,14 @@ for rep in range(3):
     torch.cuda.synchronize()
     tr = np.fromfile(os.environ["SPINFER_TRACE"], dtype=np.int64)
     g = tr[base:base + 2 * 1024].reshape(1024, 2)
-    g = g[g[:, 0] > 0]
+    smid = tr[base + 2 * 1024:base + 3 * 1024]
+    live = g[:, 0] > 0
+    g, smid = g[live], smid[live]
     t0 = g[:, 0].min()
     ent, ex = (g[:, 0] - t0) / 1e3, (g[:, 1] - t0) / 1e3
     print(f"rep {rep}: event {e0.elapsed_time(e1)*1e3:.1f} us; CTAs {len(g)}; entry spread {ent.max():.2f} us; "
           f"exit min/med/max {ex.min():.1f}/{np.median(ex):.1f}/{ex.max():.1f} us; "
           f"latest 5 exits (CTA: us) {[(int(i), round(float(ex[i]),1)) for i in np.argsort(-ex)[:5]]}")
+    if rep == 2:
+        order = np.argsort(smid)
+        print("exit (us) by SM id:", " ".join(f"{int(smid[i])}:{ex[i]:.1f}" for i in order))

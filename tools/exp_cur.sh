@@ -1,3 +1,2 @@
-SPINFER_KERNEL=tc timeout 600 python -m pytest tests/test_spmm_gpu.py -x -q --timeout 120 2>&1 | tail -2
-BENCH_ARGS="--N 32" bash tools/ab.sh "tcnowf:libspinfer_tcnowf.so:" "tcwf:libspinfer_tcwf.so:"
-timeout 200 env SPINFER_KERNEL=tc python tools/cta_times.py 32
+timeout 900 python tools/sweep.py --out gpurun_out/r1e_sweep.jsonl > gpurun_out/sweep_r1e.log 2>&1; tail -3 gpurun_out/sweep_r1e.log
+bash tools/gpu_round.sh r1e

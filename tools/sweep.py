@@ -60,6 +60,11 @@ def main():
     def timed(fn, steps):
         evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
         torch.cuda.synchronize()
+        torch.cuda._sleep(2_000_000)   # device-side lead-in, as in bench.py (no host gap inside a step's events)
+        for _ in range(2):
+            flush.zero_()
+            flush_rd.sum()
+            fn()
         for i in range(steps):
             flush.zero_()
             flush_rd.sum()

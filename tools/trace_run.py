@@ -30,7 +30,7 @@ flush.zero_()
 torch.cuda.synchronize()
 sp.spmm(T, Xd)
 torch.cuda.synchronize()
-tr = np.fromfile(os.environ["SPINFER_TRACE"], dtype=np.int64).reshape(4, 64, 20, 4)
+tr = np.fromfile(os.environ["SPINFER_TRACE"], dtype=np.int64)[:4 * 64 * 20 * 4].reshape(4, 64, 20, 4)
 
 NCW = 16
 for p in range(2):

@@ -33,7 +33,7 @@ flush.zero_()
 torch.cuda.synchronize()
 sp.spmm(T, Xd)
 torch.cuda.synchronize()
-tr = np.fromfile(os.environ["SPINFER_TRACE"], dtype=np.int64).reshape(4, 64, 20, 4)
+tr = np.fromfile(os.environ["SPINFER_TRACE"], dtype=np.int64)[:4 * 64 * 20 * 4].reshape(4, 64, 20, 4)
 
 PW = 16   # producer warp (decode warps 0-15; k-team leaders issue the MMAs)
 for p in range(2):
