@@ -97,7 +97,8 @@ SPINFER_API int spinfer_decode(const spinfer_tca *T, uint16_t *W_out, void *stre
 
 /* Bytes of device workspace spinfer_spmm needs for this shape: a fixed 64 KiB
  * region of split-K fix-up counters (one int32 per GT row; M <= 1,048,576)
- * followed by fp32 split-K partials. 0 for an invalid shape. The workspace must
+ * followed by fp32 split-K partials and, when N is not a multiple of 8, a
+ * zero-padded copy of X (K x roundup(N, 8) fp16). 0 for an invalid shape. The workspace must
  * be ZERO-FILLED before its first use; every spinfer_spmm call leaves the
  * counter region zero again, so one zeroed workspace (sized for the largest
  * shape) can be reused by successive calls of any shape on ONE stream — never
@@ -106,8 +107,9 @@ SPINFER_API size_t spinfer_spmm_workspace_bytes(int M, int K, int N);
 
 /* Y = W x X with fp32 accumulation and one round-to-nearest-even to
  * fp16 per output. X: device fp16 [K][N] row-major; Y: device fp16
- * [M][N] row-major (fully overwritten). N in {8, 16, 24, 32} (decode batch,
- * P:329). One persistent kernel launch (stream-K over GroupTiles with an
+ * [M][N] row-major (fully overwritten). 1 <= N <= 32 (decode batch; the
+ * kernels compute roundup(N, 8) columns: N not a multiple of 8 costs the same as
+ * the next multiple of 8 plus a zero-padded copy of X in the workspace). One persistent kernel launch (stream-K over GroupTiles with an
  * in-kernel split-K fix-up, P:216 / Alg. 1). */
 SPINFER_API int spinfer_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N,
                  void *workspace, size_t ws_bytes, void *stream);

@@ -198,7 +198,7 @@ def workspace(M: int, K: int, N: int, device=None) -> torch.Tensor:
 
 def spmm(T: TCA, X: torch.Tensor, Y: torch.Tensor | None = None, ws: torch.Tensor | None = None,
          stream=None) -> torch.Tensor:
-    """Y = W X: X fp16 [K][N] (CUDA), N in {8,16,24,32}; returns fp16 [M][N]."""
+    """Y = W X: X fp16 [K][N] (CUDA), 1 <= N <= 32; returns fp16 [M][N]."""
     X = _dev_u16(X, "X")
     K, N = X.shape
     if K != T.K:

@@ -78,13 +78,13 @@ int spinfer_decode(const spinfer_tca *T, uint16_t *W_out, void *stream) {
 }
 
 size_t spinfer_spmm_workspace_bytes(int M, int K, int N) {
-    if (!shape_ok(M, K) || (N != 8 && N != 16 && N != 24 && N != 32)) return 0;
+    if (!shape_ok(M, K) || N < 1 || N > 32) return 0;
     return spmm_workspace_bytes(M, K, N);
 }
 
 int spinfer_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *workspace,
                  size_t ws_bytes, void *stream) {
-    if (!X || !Y || (N != 8 && N != 16 && N != 24 && N != 32)) return SPINFER_EINVAL;
+    if (!X || !Y || N < 1 || N > 32) return SPINFER_EINVAL;
     if (!aligned16(X) || !aligned16(Y) || (workspace && !aligned16(workspace))) return SPINFER_EINVAL;
     int rc = validate_tca(T, M, K);
     if (rc) return rc;

@@ -296,6 +296,8 @@ __device__ __forceinline__ uint32_t x_swz(uint32_t k) {
 // two IMADs on the FMA pipe instead of ALU-pipe work (the ALU pipe is half rate on B200).
 constexpr uint32_t kSelA = 0x7f62u, kSelB = 0x4cbfu, kSelC = 0x2333u;
 
+// N = the caller's column count (row stride of Y); the kernel computes NT * 8 >= N columns
+// (X zero-padded to a multiple of 8) and drops the padding columns here.
 template <int NT>
 __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const float (&acc)[4][NT][4], int lane) {
 #pragma unroll
@@ -306,8 +308,15 @@ __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const 
             int col = nt * 8 + 2 * (lane & 3);
             __half2 lo = __floats2half2_rn(acc[tr][nt][0], acc[tr][nt][1]);   // one RNE per output (A11)
             __half2 hi = __floats2half2_rn(acc[tr][nt][2], acc[tr][nt][3]);
-            *reinterpret_cast<__half2 *>(Y + (size_t)r0 * N + col) = lo;
-            *reinterpret_cast<__half2 *>(Y + (size_t)(r0 + 8) * N + col) = hi;
+            if (N == NT * 8) {
+                *reinterpret_cast<__half2 *>(Y + (size_t)r0 * N + col) = lo;
+                *reinterpret_cast<__half2 *>(Y + (size_t)(r0 + 8) * N + col) = hi;
+            } else {
+                __half *y0 = reinterpret_cast<__half *>(Y + (size_t)r0 * N);
+                __half *y1 = reinterpret_cast<__half *>(Y + (size_t)(r0 + 8) * N);
+                if (col < N) { y0[col] = __low2half(lo); y1[col] = __low2half(hi); }
+                if (col + 1 < N) { y0[col + 1] = __high2half(lo); y1[col + 1] = __high2half(hi); }
+            }
         }
 }
 
@@ -336,7 +345,7 @@ __device__ __forceinline__ void fixup_sum(const Params &prm, int rb, int r, int 
             }
     }
     const int grow = kR * rb + r;
-    store_y<NT>(prm.Y, N, grow * 64, acc, lane);
+    store_y<NT>(prm.Y, prm.N, grow * 64, acc, lane);
     if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed
 }
 
@@ -529,7 +538,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                         }
                     const int grow = kR * rb + r;
                     if (complete) {
-                        store_y<NT>(prm.Y, N, grow * 64, acc, lane);
+                        store_y<NT>(prm.Y, prm.N, grow * 64, acc, lane);
                     } else {
                         float4 *part = reinterpret_cast<float4 *>(prm.ws_part) + (((size_t)p * 2 + myslot) * kR + r) * (64 * N / 4);
 #pragma unroll
@@ -939,7 +948,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                 const int grow = kR * rb + r;
                 const int row_base = grow * 64;
                 if (e.complete()) {
-                    store_y<NT>(prm.Y, N, row_base, acc, lane);
+                    store_y<NT>(prm.Y, prm.N, row_base, acc, lane);
                 } else {
                     // split rowblock (split-K fix-up, the paper's ReductionWorkspace P:231): park the
                     // fp32 partial; the fix-up warp counts it and the last contributor sums all
@@ -1041,6 +1050,13 @@ struct SegFlags {
 
 template <int NB>
 __device__ __forceinline__ void store_y_row(uint16_t *Y, size_t grow, int N, const float (&v)[NB]) {
+    if (N % 8) {   // N not a multiple of 8 (X was zero-padded): rows are not 16-byte aligned
+        __half *y = reinterpret_cast<__half *>(Y + grow * (size_t)N);
+#pragma unroll
+        for (int j = 0; j < NB; ++j)
+            if (j < N) y[j] = __float2half_rn(v[j]);   // one RNE per output (A11)
+        return;
+    }
     uint4 *yp = reinterpret_cast<uint4 *>(Y + grow * (size_t)N);
 #pragma unroll
     for (int c8 = 0; c8 < NB / 8; ++c8)
@@ -1128,6 +1144,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         // fix[A/C]; this warp counts it and, as the last contributor, sums all partials in CTA
         // order (deterministic), writes Y and re-zeroes the counter (ReductionWorkspace).
         const int N = prm.N;
+    const int Nw = (N + 7) & ~7;   // partial row stride (X was padded to a multiple of 8)
         const int a_rb = u0 / KG, c_rb = (u1 - 1) / KG;
         const bool has_a = (u0 % KG) != 0;
         const bool has_c = (u1 % KG) != 0 && !(has_a && c_rb == a_rb);
@@ -1150,10 +1167,10 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
                 for (int j = 0; j < NB; ++j) v[j] = 0.f;
                 for (int qq = pf; qq <= pl; ++qq) {
                     const int sl = (rb == unit_start(qq, U, prm.P) / KG) ? 0 : 1;
-                    const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part + (((size_t)qq * 2 + sl) * 128 + row_in) * N);
+                    const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part + (((size_t)qq * 2 + sl) * 128 + row_in) * Nw);
 #pragma unroll
                     for (int c4 = 0; c4 < NB / 4; ++c4)
-                        if (c4 * 4 < N) {
+                        if (c4 * 4 < Nw) {
                             const float4 x = ldg_cg_f4(pp + c4);
                             v[4 * c4] += x.x; v[4 * c4 + 1] += x.y; v[4 * c4 + 2] += x.z; v[4 * c4 + 3] += x.w;
                         }
@@ -1310,6 +1327,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
     const uint32_t selB = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 1];
     const uint32_t selC = reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 2];
     const int N = prm.N;
+    const int Nw = (N + 7) & ~7;   // partial row stride (X was padded to a multiple of 8)
     const int row_in = 32 * q + lane;               // row within the 128-row rowblock (= TMEM lane)
     const uint32_t tbl_lane = (uint32_t)(lane >> 4) * 512u + (uint32_t)(q & 1) * 64u;   // + GT * 1024 + tc * 128
 
@@ -1346,10 +1364,10 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         // split rowblock: park this CTA's fp32 partial; the producer warp does the fix-up
         const int myslot = (rb == u0 / KG) ? 0 : 1;
         if (valid) {
-            float4 *pp = reinterpret_cast<float4 *>(prm.ws_part + (((size_t)p * 2 + myslot) * 128 + row_in) * N);
+            float4 *pp = reinterpret_cast<float4 *>(prm.ws_part + (((size_t)p * 2 + myslot) * 128 + row_in) * Nw);
 #pragma unroll
             for (int c4 = 0; c4 < NB / 4; ++c4)
-                if (c4 * 4 < N) pp[c4] = make_float4(v[4 * c4], v[4 * c4 + 1], v[4 * c4 + 2], v[4 * c4 + 3]);
+                if (c4 * 4 < Nw) pp[c4] = make_float4(v[4 * c4], v[4 * c4 + 1], v[4 * c4 + 2], v[4 * c4 + 3]);
         }
 #if SPINFER_TC_WARPFIX
         // split-K fix-up per lane quarter, by the warp that parked it (one counter per rowblock
@@ -1372,10 +1390,10 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
             for (int j = 0; j < NB; ++j) v[j] = 0.f;
             for (int qq = pf; qq <= pl; ++qq) {
                 const int sl = (rb == unit_start(qq, U, prm.P) / KG) ? 0 : 1;
-                const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part + (((size_t)qq * 2 + sl) * 128 + row_in) * N);
+                const float4 *pp = reinterpret_cast<const float4 *>(prm.ws_part + (((size_t)qq * 2 + sl) * 128 + row_in) * Nw);
 #pragma unroll
                 for (int c4 = 0; c4 < NB / 4; ++c4)
-                    if (c4 * 4 < N) {
+                    if (c4 * 4 < Nw) {
                         const float4 x = ldg_cg_f4(pp + c4);
                         v[4 * c4] += x.x; v[4 * c4 + 1] += x.y; v[4 * c4 + 2] += x.z; v[4 * c4 + 3] += x.w;
                     }
@@ -1541,6 +1559,16 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
     if (lane == 0) trace_k(prm, p, warp, 3);
 }
 
+// X [K][N] -> Xp [K][Np] with zero columns N..Np-1 (N not a multiple of 8)
+__global__ void k_pad_x(const uint16_t *__restrict__ X, uint16_t *__restrict__ Xp, int K, int N, int Np) {
+    const long long tot = (long long)K * Np;
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < tot; i += (long long)gridDim.x * blockDim.x) {
+        const int k = (int)(i / Np), n = (int)(i - (long long)k * Np);
+        Xp[i] = n < N ? X[(size_t)k * N + n] : (uint16_t)0;
+    }
+}
+inline size_t align_up_sz(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
 struct Plan {
     int P, G, S;
     long long U;
@@ -1687,9 +1715,11 @@ size_t spmm_workspace_bytes(int M, int K, int N) {
     const int MG = M / kGT, KG = K / kGT;
     const long long U = (long long)((MG + kR - 1) / kR) * KG;
     const int P = choose_P(U);
-    size_t part = (size_t)P * 2 * kR * 64 * N * 4;
-    size_t epi = SPINFER_AEPI ? (size_t)P * 2 * kR * 8 * 64 * N * 4 : 0;   // asynchronous epilogue partials
-    return kCounterBytes + part + epi;
+    const int Np = (N + 7) & ~7;   // computed columns (X zero-padded to a multiple of 8)
+    size_t part = (size_t)P * 2 * kR * 64 * Np * 4;
+    size_t epi = SPINFER_AEPI ? (size_t)P * 2 * kR * 8 * 64 * Np * 4 : 0;   // asynchronous epilogue partials
+    size_t xpad = (N % 8) ? align_up_sz((size_t)K * Np * 2, 256) : 0;      // zero-padded copy of X
+    return kCounterBytes + part + epi + xpad;
 }
 
 int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *ws, size_t ws_bytes,
@@ -1699,27 +1729,39 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     // N <= 16, the tcgen05 kernel (accumulators in TMEM) for N >= 24, where mma.sync needs twice
     // the HMMAs and accumulator registers (config 2 shape, mean us: N=24 114.9 vs 112.1, N=32
     // 126.8 vs 111.0). SPINFER_KERNEL=mma|tc overrides (tests and experiments).
+    // N not a multiple of 8: the kernels compute Np = roundup(N, 8) columns from a zero-padded
+    // copy of X in the workspace (k_pad_x) and store only the N real columns of Y
+    const int Np = (N + 7) & ~7;
     const char *ke = getenv("SPINFER_KERNEL");
-    bool tc = N >= 24;
+    bool tc = Np >= 24;
     if (ke && ke[0] == 't') tc = true;
     if (ke && ke[0] == 'm') tc = false;
     // the tcgen05 kernel's fix-up keeps one counter per rowblock and TMEM lane quarter
     if (tc && 4LL * ((M / kGT + kR - 1) / kR) > kMaxCounters) tc = false;
-    if (!make_plan(M, K, N, T->max_gt_values, &pl, tc)) return SPINFER_EINVAL;
+    if (!make_plan(M, K, Np, T->max_gt_values, &pl, tc)) return SPINFER_EINVAL;
     const size_t need = spmm_workspace_bytes(M, K, N);
     if (need == 0) return SPINFER_EINVAL;
     if (ws_bytes < need || ws == nullptr) return SPINFER_ENOSPC;
     Params &q = pl.prm;
-    if (int rc = encode_x_map(&q.tmap_x, X, K, N, tc ? (N <= 16 ? 16 : 32) : N, 64 * pl.G)) return rc;
+    const uint16_t *Xk = X;
+    if (N % 8) {
+        uint16_t *Xp = reinterpret_cast<uint16_t *>(reinterpret_cast<uint8_t *>(ws) + kCounterBytes +
+                                                    (size_t)pl.P * 2 * kR * 64 * Np * 4 +
+                                                    (SPINFER_AEPI ? (size_t)pl.P * 2 * kR * 8 * 64 * Np * 4 : 0));
+        const long long tot = (long long)K * Np;
+        k_pad_x<<<(int)std::min<long long>((tot + 255) / 256, 4096), 256, 0, st>>>(X, Xp, K, N, Np);
+        Xk = Xp;
+    }
+    if (int rc = encode_x_map(&q.tmap_x, Xk, K, Np, tc ? (Np <= 16 ? 16 : 32) : Np, 64 * pl.G)) return rc;
     q.N = N;
     q.off = T->gtile_offset;
     q.bm = T->bitmap;
     q.vals = T->values;
-    q.X = X;
+    q.X = Xk;
     q.Y = Y;
     q.ws_cnt = reinterpret_cast<int32_t *>(ws);
     q.ws_part = reinterpret_cast<float *>(reinterpret_cast<uint8_t *>(ws) + kCounterBytes);
-    q.ws_epi = q.ws_part + (size_t)pl.P * 2 * kR * 64 * N;
+    q.ws_epi = q.ws_part + (size_t)pl.P * 2 * kR * 64 * Np;
     q.avg_gt = (float)((double)T->n_values / ((double)(M / kGT) * (double)(K / kGT)));
     q.dbg = 0;
     if (const char *e = getenv("SPINFER_DEBUG_MODE")) q.dbg = atoi(e);
@@ -1734,8 +1776,8 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     }
     int rc = SPINFER_EINVAL;
     if (tc) {
-        rc = N <= 16 ? launch_tc<16>(pl, st) : launch_tc<32>(pl, st);
-    } else switch (N) {
+        rc = Np <= 16 ? launch_tc<16>(pl, st) : launch_tc<32>(pl, st);
+    } else switch (Np) {
         case 8: rc = launch_nt<1>(pl, st); break;
         case 16: rc = launch_nt<2>(pl, st); break;
         case 24: rc = launch_nt<3>(pl, st); break;

@@ -151,11 +151,40 @@ def test_spmm_config2_sampled_rows(N):
     assert np.all(np.abs(f64(Y) - Yc) <= full_bound + 1e-6 * np.abs(Yc))
 
 
+@pytest.mark.parametrize("kernel", ["default", "mma", "tc"])
+@pytest.mark.parametrize("N", [1, 2, 3, 5, 7, 12, 20, 31])
+@pytest.mark.parametrize("M,K", [(256, 512), (320, 1472)])
+def test_spmm_any_N(M, K, N, kernel, monkeypatch):
+    """N not a multiple of 8: X is zero-padded to a multiple of 8 in the
+    workspace, only the N real columns of Y are written (odd row strides included)."""
+    if kernel != "default":
+        monkeypatch.setenv("SPINFER_KERNEL", kernel)
+    import torch
+    sp = _sp()
+    W = synth.weight(M, K, 0.5, seed=N)
+    X = synth.activation(K, N, seed=N + 1)
+    T = sp.encode(to_dev(W))
+    guard = torch.full((M * N + 64,), 0x7777, dtype=torch.int16, device="cuda")   # canary after Y
+    Y = guard[: M * N].view(M, N).view(torch.float16)
+    sp.spmm(T, to_dev(X), Y)
+    torch.cuda.synchronize()
+    assert bool((guard[M * N:] == 0x7777).all()), "write past Y"
+    Yref = oracle.spmm_f64(oracle.encode(W), X)
+    assert_within(f16_bits(Y), Yref, north_star_bound(W, X), f"{M}x{K}x{N} {kernel}")
+
+
+@pytest.mark.parametrize("N", [1, 5, 13])
+def test_spmm_any_N_integer_exact(N):
+    W, X, Y, Yref = run_case(384, 1024, N, 0.5, seed=300 + N, mode="int")
+    assert np.max(np.abs(Yref)) <= 2048
+    assert np.array_equal(Y, Yref.astype(np.float16).view(np.uint16))
+
+
 def test_spmm_errors():
     import torch
     sp = _sp()
     T = sp.encode(to_dev(synth.weight(128, 128, 0.5)))
-    X = torch.zeros((128, 12), dtype=torch.float16, device="cuda")
+    X = torch.zeros((128, 33), dtype=torch.float16, device="cuda")   # N > 32
     with pytest.raises(sp.SpinferError) as e:
         sp.spmm(T, X)
     assert e.value.status == -1
