@@ -94,6 +94,11 @@ constexpr int kMaxStages = 8;
 #ifndef SPINFER_PAGEPF
 #define SPINFER_PAGEPF 1
 #endif
+// bitmaps complete on their own mbarrier: the scan builds a stage's table while the stage's
+// values are still landing; consumers then wait for the table and for the values
+#ifndef SPINFER_BMBAR
+#define SPINFER_BMBAR 0
+#endif
 #ifndef SPINFER_EPREF
 #define SPINFER_EPREF 0
 #endif
@@ -150,11 +155,13 @@ __device__ __forceinline__ void trace_ev(const Params &prm, int p, int i, int w,
 }
 constexpr size_t kTraceBase2 = (size_t)kTraceCTAs * kTraceStages * kTraceW * kTraceEv;   // then [CTA][entry, exit] ns, [CTA] smid
 constexpr int kTraceMaxCTAs = 1024;
+#if SPINFER_INSTRUMENT == 1
 __device__ __forceinline__ unsigned long long globaltimer_ns() {
     unsigned long long t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
     return t;
 }
+#endif
 __device__ __forceinline__ void trace_k(const Params &prm, int p, int w, int ev) {
 #if SPINFER_INSTRUMENT == 1
     if (prm.trace && p < kTraceCTAs && w < kTraceW)
@@ -375,11 +382,13 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     const uint32_t bar_fix = sbase + 208;   // [split segment A/C][GT row]: partial parked (32 lanes)
     const uint32_t bar_epi = sbase + 256;   // [buffer][GT row]: the row's consumer warps parked their partials
     const uint32_t bar_epifree = sbase + 288;   // [buffer]: the fix-up warp has read the buffer
+    const uint32_t bar_bm = sbase + 320;    // [S]: the slot's bitmaps landed (SPINFER_BMBAR)
 
     if (lane == 0) trace_k(prm, p, warp, 0);
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
             mbar_init(bar_full + 8 * s, 1);       // the producer's arrive.expect_tx (+ TMA transaction bytes)
+            mbar_init(bar_bm + 8 * s, 1);
             mbar_init(bar_empty + 8 * s, kCW);
         }
         for (int s = 0; s < S; ++s) mbar_init(bar_scan + 8 * s, kScanWarps);   // one elected arrive per scan warp
@@ -449,10 +458,18 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             const uint32_t bmb = (uint32_t)sg.g * 512u;
             // X and bitmaps first (no offsets needed); the arrive comes with the value bytes last,
             // so the phase cannot complete before every transaction is registered
+#if SPINFER_BMBAR
+            mbar_arrive_expect_tx(bar_bm + 8 * slot, (uint32_t)sg.rows * bmb);
+            for (int r = 0; r < sg.rows; ++r)
+                bulk_g2s(st + prm.st_bm + (uint32_t)(r * G) * 512u,
+                         prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc) * 64, bmb, bar_bm + 8 * slot, pol_w);
+            mbar_expect_tx(fb, (uint32_t)G * xbytes);
+#else
             mbar_expect_tx(fb, (uint32_t)sg.rows * bmb + (uint32_t)G * xbytes);
             for (int r = 0; r < sg.rows; ++r)
                 bulk_g2s(st + prm.st_bm + (uint32_t)(r * G) * 512u,
                          prm.bm + ((size_t)(kR * sg.rb + r) * KG + sg.gc) * 64, bmb, fb, pol_w);
+#endif
             // X slab rows [64 gc, 64 (gc + G)) in one tensor TMA (box {N, 64 G}; rows past K are
             // zero-filled): L2-resident (every CTA reads X), default policy
             tma_2d_g2s(st, &prm.tmap_x, 0, 64 * sg.gc, fb);
@@ -636,7 +653,11 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
 #if SPINFER_SCANSPIN
             mbar_wait(bar_full + 8 * slot, it.par());
 #else
+#if SPINFER_BMBAR
+            mbar_wait_sleep(bar_bm + 8 * slot, it.par());   // the scan reads only the bitmaps
+#else
             mbar_wait_sleep(bar_full + 8 * slot, it.par());
+#endif
 #endif
             if (lane == 0) trace_ev(prm, p, i, warp, 1);
             uint2 ba[Q], bb[Q];
@@ -795,6 +816,9 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             mbar_wait(bar_scan + 8 * s.slot(), s.par());
 #else
             mbar_wait_sleep(bar_scan + 8 * s.slot(), s.par());   // implies full[slot] (see above)
+#endif
+#if SPINFER_BMBAR
+            mbar_wait_sleep(bar_full + 8 * s.slot(), s.par());   // values and X (usually landed already)
 #endif
             if (lane == 0) trace_ev(prm, p, si, warp, 1);
         }

@@ -1,3 +1,3 @@
-timeout 900 python -m pytest tests -m gpu -x -q --timeout 300 2>&1 | tail -4
-timeout 100 python bench.py --N 16 --steps 20 --warmup 3 --no-cpu-baseline --no-e2e --json-out gpurun_out/nn.json >/dev/null 2>&1; python -c "import json;d=json.load(open('gpurun_out/nn.json'));print('N16', round(d['us_per_spmm'],1), d['cublas_fp16']['us'])"
-for N in 1 4; do timeout 100 python bench.py --N $N --steps 20 --warmup 3 --no-cpu-baseline --no-e2e --json-out gpurun_out/nn.json >/dev/null 2>&1; python -c "import json;d=json.load(open('gpurun_out/nn.json'));print('N$N', round(d['us_per_spmm'],1), d['cublas_fp16']['us'])"; done
+timeout 600 python -m pytest tests/test_spmm_gpu.py -x -q --timeout 120 -k "not tc" 2>&1 | tail -2
+bash tools/ab.sh "nobmbar:libspinfer_nobmbar.so:" "bmbar:libspinfer_bmbar.so:"
+BENCH_ARGS="--N 8" bash tools/ab.sh "nobmbar8:libspinfer_nobmbar.so:" "bmbar8:libspinfer_bmbar.so:"
