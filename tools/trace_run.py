@@ -48,19 +48,19 @@ for p in range(2):
         epi = int(np.sum(a[:, 3] - a[:, 2]))
         gap = int(np.sum(a[1:, 0] - a[:-1, 3]))
         print(f"{w:4d} {rel(a[0,0]):6d} {wait:6d} {work:6d} {epi:7d} {gap:6d} {rel(k[w,3]):6d}")
-    for w in (16, 17):
+    for w in (17, 18):   # scan warps (warp 16 = fix-up, 19 = producer)
         a = tr[p, :nst, w, :]
         wait = int(np.sum(a[:, 1] - a[:, 0]))
         busy = int(np.sum(a[:, 3] - a[:, 1]))
         pre = int(np.sum(a[:, 2] - a[:, 1]))
         print(f"scan {w}: wait {wait} scan {busy} per-stage scan {busy / max(nst, 1):.0f} "
               f"(load+prefix {pre / max(nst, 1):.0f}, stores+publish {(busy - pre) / max(nst, 1):.0f})")
-    a = tr[p, :nst, 18, :]
+    a = tr[p, :nst, 19, :]
     print(f"producer: first issue {rel(a[0,1])}, wait-on-empty sum {int(np.sum(a[:,1]-a[:,0]))}")
-    print("stage  prod_issued  scan_full(16)  scan_done(16)  cons_wait_end(min..max over warps)  rel(max)")
+    print("stage  prod_issued  scan_full(17)  scan_done(17)  cons_wait_end(min..max over warps)  rel(max)")
     for i in range(0, nst, max(1, nst // 16)):
         c1 = tr[p, i, :NCW, 1]
-        print(f"{i:4d} {rel(tr[p,i,18,1]):10d} {rel(tr[p,i,16,1]):10d} {rel(tr[p,i,16,3]):10d} "
+        print(f"{i:4d} {rel(tr[p,i,19,1]):10d} {rel(tr[p,i,17,1]):10d} {rel(tr[p,i,17,3]):10d} "
               f"{rel(c1.min()):10d}..{rel(c1.max()):<10d} {rel(tr[p,i,:NCW,3].max()):10d}")
 
 # per-stage release latency (decode done -> slot released) of a few consumer warps: segment
