@@ -31,7 +31,22 @@ OPT = {
 }
 
 
+# Other model families of the paper's Fig. 10 (external: the public model configs):
+# gated MLPs (gate and up projections fused as one 2*ffn x h weight), grouped-query attention
+# (QKV = h + 2 * kv_heads * head_dim rows). Every M and K is a multiple of 64.
+GATED = {
+    "llama2-7b": {"h": 4096, "ffn": 11008, "kv": 4096},
+    "llama2-70b": {"h": 8192, "ffn": 28672, "kv": 2 * 8 * 128 // 2},
+    "llama3-8b": {"h": 4096, "ffn": 14336, "kv": 8 * 128},
+    "qwen2-7b": {"h": 3584, "ffn": 18944, "kv": 4 * 128},
+    "mixtral-8x7b-expert": {"h": 4096, "ffn": 14336, "kv": 8 * 128},
+}
+
+
 def layers(m):
+    if m in GATED:
+        h, f, kv = GATED[m]["h"], GATED[m]["ffn"], GATED[m]["kv"]
+        return {"QKV": (h + 2 * kv, h), "O": (h, h), "GateUp": (2 * f, h), "Down": (h, f)}
     h, f = OPT[m]["h"], OPT[m]["ffn"]
     return {"QKV": (3 * h, h), "O": (h, h), "FC1": (f, h), "FC2": (h, f)}
 
@@ -108,7 +123,7 @@ def main():
                     nbytes = sp.algorithmic_bytes(T, N)
                     us, usc = statistics.median(t), statistics.median(tc)
                     gbs = nbytes / (us * 1e-6) / 1e9
-                    rec = {"model": f"OPT-{m.upper()}", "layer": lname, "M": M, "K": K, "N": N, "sparsity": s,
+                    rec = {"model": f"OPT-{m.upper()}" if m in OPT else m, "layer": lname, "M": M, "K": K, "N": N, "sparsity": s,
                            "us_median": us, "us_mean": statistics.mean(t), "gbs": gbs,
                            "frac_measured_peak": gbs / peak if peak else None, "frac_8tbs": gbs / 8000.0,
                            "tflops_dense_equiv": 2 * M * K * N / (us * 1e-6) / 1e12,
