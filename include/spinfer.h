@@ -114,6 +114,18 @@ SPINFER_API size_t spinfer_spmm_workspace_bytes(int M, int K, int N);
 SPINFER_API int spinfer_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N,
                  void *workspace, size_t ws_bytes, void *stream);
 
+/* Y = act(W x X + bias) with the epilogue fused into the SpMM kernels (SURVEY §8(f) rank 4:
+ * the FC1 layers of the paper's OPT models run bias + ReLU after the SpMM).
+ * bias: device fp16 [M] (one value per output row) or NULL (no bias). act: SPINFER_ACT_NONE or
+ * SPINFER_ACT_RELU. The bias is added to the fp32 accumulator, the activation applied in fp32,
+ * then one RNE to fp16 per output. Everything else as spinfer_spmm (which is this call with
+ * bias = NULL, act = SPINFER_ACT_NONE). SPINFER_EINVAL for an unknown act or a bias not 2-byte
+ * aligned. */
+#define SPINFER_ACT_NONE 0
+#define SPINFER_ACT_RELU 1
+SPINFER_API int spinfer_spmm_ex(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N,
+                                const uint16_t *bias, int act, void *workspace, size_t ws_bytes, void *stream);
+
 /* Tensor-parallel row partition: rank `rank` of `world` owns rows
  * [*row_begin, *row_begin + *row_count) — contiguous, multiples of 64, sizes
  * differ by at most 64 (host only). */

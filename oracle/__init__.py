@@ -63,6 +63,7 @@ def _load():
     L.oracle_smbd_lane.restype = None
     L.oracle_smbd_tctile.argtypes = [_P(u64), _P(u16), ctypes.c_int, _P(ctypes.c_uint32)]
     L.oracle_smbd_tctile.restype = None
+    L.oracle_bias_act_f64.argtypes = [_P(dbl), ctypes.c_int, ctypes.c_int, _P(u16), ctypes.c_int]
     L.oracle_tp_rows.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int, _P(ctypes.c_int), _P(ctypes.c_int)]
     _lib = L
     return L
@@ -181,6 +182,19 @@ def spmm_f64(T: TCA, X: np.ndarray) -> np.ndarray:
     _check(_load().oracle_spmm_tca_f64(_ptr(T.gtile_offset, ctypes.c_int32), _ptr(T.bitmap, ctypes.c_uint64),
                                        _ptr(vals, ctypes.c_uint16), _ptr(X, ctypes.c_uint16), T.M, T.K, N,
                                        _ptr(Y, ctypes.c_double)), "oracle_spmm_tca_f64")
+    return Y
+
+
+def bias_act_f64(Y: np.ndarray, bias=None, act: str | None = None) -> np.ndarray:
+    """C7: the fused FC epilogue act(Y + bias) on an fp64 product (returns a new array)."""
+    Y = np.array(Y, dtype=np.float64, order="C", copy=True)
+    M, N = Y.shape
+    b = None if bias is None else np.ascontiguousarray(bias, dtype=np.uint16)
+    if b is not None and b.shape != (M,):
+        raise ValueError("bias must be fp16 bits [M]")
+    a = {None: 0, "none": 0, "relu": 1}[act]
+    _check(_load().oracle_bias_act_f64(_ptr(Y, ctypes.c_double), M, N,
+                                       _ptr(b, ctypes.c_uint16) if b is not None else None, a), "oracle_bias_act_f64")
     return Y
 
 

@@ -294,3 +294,19 @@ int oracle_tp_rows(int M, int world, int rank, int *row_begin, int *row_count) {
     *row_count = gn * O_GT;
     return O_OK;
 }
+
+/* ---- C7: fused FC epilogue (the OPT FC1 layers run bias + ReLU after the
+ * SpMM): Y[i][n] = act(Y[i][n] + bias[i]) in fp64, act 0 = identity, 1 = ReLU
+ * (max(v, 0)). bias may be NULL (no bias). Applied to the exact fp64 product of C3. */
+int oracle_bias_act_f64(double *Y, int M, int N, const uint16_t *bias, int act) {
+    if (!Y || M < 0 || N < 0 || (act != 0 && act != 1)) return O_EINVAL;
+    for (int i = 0; i < M; ++i) {
+        const double b = bias ? oracle_f16_to_f64(bias[i]) : 0.0;
+        for (int n = 0; n < N; ++n) {
+            double v = Y[(size_t)i * N + n] + b;
+            if (act == 1 && v < 0.0) v = 0.0;
+            Y[(size_t)i * N + n] = v;
+        }
+    }
+    return O_OK;
+}

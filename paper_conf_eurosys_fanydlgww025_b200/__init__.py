@@ -42,7 +42,7 @@ _lib = None
 
 # Exported symbols (must match include/spinfer.h; checked by tests/test_abi.py).
 SYMBOLS = ["spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spinfer_spmm_workspace_bytes",
-           "spinfer_spmm", "spinfer_tp_rows", "spinfer_spmm_tp", "spinfer_status_str", "spinfer_version"]
+           "spinfer_spmm", "spinfer_spmm_ex", "spinfer_tp_rows", "spinfer_spmm_tp", "spinfer_status_str", "spinfer_version"]
 
 
 def lib() -> ctypes.CDLL:
@@ -62,6 +62,7 @@ def lib() -> ctypes.CDLL:
     L.spinfer_spmm_workspace_bytes.argtypes = [i32, i32, i32]
     L.spinfer_spmm_workspace_bytes.restype = sz
     L.spinfer_spmm.argtypes = [P(_Tca), vp, vp, i32, i32, i32, vp, sz, vp]
+    L.spinfer_spmm_ex.argtypes = [P(_Tca), vp, vp, i32, i32, i32, vp, i32, vp, sz, vp]
     L.spinfer_tp_rows.argtypes = [i32, i32, i32, P(ctypes.c_int), P(ctypes.c_int)]
     L.spinfer_spmm_tp.argtypes = [P(_Tca), vp, vp, i32, i32, i32, i32, i32, vp, sz, vp]
     L.spinfer_status_str.argtypes = [i32]
@@ -196,9 +197,13 @@ def workspace(M: int, K: int, N: int, device=None) -> torch.Tensor:
     return ws
 
 
+ACT_NONE, ACT_RELU = 0, 1   # spinfer.h SPINFER_ACT_*
+
+
 def spmm(T: TCA, X: torch.Tensor, Y: torch.Tensor | None = None, ws: torch.Tensor | None = None,
-         stream=None) -> torch.Tensor:
-    """Y = W X: X fp16 [K][N] (CUDA), 1 <= N <= 32; returns fp16 [M][N]."""
+         stream=None, bias: torch.Tensor | None = None, act: str | None = None) -> torch.Tensor:
+    """Y = act(W X + bias): X fp16 [K][N] (CUDA), 1 <= N <= 32; bias fp16 [M] or
+    None; act None or "relu" (fused into the SpMM epilogue, spinfer_spmm_ex); returns fp16 [M][N]."""
     X = _dev_u16(X, "X")
     K, N = X.shape
     if K != T.K:
@@ -208,10 +213,21 @@ def spmm(T: TCA, X: torch.Tensor, Y: torch.Tensor | None = None, ws: torch.Tenso
     Yv = _dev_u16(Y, "Y")
     if ws is None:
         ws = workspace(T.M, T.K, N, X.device)
+    actc = {None: ACT_NONE, "none": ACT_NONE, "relu": ACT_RELU}[act]
+    bptr = None
+    if bias is not None:
+        bv = _dev_u16(bias, "bias")
+        if bv.numel() != T.M:
+            raise ValueError(f"bias has {bv.numel()} entries, W has M={T.M}")
+        bptr = bv.data_ptr()
     cs = T.c_struct()
     with torch.cuda.device(X.device):
-        _check(lib().spinfer_spmm(ctypes.byref(cs), X.data_ptr(), Yv.data_ptr(), T.M, T.K, N, ws.data_ptr(),
-                                  ws.numel(), _stream(stream)), "spinfer_spmm")
+        if bptr is None and actc == ACT_NONE:
+            _check(lib().spinfer_spmm(ctypes.byref(cs), X.data_ptr(), Yv.data_ptr(), T.M, T.K, N, ws.data_ptr(),
+                                      ws.numel(), _stream(stream)), "spinfer_spmm")
+        else:
+            _check(lib().spinfer_spmm_ex(ctypes.byref(cs), X.data_ptr(), Yv.data_ptr(), T.M, T.K, N, bptr, actc,
+                                         ws.data_ptr(), ws.numel(), _stream(stream)), "spinfer_spmm_ex")
     return Y
 
 

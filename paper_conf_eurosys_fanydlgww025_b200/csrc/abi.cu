@@ -82,14 +82,21 @@ size_t spinfer_spmm_workspace_bytes(int M, int K, int N) {
     return spmm_workspace_bytes(M, K, N);
 }
 
-int spinfer_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *workspace,
-                 size_t ws_bytes, void *stream) {
+int spinfer_spmm_ex(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N,
+                    const uint16_t *bias, int act, void *workspace, size_t ws_bytes, void *stream) {
     if (!X || !Y || N < 1 || N > 32) return SPINFER_EINVAL;
+    if (act != SPINFER_ACT_NONE && act != SPINFER_ACT_RELU) return SPINFER_EINVAL;
+    if (bias && (reinterpret_cast<uintptr_t>(bias) & 1u)) return SPINFER_EINVAL;
     if (!aligned16(X) || !aligned16(Y) || (workspace && !aligned16(workspace))) return SPINFER_EINVAL;
     int rc = validate_tca(T, M, K);
     if (rc) return rc;
     if ((rc = check_device())) return rc;
-    return launch_spmm(T, X, Y, M, K, N, workspace, ws_bytes, reinterpret_cast<cudaStream_t>(stream));
+    return launch_spmm(T, X, Y, M, K, N, bias, act, workspace, ws_bytes, reinterpret_cast<cudaStream_t>(stream));
+}
+
+int spinfer_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *workspace,
+                 size_t ws_bytes, void *stream) {
+    return spinfer_spmm_ex(T, X, Y, M, K, N, nullptr, SPINFER_ACT_NONE, workspace, ws_bytes, stream);
 }
 
 int spinfer_tp_rows(int M, int world, int rank, int *row_begin, int *row_count) {

@@ -21,7 +21,7 @@ int launch_decode(const spinfer_tca *T, uint16_t *W_out, cudaStream_t st);
 
 // spmm.cu
 size_t spmm_workspace_bytes(int M, int K, int N);
-int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *ws,
+int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias, int act, void *ws,
                 size_t ws_bytes, cudaStream_t st);
 
 }  // namespace spinfer

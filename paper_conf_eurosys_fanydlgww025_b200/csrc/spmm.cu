@@ -122,6 +122,8 @@ struct Params {
     const uint16_t *X;
     uint16_t *Y;
     float *ws_part;
+    const uint16_t *bias;   // fused epilogue (spinfer_spmm_ex): fp16 [M] or null
+    int act;                // SPINFER_ACT_NONE / SPINFER_ACT_RELU
     float *ws_epi;      // [P][2 buffers][kR][8 warps][64 x N] fp32 partials of the asynchronous epilogue
     int32_t *ws_cnt;
     int KG, MG;
@@ -305,13 +307,34 @@ constexpr uint32_t kSelA = 0x7f62u, kSelB = 0x4cbfu, kSelC = 0x2333u;
 
 // N = the caller's column count (row stride of Y); the kernel computes NT * 8 >= N columns
 // (X zero-padded to a multiple of 8) and drops the padding columns here.
-template <int NT>
-__device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const float (&acc)[4][NT][4], int lane) {
+// Fused epilogue of one output (spinfer_spmm_ex): + bias[row] and the activation, in fp32.
+__device__ __forceinline__ float epi_act(float v, float b, int act) {
+    v += b;
+    return act == SPINFER_ACT_RELU ? fmaxf(v, 0.f) : v;
+}
+
+// prm.N = the caller's column count (row stride of Y); the kernel computes NT * 8 >= N columns
+// (X zero-padded to a multiple of 8) and drops the padding columns here.
+template <int NT, bool EPI>
+__device__ __forceinline__ void store_y(const Params &prm, int row_base, float (&acc)[4][NT][4], int lane) {
+    uint16_t *const Y = prm.Y;
+    const int N = prm.N;
 #pragma unroll
-    for (int tr = 0; tr < 4; ++tr)
+    for (int tr = 0; tr < 4; ++tr) {
+        const int r0 = row_base + tr * 16 + (lane >> 2);
+        if (EPI) {   // fused epilogue: a separate kernel instantiation, so the plain path pays nothing
+            const float b0 = prm.bias ? __half2float(__ushort_as_half(prm.bias[r0])) : 0.f;
+            const float b1 = prm.bias ? __half2float(__ushort_as_half(prm.bias[r0 + 8])) : 0.f;
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) {
+                acc[tr][nt][0] = epi_act(acc[tr][nt][0], b0, prm.act);
+                acc[tr][nt][1] = epi_act(acc[tr][nt][1], b0, prm.act);
+                acc[tr][nt][2] = epi_act(acc[tr][nt][2], b1, prm.act);
+                acc[tr][nt][3] = epi_act(acc[tr][nt][3], b1, prm.act);
+            }
+        }
 #pragma unroll
         for (int nt = 0; nt < NT; ++nt) {
-            int r0 = row_base + tr * 16 + (lane >> 2);
             int col = nt * 8 + 2 * (lane & 3);
             __half2 lo = __floats2half2_rn(acc[tr][nt][0], acc[tr][nt][1]);   // one RNE per output (A11)
             __half2 hi = __floats2half2_rn(acc[tr][nt][2], acc[tr][nt][3]);
@@ -325,11 +348,12 @@ __device__ __forceinline__ void store_y(uint16_t *Y, int N, int row_base, const 
                 if (col + 1 < N) { y0[col + 1] = __high2half(lo); y1[col + 1] = __high2half(hi); }
             }
         }
+    }
 }
 
 // Last contributor of a split rowblock: sum every contributor's fp32 partial in CTA order
 // (deterministic; its own partial included), write Y, re-zero the counter.
-template <int NT>
+template <int NT, bool EPI>
 __device__ __forceinline__ void fixup_sum(const Params &prm, int rb, int r, int pf, int pl, int lane) {
     constexpr int N = NT * 8;
     __threadfence();
@@ -352,11 +376,11 @@ __device__ __forceinline__ void fixup_sum(const Params &prm, int rb, int r, int 
             }
     }
     const int grow = kR * rb + r;
-    store_y<NT>(prm.Y, prm.N, grow * 64, acc, lane);
+    store_y<NT, EPI>(prm, grow * 64, acc, lane);
     if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed
 }
 
-template <int NT>
+template <int NT, bool EPI>
 __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_constant__ Params prm) {
     constexpr int N = NT * 8;
     constexpr int KQ = Cfg<NT>::KQ, kCW = Cfg<NT>::CW;
@@ -517,7 +541,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                     int old = 0;
                     if (lane == 0) old = atomicAdd(prm.ws_cnt + kR * rb + r, 1);
                     old = __shfl_sync(0xffffffffu, old, 0);
-                    if (old == pl - pf) fixup_sum<NT>(prm, rb, r, pf, pl, lane);   // last contributor
+                    if (old == pl - pf) fixup_sum<NT, EPI>(prm, rb, r, pf, pl, lane);   // last contributor
                 };
                 if (last) {
                     if (!complete)
@@ -555,7 +579,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                         }
                     const int grow = kR * rb + r;
                     if (complete) {
-                        store_y<NT>(prm.Y, prm.N, grow * 64, acc, lane);
+                        store_y<NT, EPI>(prm, grow * 64, acc, lane);
                     } else {
                         float4 *part = reinterpret_cast<float4 *>(prm.ws_part) + (((size_t)p * 2 + myslot) * kR + r) * (64 * N / 4);
 #pragma unroll
@@ -602,7 +626,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                 int old = 0;
                 if (lane == 0) old = atomicAdd(prm.ws_cnt + kR * rb + r, 1);
                 old = __shfl_sync(0xffffffffu, old, 0);
-                if (old == pl - pf) fixup_sum<NT>(prm, rb, r, pf, pl, lane);   // last contributor
+                if (old == pl - pf) fixup_sum<NT, EPI>(prm, rb, r, pf, pl, lane);   // last contributor
             }
         }
         return;
@@ -972,7 +996,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                 const int grow = kR * rb + r;
                 const int row_base = grow * 64;
                 if (e.complete()) {
-                    store_y<NT>(prm.Y, prm.N, row_base, acc, lane);
+                    store_y<NT, EPI>(prm, row_base, acc, lane);
                 } else {
                     // split rowblock (split-K fix-up, the paper's ReductionWorkspace P:231): park the
                     // fp32 partial; the fix-up warp counts it and the last contributor sums all
@@ -1073,7 +1097,14 @@ struct SegFlags {
 };
 
 template <int NB>
-__device__ __forceinline__ void store_y_row(uint16_t *Y, size_t grow, int N, const float (&v)[NB]) {
+__device__ __forceinline__ void store_y_row(const Params &prm, size_t grow, float (&v)[NB]) {
+    uint16_t *const Y = prm.Y;
+    const int N = prm.N;
+    if (prm.bias || prm.act) {   // fused epilogue (spinfer_spmm_ex)
+        const float b = prm.bias ? __half2float(__ushort_as_half(prm.bias[grow])) : 0.f;
+#pragma unroll
+        for (int j = 0; j < NB; ++j) v[j] = epi_act(v[j], b, prm.act);
+    }
     if (N % 8) {   // N not a multiple of 8 (X was zero-padded): rows are not 16-byte aligned
         __half *y = reinterpret_cast<__half *>(Y + grow * (size_t)N);
 #pragma unroll
@@ -1199,7 +1230,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
                             v[4 * c4] += x.x; v[4 * c4 + 1] += x.y; v[4 * c4 + 2] += x.z; v[4 * c4 + 3] += x.w;
                         }
                 }
-                store_y_row<NB>(prm.Y, (size_t)rb * 128 + (size_t)row_in, N, v);
+                store_y_row<NB>(prm, (size_t)rb * 128 + (size_t)row_in, v);
             }
             if (lane == 0) prm.ws_cnt[rb] = 0;   // leave the workspace zeroed
         };
@@ -1382,7 +1413,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         if (lane == 0) mbar_arrive(bar_de + 8u * db);
         const bool valid = row_in < 64 * rows;
         if (complete) {
-            if (valid) store_y_row<NB>(prm.Y, (size_t)rb * 128 + (size_t)row_in, N, v);
+            if (valid) store_y_row<NB>(prm, (size_t)rb * 128 + (size_t)row_in, v);
             return;
         }
         // split rowblock: park this CTA's fp32 partial; the producer warp does the fix-up
@@ -1422,7 +1453,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
                         v[4 * c4] += x.x; v[4 * c4 + 1] += x.y; v[4 * c4 + 2] += x.z; v[4 * c4 + 3] += x.w;
                     }
             }
-            store_y_row<NB>(prm.Y, (size_t)rb * 128 + (size_t)row_in, N, v);
+            store_y_row<NB>(prm, (size_t)rb * 128 + (size_t)row_in, v);
         }
         if (lane == 0) prm.ws_cnt[4 * rb + q] = 0;   // leave the workspace zeroed
 #else
@@ -1702,18 +1733,18 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl, bool tc) {
     return false;
 }
 
-template <int NT>
+template <int NT, bool EPI>
 int launch_nt(const Plan &pl, cudaStream_t st) {
     static int configured_smem[64] = {0};   // per device: max dynamic smem already set for this instantiation
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev < 0 || dev >= 64) dev = 0;
     if ((int)pl.smem > configured_smem[dev]) {
-        if (cudaFuncSetAttribute(k_spmm<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem) != cudaSuccess)
+        if (cudaFuncSetAttribute(k_spmm<NT, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem) != cudaSuccess)
             return SPINFER_ECUDA;
         configured_smem[dev] = (int)pl.smem;
     }
-    k_spmm<NT><<<pl.P, Cfg<NT>::Threads, pl.smem, st>>>(pl.prm);
+    k_spmm<NT, EPI><<<pl.P, Cfg<NT>::Threads, pl.smem, st>>>(pl.prm);
     return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
 }
 
@@ -1746,8 +1777,8 @@ size_t spmm_workspace_bytes(int M, int K, int N) {
     return kCounterBytes + part + epi + xpad;
 }
 
-int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, void *ws, size_t ws_bytes,
-                cudaStream_t st) {
+int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias, int act,
+                void *ws, size_t ws_bytes, cudaStream_t st) {
     Plan pl;
     // Kernel choice by N, from the B200 measurements: the mma.sync kernel for
     // N <= 16, the tcgen05 kernel (accumulators in TMEM) for N >= 24, where mma.sync needs twice
@@ -1783,6 +1814,9 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     q.vals = T->values;
     q.X = Xk;
     q.Y = Y;
+    q.bias = bias;
+    q.act = act;
+    const bool epi = bias != nullptr || act != SPINFER_ACT_NONE;
     q.ws_cnt = reinterpret_cast<int32_t *>(ws);
     q.ws_part = reinterpret_cast<float *>(reinterpret_cast<uint8_t *>(ws) + kCounterBytes);
     q.ws_epi = q.ws_part + (size_t)pl.P * 2 * kR * 64 * Np;
@@ -1802,10 +1836,10 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     if (tc) {
         rc = Np <= 16 ? launch_tc<16>(pl, st) : launch_tc<32>(pl, st);
     } else switch (Np) {
-        case 8: rc = launch_nt<1>(pl, st); break;
-        case 16: rc = launch_nt<2>(pl, st); break;
-        case 24: rc = launch_nt<3>(pl, st); break;
-        case 32: rc = launch_nt<4>(pl, st); break;
+        case 8: rc = epi ? launch_nt<1, true>(pl, st) : launch_nt<1, false>(pl, st); break;
+        case 16: rc = epi ? launch_nt<2, true>(pl, st) : launch_nt<2, false>(pl, st); break;
+        case 24: rc = epi ? launch_nt<3, true>(pl, st) : launch_nt<3, false>(pl, st); break;
+        case 32: rc = epi ? launch_nt<4, true>(pl, st) : launch_nt<4, false>(pl, st); break;
         default: break;
     }
     if (trace_path && rc == SPINFER_OK) {   // debug only: synchronous dump of the stage timeline

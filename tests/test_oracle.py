@@ -320,3 +320,27 @@ def test_shard_is_slice_of_encoding():
             assert np.array_equal(S.gtile_offset, E.gtile_offset)
             assert np.array_equal(S.bitmap, E.bitmap)
             assert np.array_equal(S.values, E.values)
+
+
+def test_bias_act_worked_example():
+    """C7 fused FC epilogue, values worked by hand: act(Y + b) with b = (1.0, -0.5)."""
+    Y = np.array([[-1.5, 2.0], [0.25, -0.25]])
+    b = np.array([0x3C00, 0xB800], dtype=np.uint16)             # fp16 1.0, -0.5
+    assert np.array_equal(oracle.bias_act_f64(Y, b, None), [[-0.5, 3.0], [-0.25, -0.75]])
+    assert np.array_equal(oracle.bias_act_f64(Y, b, "relu"), [[0.0, 3.0], [0.0, 0.0]])
+    assert np.array_equal(oracle.bias_act_f64(Y, None, "relu"), [[0.0, 2.0], [0.25, 0.0]])
+    assert np.array_equal(oracle.bias_act_f64(Y), Y)
+
+
+def test_bias_act_identity_weight():
+    """W = I: the SpMM returns X exactly, so the fused epilogue must give max(X + b, 0) with the
+    hand-checkable fp16 inputs below (X row i = (i - 2, 2 - i) halves, b_i = -0.5 i)."""
+    M = 64
+    W = np.zeros((M, M), dtype=np.uint16)
+    W[np.arange(M), np.arange(M)] = 0x3C00
+    X = np.array([[oracle.f64_to_f16(i - 2.0), oracle.f64_to_f16(2.0 - i)] for i in range(M)], dtype=np.uint16)
+    b = np.array([oracle.f64_to_f16(-0.5 * i) for i in range(M)], dtype=np.uint16)
+    Y = oracle.bias_act_f64(oracle.spmm_f64(oracle.encode(W), X), b, "relu")
+    i = np.arange(M, dtype=np.float64)
+    exp = np.stack([np.maximum(i - 2.0 - 0.5 * i, 0.0), np.maximum(2.0 - i - 0.5 * i, 0.0)], axis=1)
+    assert np.array_equal(Y, exp)

@@ -180,6 +180,46 @@ def test_spmm_any_N_integer_exact(N):
     assert np.array_equal(Y, Yref.astype(np.float16).view(np.uint16))
 
 
+@pytest.mark.parametrize("kernel", ["mma", "tc"])
+@pytest.mark.parametrize("act", [None, "relu"])
+@pytest.mark.parametrize("N", [5, 16, 32])
+def test_spmm_bias_act(N, act, kernel, monkeypatch):
+    """spinfer_spmm_ex: act(W X + bias) fused into the epilogue, on complete rowblocks and (4 CTAs
+    on a long K) split rowblocks finished by the split-K fix-up; vs the oracle's C7 epilogue."""
+    monkeypatch.setenv("SPINFER_KERNEL", kernel)
+    monkeypatch.setenv("SPINFER_MAX_CTAS", "4")
+    import torch
+    sp = _sp()
+    M, K = 384, 2048
+    W = synth.weight(M, K, 0.5, seed=N + 11)
+    X = synth.activation(K, N, seed=N + 12)
+    bias = synth.activation(M, 1, seed=N + 13).reshape(M)
+    T = sp.encode(to_dev(W))
+    Y = sp.spmm(T, to_dev(X), bias=to_dev(bias).view(torch.float16), act=act)
+    torch.cuda.synchronize()
+    Yref = oracle.bias_act_f64(oracle.spmm_f64(oracle.encode(W), X), bias, act)
+    assert_within(f16_bits(Y), Yref, north_star_bound(W, X), f"bias act={act} N={N} {kernel}")
+    if act == "relu":
+        assert (f16_bits(Y) & 0x8000).sum() == 0 or np.all(f64(f16_bits(Y)) >= 0)
+
+
+@pytest.mark.parametrize("kernel", ["mma", "tc"])
+def test_spmm_bias_relu_integer_exact(kernel, monkeypatch):
+    monkeypatch.setenv("SPINFER_KERNEL", kernel)
+    monkeypatch.setenv("SPINFER_MAX_CTAS", "4")
+    import torch
+    sp = _sp()
+    M, K, N = 384, 2048, 16
+    W = synth.weight(M, K, 0.5, seed=5, mode="int")
+    X = synth.activation(K, N, seed=6, mode="int")
+    bias = np.array([oracle.f64_to_f16(float((i % 9) - 4)) for i in range(M)], dtype=np.uint16)
+    Y = sp.spmm(sp.encode(to_dev(W)), to_dev(X), bias=to_dev(bias).view(torch.float16), act="relu")
+    torch.cuda.synchronize()
+    Yref = oracle.bias_act_f64(oracle.spmm_f64(oracle.encode(W), X), bias, "relu")
+    assert np.abs(Yref).max() <= 2048
+    assert np.array_equal(f16_bits(Y), Yref.astype(np.float16).view(np.uint16))
+
+
 def test_spmm_errors():
     import torch
     sp = _sp()
@@ -196,3 +236,9 @@ def test_spmm_errors():
     with pytest.raises(sp.SpinferError) as e:
         sp.spmm(T, Xbig[1:1 + 128 * 16].view(128, 16))   # misaligned by 2 bytes
     assert e.value.status == -1
+    cs = T.c_struct()
+    import ctypes
+    ws = sp.workspace(128, 128, 16)
+    rc = sp.lib().spinfer_spmm_ex(ctypes.byref(cs), X.data_ptr(), X.data_ptr(), 128, 128, 16, None, 7,
+                                  ws.data_ptr(), ws.numel(), None)
+    assert rc == -1                                     # unknown activation

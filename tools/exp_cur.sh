@@ -1,1 +1,2 @@
-timeout 900 python tools/sweep.py --models llama2-7b,llama2-70b,llama3-8b,qwen2-7b,mixtral-8x7b-expert --s 0.5,0.7 --N 1,8,16,32 --out gpurun_out/r1e_sweep_more.jsonl > gpurun_out/sweep_more.log 2>&1; grep -A60 "^model" gpurun_out/sweep_more.log
+timeout 900 python -m pytest tests/test_spmm_gpu.py -x -q --timeout 300 2>&1 | tail -2
+bash tools/ab.sh "noepi:libspinfer_noepi.so:" "epi2:libspinfer_epi2.so:"
