@@ -47,6 +47,8 @@ class Layer:
     row_count: int
     shard: object = None          # TCA (GPU) or any object spmm_fn understands
     x_rows: Optional[int] = None  # consume only the first x_rows rows of the previous output (stand-in attention)
+    act: Optional[str] = None     # fused epilogue activation ("relu" for the OPT FC1 layers), spinfer_spmm_ex
+    bias: object = None           # this rank's bias rows (fp16 [row_count]) or None
 
 
 def gather_rows(Y_full: torch.Tensor, M: int, world: int, rank: int, group=None) -> torch.Tensor:
@@ -76,7 +78,13 @@ def gather_rows(Y_full: torch.Tensor, M: int, world: int, rank: int, group=None)
 
 def gpu_spmm_fn(layer: Layer, X: torch.Tensor, Y_full: torch.Tensor, world: int, rank: int):
     import paper_conf_eurosys_fanydlgww025_b200 as sp
-    sp.spmm_tp(layer.shard, X, Y_full, layer.M, world, rank)
+    if layer.act is None and layer.bias is None:
+        sp.spmm_tp(layer.shard, X, Y_full, layer.M, world, rank)
+    else:
+        # the rank's rows of Y_full are one contiguous [row_count][N] block: the fused-epilogue
+        # SpMM writes straight into it (what spinfer_spmm_tp does for the plain SpMM)
+        b, c = tp_rows(layer.M, world, rank)
+        sp.spmm(layer.shard, X, Y_full[b:b + c], bias=layer.bias, act=layer.act)
 
 
 def run_stack(layers: Sequence[Layer], X: torch.Tensor, world: int, rank: int, group=None,
@@ -112,12 +120,13 @@ def opt_layer_shapes(model: str):
     return [("qkv", 3 * h, h), ("o", h, h), ("fc1", f, h), ("fc2", h, f)]
 
 
-def opt_stack_layers(model: str, world: int, rank: int) -> List[Layer]:
+def opt_stack_layers(model: str, world: int, rank: int, relu: bool = False) -> List[Layer]:
     """Config 5 stack: QKV -> O (consumes the Q block = first h rows of QKV's output,
-    the stand-in for attention) -> FC1 -> FC2 (no activation)."""
+    the stand-in for attention) -> FC1 (-> ReLU, fused, when relu=True) -> FC2."""
     h, _ = OPT[model]
     out = []
     for name, M, K in opt_layer_shapes(model):
         b, c = tp_rows(M, world, rank)
-        out.append(Layer(name, M, K, b, c, x_rows=h if name == "o" else None))
+        out.append(Layer(name, M, K, b, c, x_rows=h if name == "o" else None,
+                         act="relu" if (relu and name == "fc1") else None))
     return out
