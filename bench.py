@@ -124,14 +124,19 @@ class ClockSampler:
                 for name, bit in self.REASONS.items():
                     if r & bit:
                         self.reasons.add(name)
-                time.sleep(0.001)
+                time.sleep(0.0005)
         except Exception as e:  # pragma: no cover - NVML missing
             self.reasons.add(f"nvml unavailable: {type(e).__name__}")
 
     def __enter__(self):
         self._t = threading.Thread(target=self._run, daemon=True)
         self._t.start()
-        time.sleep(0.02)
+        # NVML initialisation can outlast a short timed region: wait for the first sample, then
+        # count only the samples taken from here on (the region itself)
+        t0 = time.time()
+        while not self.sm and not self.reasons and time.time() - t0 < 5.0:
+            time.sleep(0.001)
+        self._mark = len(self.sm)
         return self
 
     def __exit__(self, *exc):
@@ -140,8 +145,9 @@ class ClockSampler:
             self._t.join(timeout=10)
 
     def summary(self):
-        return {"sm_mhz": statistics.median(self.sm) if self.sm else None, "sm_max_mhz": self.max_sm,
-                "reasons": sorted(self.reasons), "samples": len(self.sm)}
+        sm = self.sm[getattr(self, "_mark", 0):]
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": self.max_sm,
+                "reasons": sorted(self.reasons), "samples": len(sm)}
 
 
 # ----------------------------------------------------------------------------- reference arm
