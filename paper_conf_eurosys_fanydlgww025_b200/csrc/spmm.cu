@@ -99,6 +99,12 @@ constexpr int kMaxStages = 8;
 #ifndef SPINFER_BMBAR
 #define SPINFER_BMBAR 0
 #endif
+// slot release: the consumer warps count themselves on a shared counter and only the last one
+// arrives on the slot's empty mbarrier (1 barrier event per stage instead of 16: every mbarrier
+// event wakes every suspended waiter of the CTA)
+#ifndef SPINFER_RELCNT
+#define SPINFER_RELCNT 0
+#endif
 #ifndef SPINFER_EPREF
 #define SPINFER_EPREF 0
 #endif
@@ -407,13 +413,15 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     const uint32_t bar_epi = sbase + 256;   // [buffer][GT row]: the row's consumer warps parked their partials
     const uint32_t bar_epifree = sbase + 288;   // [buffer]: the fix-up warp has read the buffer
     const uint32_t bar_bm = sbase + 320;    // [S]: the slot's bitmaps landed (SPINFER_BMBAR)
+    const uint32_t rel_cnt = sbase + 384;   // [S] u32: consumer warps done with the slot (SPINFER_RELCNT)
 
     if (lane == 0) trace_k(prm, p, warp, 0);
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
             mbar_init(bar_full + 8 * s, 1);       // the producer's arrive.expect_tx (+ TMA transaction bytes)
             mbar_init(bar_bm + 8 * s, 1);
-            mbar_init(bar_empty + 8 * s, kCW);
+            mbar_init(bar_empty + 8 * s, SPINFER_RELCNT ? 1 : kCW);
+            reinterpret_cast<uint32_t *>(smem + 384)[s] = 0u;
         }
         for (int s = 0; s < S; ++s) mbar_init(bar_scan + 8 * s, kScanWarps);   // one elected arrive per scan warp
         for (int k = 0; k < 2 * kR; ++k) mbar_init(bar_fix + 8 * k, 32);
@@ -1018,7 +1026,14 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
         }
         __syncwarp();
         if (lane == 0 && !reuse0) {
+#if SPINFER_RELCNT
+            // acq_rel: this warp's reads of the slot happen-before the count; the last warp's
+            // acquire makes all of them happen-before its arrive (release) and the refill
+            const uint32_t old = atom_add_acqrel_shared(rel_cnt + 4u * (uint32_t)e.slot(), 1u);
+            if (old % (uint32_t)kCW == (uint32_t)kCW - 1u) mbar_arrive(bar_empty + 8 * e.slot());
+#else
             mbar_arrive(bar_empty + 8 * e.slot());   // frees the ring slot and its table
+#endif
             trace_ev(prm, p, i, cw, 3);
         }
     }

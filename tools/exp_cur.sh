@@ -1,1 +1,2 @@
-for i in 1 2; do timeout 300 python bench.py > gpurun_out/b$i.jsonl 2>/dev/null; python -c "import json; d=json.loads(open('gpurun_out/b$i.jsonl').readline()); print(d['us_per_spmm'], d['clocks'])"; done
+SPINFER_LIB=$PWD/paper_conf_eurosys_fanydlgww025_b200/libspinfer_relcnt.so timeout 900 python -m pytest tests/test_spmm_gpu.py -x -q --timeout 300 2>&1 | tail -2
+bash tools/ab.sh "norelcnt:libspinfer_norelcnt.so:" "relcnt:libspinfer_relcnt.so:"
