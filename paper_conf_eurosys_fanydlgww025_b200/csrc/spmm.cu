@@ -413,7 +413,9 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
     const uint32_t bar_epi = sbase + 256;   // [buffer][GT row]: the row's consumer warps parked their partials
     const uint32_t bar_epifree = sbase + 288;   // [buffer]: the fix-up warp has read the buffer
     const uint32_t bar_bm = sbase + 320;    // [S]: the slot's bitmaps landed (SPINFER_BMBAR)
+#if SPINFER_RELCNT
     const uint32_t rel_cnt = sbase + 384;   // [S] u32: consumer warps done with the slot (SPINFER_RELCNT)
+#endif
 
     if (lane == 0) trace_k(prm, p, warp, 0);
     if (threadIdx.x == 0) {
