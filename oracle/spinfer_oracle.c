@@ -69,8 +69,11 @@ static int nonzero16(uint16_t bits) { return (bits & 0x7FFF) != 0; }   /* readin
 
 /* ---- sizes, eq. (9) ---- */
 
-int64_t oracle_ngt(int M, int K) { return (int64_t)(M / O_GT) * (K / O_GT); }      /* NGT */
-int64_t oracle_nbt(int M, int K) { return (int64_t)(M / O_BT) * (K / O_BT); }      /* NBT */
+/* Reading A8: a shape that is not a multiple of the GT is zero-padded to the next multiple of 64
+ * in both dimensions (elements outside M x K are zeros: no bit set, no value stored). */
+static int cdiv(int a, int b) { return (a + b - 1) / b; }
+int64_t oracle_ngt(int M, int K) { return (int64_t)cdiv(M, O_GT) * cdiv(K, O_GT); }   /* NGT */
+int64_t oracle_nbt(int M, int K) { return oracle_ngt(M, K) * 64; }                      /* NBT */
 
 /* Stor_TCA-BME = 4B(NGT+1) + 8B*NBT + 2B*NNZ, eq. (9) P:210. Pass n_values
  * (padded count) to get the buffer size actually allocated, nnz for eq. (9). */
@@ -84,7 +87,12 @@ double oracle_compression_ratio(int M, int K, int64_t n_values) {
 }
 
 static int valid_shape(int M, int K) {
-    return M > 0 && K > 0 && (M % O_GT) == 0 && (K % O_GT) == 0;   /* reading A8 */
+    return M > 0 && K > 0;   /* any shape, zero-padded to whole GroupTiles (reading A8) */
+}
+
+/* W[r][c] of the zero-padded matrix (reading A8) */
+static uint16_t w_at(const uint16_t *W, int M, int K, int r, int c) {
+    return (r < M && c < K) ? W[(size_t)r * K + c] : (uint16_t)0;
 }
 
 /* Element (r, c) of BT number `bt` (0..3, column-major in the TT) of
@@ -102,14 +110,14 @@ static void bt_elem(int gr, int gc, int tt, int bt, int b, int *r, int *c) {
 int oracle_encode_count(const uint16_t *W, int M, int K, int64_t *nnz, int64_t *n_values, int32_t *max_gt_values) {
     if (!W || !valid_shape(M, K)) return O_EINVAL;
     int64_t running = 0, z = 0; int32_t mx = 0;
-    for (int gr = 0; gr < M / O_GT; ++gr)
-        for (int gc = 0; gc < K / O_GT; ++gc) {           /* GTs row-major */
+    for (int gr = 0; gr < cdiv(M, O_GT); ++gr)
+        for (int gc = 0; gc < cdiv(K, O_GT); ++gc) {      /* GTs row-major */
             int64_t start = running;
             for (int tt = 0; tt < 16; ++tt)
                 for (int bt = 0; bt < 4; ++bt)
                     for (int b = 0; b < 64; ++b) {
                         int r, c; bt_elem(gr, gc, tt, bt, b, &r, &c);
-                        if (nonzero16(W[(size_t)r * K + c])) { ++running; ++z; }
+                        if (nonzero16(w_at(W, M, K, r, c))) { ++running; ++z; }
                     }
             while (running % 8 != 0) ++running;           /* 16-B padding (reading A6) */
             if (running - start > mx) mx = (int32_t)(running - start);
@@ -125,8 +133,8 @@ int oracle_encode_count(const uint16_t *W, int M, int K, int64_t *nnz, int64_t *
 int oracle_encode(const uint16_t *W, int M, int K, int32_t *gtile_offset, uint64_t *bitmap, uint16_t *values) {
     if (!W || !gtile_offset || !bitmap || !valid_shape(M, K)) return O_EINVAL;
     int64_t running = 0;
-    int KG = K / O_GT;
-    for (int gr = 0; gr < M / O_GT; ++gr)
+    int KG = cdiv(K, O_GT);
+    for (int gr = 0; gr < cdiv(M, O_GT); ++gr)
         for (int gc = 0; gc < KG; ++gc) {                 /* GTs row-major */
             int64_t g = (int64_t)gr * KG + gc;
             gtile_offset[g] = (int32_t)running;           /* start of GT g's values */
@@ -135,7 +143,7 @@ int oracle_encode(const uint16_t *W, int M, int K, int32_t *gtile_offset, uint64
                     uint64_t bm = 0;
                     for (int b = 0; b < 64; ++b) {
                         int r, c; bt_elem(gr, gc, tt, bt, b, &r, &c);
-                        uint16_t v = W[(size_t)r * K + c];
+                        uint16_t v = w_at(W, M, K, r, c);
                         if (nonzero16(v)) {
                             bm |= (uint64_t)1 << b;                  /* set bit = non-zero */
                             values[running++] = v;                   /* nested order */
@@ -153,8 +161,8 @@ int oracle_encode(const uint16_t *W, int M, int K, int32_t *gtile_offset, uint64
 int oracle_decode(const int32_t *gtile_offset, const uint64_t *bitmap, const uint16_t *values,
                   int M, int K, uint16_t *W_out) {
     if (!gtile_offset || !bitmap || !W_out || !valid_shape(M, K)) return O_EINVAL;
-    int KG = K / O_GT;
-    for (int gr = 0; gr < M / O_GT; ++gr)
+    int KG = cdiv(K, O_GT);
+    for (int gr = 0; gr < cdiv(M, O_GT); ++gr)
         for (int gc = 0; gc < KG; ++gc) {
             int64_t g = (int64_t)gr * KG + gc;
             int64_t pos = gtile_offset[g];
@@ -163,7 +171,8 @@ int oracle_decode(const int32_t *gtile_offset, const uint64_t *bitmap, const uin
                     uint64_t bm = bitmap[(g * 16 + tt) * 4 + bt];
                     for (int b = 0; b < 64; ++b) {
                         int r, c; bt_elem(gr, gc, tt, bt, b, &r, &c);
-                        W_out[(size_t)r * K + c] = ((bm >> b) & 1) ? values[pos++] : 0x0000;
+                        uint16_t v = ((bm >> b) & 1) ? values[pos++] : 0x0000;
+                        if (r < M && c < K) W_out[(size_t)r * K + c] = v;   /* padding dropped (A8) */
                     }
                 }
         }
@@ -190,9 +199,9 @@ int oracle_spmm_tca_f64(const int32_t *gtile_offset, const uint64_t *bitmap, con
                         const uint16_t *X, int M, int K, int N, double *Y) {
     if (!gtile_offset || !bitmap || !X || !Y || !valid_shape(M, K) || N <= 0) return O_EINVAL;
     memset(Y, 0, sizeof(double) * (size_t)M * N);
-    int KG = K / O_GT;
+    int KG = cdiv(K, O_GT);
     double *xrow = (double *)malloc(sizeof(double) * (size_t)N);
-    for (int gr = 0; gr < M / O_GT; ++gr)
+    for (int gr = 0; gr < cdiv(M, O_GT); ++gr)
         for (int gc = 0; gc < KG; ++gc) {
             int64_t g = (int64_t)gr * KG + gc;
             int64_t pos = gtile_offset[g];
@@ -203,6 +212,7 @@ int oracle_spmm_tca_f64(const int32_t *gtile_offset, const uint64_t *bitmap, con
                         if (!((bm >> b) & 1)) continue;
                         int r, c; bt_elem(gr, gc, tt, bt, b, &r, &c);
                         double w = oracle_f16_to_f64(values[pos++]);
+                        if (r >= M || c >= K) return O_EINVAL;   /* a bit in the padding: not an encoding */
                         for (int n = 0; n < N; ++n) xrow[n] = oracle_f16_to_f64(X[(size_t)c * N + n]);
                         for (int n = 0; n < N; ++n) Y[(size_t)r * N + n] += w * xrow[n];
                     }
@@ -220,7 +230,7 @@ int oracle_spmm_tca_rows_f64(const int32_t *gtile_offset, const uint64_t *bitmap
                              const uint16_t *X, int M, int K, int N,
                              const int32_t *rows, int nrows, double *Yrows) {
     if (!gtile_offset || !bitmap || !X || !Yrows || !rows || !valid_shape(M, K) || N <= 0) return O_EINVAL;
-    int KG = K / O_GT;
+    int KG = cdiv(K, O_GT);
     for (int q = 0; q < nrows; ++q) {
         int row = rows[q];
         if (row < 0 || row >= M) return O_EINVAL;
@@ -238,6 +248,7 @@ int oracle_spmm_tca_rows_f64(const int32_t *gtile_offset, const uint64_t *bitmap
                         int r, c; bt_elem(gr, gc, tt, bt, b, &r, &c);
                         uint16_t v = values[pos++];
                         if (r != row) continue;
+                        if (c >= K) return O_EINVAL;              /* a bit in the padding */
                         double w = oracle_f16_to_f64(v);
                         for (int n = 0; n < N; ++n) y[n] += w * oracle_f16_to_f64(X[(size_t)c * N + n]);
                     }
@@ -286,12 +297,14 @@ void oracle_smbd_tctile(const uint64_t bm[4], const uint16_t *tt_values, int lan
  * Rank r of `world` owns GT rows [r*q + min(r, rem), ...) with q = MG / world,
  * rem = MG % world: contiguous, multiples of 64 rows, sizes differ by <= 1 GT row. */
 int oracle_tp_rows(int M, int world, int rank, int *row_begin, int *row_count) {
-    if (M <= 0 || M % O_GT || world <= 0 || rank < 0 || rank >= world || !row_begin || !row_count) return O_EINVAL;
-    int MG = M / O_GT, q = MG / world, rem = MG % world;
+    if (M <= 0 || world <= 0 || rank < 0 || rank >= world || !row_begin || !row_count) return O_EINVAL;
+    int MG = cdiv(M, O_GT), q = MG / world, rem = MG % world;
     int gb = rank * q + (rank < rem ? rank : rem);
     int gn = q + (rank < rem ? 1 : 0);
     *row_begin = gb * O_GT;
     *row_count = gn * O_GT;
+    if (*row_begin > M) *row_begin = M;                    /* A8: the ragged tail belongs to the */
+    if (*row_begin + *row_count > M) *row_count = M - *row_begin;   /* rank owning the last GT row */
     return O_OK;
 }
 

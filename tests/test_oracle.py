@@ -31,7 +31,7 @@ def closed_form_bt(r, c, K):
     """Global BitmapTile index and bit of element (r, c) — SURVEY §8(c) closed form,
     derived from P:192 (BTs column-major in a TT), P:194 (TTs column-major in a GT,
     GTs row-major) and P:287 (bit b <-> (b/8, b%8))."""
-    g = (r // 64) * (K // 64) + c // 64
+    g = (r // 64) * (-(-K // 64)) + c // 64     # K/64 rounded up: ragged shapes are zero-padded (A8)
     tt = ((c % 64) // 16) * 4 + (r % 64) // 16
     bt = ((c % 16) // 8) * 2 + (r % 16) // 8
     return (g * 16 + tt) * 4 + bt, (r % 8) * 8 + c % 8
@@ -221,9 +221,42 @@ def test_roundtrip_hypothesis(mg, kg, s, seed):
 
 def test_invalid_shapes():
     with pytest.raises(oracle.OracleError):
-        oracle.encode(np.zeros((65, 64), dtype=np.uint16))
+        oracle.spmm_f64(oracle.encode(np.ones((64, 64), dtype=np.uint16)), np.zeros((64, 0), dtype=np.uint16))
     with pytest.raises(oracle.OracleError):
-        oracle.encode(np.zeros((64, 96), dtype=np.uint16))
+        oracle.tp_rows(0, 1, 0)
+
+
+@pytest.mark.parametrize("M,K", [(1, 1), (65, 64), (64, 96), (70, 100), (130, 9)])
+def test_ragged_shapes_single_nonzero_brute_force(M, K):
+    """Reading A8: a shape that is not a multiple of 64 is zero-padded to whole GroupTiles. Every
+    single-non-zero position lands on the closed-form BT and bit (with K/64 rounded up), the
+    padding holds no bit, NGT = ceil(M/64) ceil(K/64), NBT = 64 NGT, and decode returns W."""
+    ngt = (-(-M // 64)) * (-(-K // 64))
+    for r in range(M):
+        for c in range(0, K, max(1, K // 7)):
+            W = np.zeros((M, K), dtype=np.uint16)
+            W[r, c] = 0x3C00
+            T = oracle.encode(W)
+            assert T.gtile_offset.shape == (ngt + 1,) and T.bitmap.shape == (64 * ngt,)
+            bt, bit = closed_form_bt(r, c, K)
+            nz = np.flatnonzero(T.bitmap)
+            assert nz.tolist() == [bt] and int(T.bitmap[bt]) == 1 << bit
+            assert np.array_equal(oracle.decode(T), W)
+
+
+def test_ragged_round_trip_and_product():
+    rng = np.random.default_rng(9)
+    for M, K in [(100, 70), (200, 130), (64, 65), (1, 300)]:
+        W = synth.weight(M, K, 0.5, seed=M * 1000 + K)
+        X = synth.activation(K, 5, seed=K)
+        T = oracle.encode(W)
+        assert np.array_equal(oracle.decode(T), canon(W))
+        assert int(sum(bin(int(b)).count("1") for b in T.bitmap)) == T.nnz == int(np.count_nonzero(W & 0x7FFF))
+        ref = W.view(np.float16).astype(np.float64) @ X.view(np.float16).astype(np.float64)
+        assert np.array_equal(oracle.spmm_f64(T, X), ref)
+        rows = rng.choice(M, size=min(M, 5), replace=False).astype(np.int32)
+        assert np.array_equal(oracle.spmm_rows_f64(T, X, rows), ref[rows])
+        assert oracle.storage_bytes(M, K, T.n_values) == 4 * (oracle.ngt(M, K) + 1) + 8 * 64 * oracle.ngt(M, K) + 2 * T.n_values
 
 
 # ---------------------------------------------------------------- checkerboard / eq. (9)
