@@ -10,16 +10,18 @@
  * TCA-BME: 8x8 BitmapTiles (one uint64 bitmap each) grouped
  * 2x2 column-major into 16x16 TCTiles, TCTiles column-major inside
  * 64x64 GroupTiles, GroupTiles row-major. Three arrays:
- *   gtile_offset int32[NGT+1], NGT = (M/64)(K/64): start (in fp16 elements) of
+ *   gtile_offset int32[NGT+1], NGT = ceil(M/64) ceil(K/64): start (in fp16 elements) of
  *                each GroupTile's values, gtile_offset[0] = 0,
  *                gtile_offset[NGT] = n_values;
- *   bitmap       uint64[NBT], NBT = M*K/64, in GroupTile -> TCTile -> BitmapTile
+ *   bitmap       uint64[NBT], NBT = 64 NGT, in GroupTile -> TCTile -> BitmapTile
  *                order; bit b <-> (row b/8, col b%8) of the BitmapTile;
  *   values       fp16[n_values], non-zeros in the same nested order, ascending
  *                bit order inside a BitmapTile; each GroupTile's
  *                segment is padded with +0.0 to a multiple of 8 halves (16 B,
  *                P:266). Storage = eq. (9) + padding (<= 7 halves/GT).
  * "Non-zero" means (bits & 0x7FFF) != 0: -0.0 is dropped, NaN/Inf are kept.
+ * M and K need not be multiples of 64: the matrix is zero-padded to whole
+ * GroupTiles (no bit set and no value stored in the padding, A8).
  * All readings of silent/garbled points are listed in DESIGN.md.
  *
  * Conventions for every call:
@@ -48,8 +50,8 @@ extern "C" {
 
 typedef enum {
     SPINFER_OK = 0,
-    SPINFER_EINVAL = -1,     /* null pointer, bad shape (M or K not a positive multiple of 64,
-                                N not in {8,16,24,32}), misaligned pointer, struct/call mismatch */
+    SPINFER_EINVAL = -1,     /* null pointer, bad shape (M or K <= 0, N not in [1, 32]),
+                                misaligned pointer, struct/call mismatch, unknown activation */
     SPINFER_ENOSPC = -2,     /* workspace too small */
     SPINFER_EOVERFLOW = -3,  /* n_values would reach 2^31 (gtile_offset is int32) */
     SPINFER_ECUDA = -4,      /* CUDA launch/runtime error */
@@ -67,7 +69,7 @@ typedef enum {
 /* Host-side descriptor of one TCA-BME matrix. The three device arrays are
  * caller-owned (e.g. torch tensors). */
 typedef struct {
-    int32_t M, K;             /* M % 64 == 0, K % 64 == 0 */
+    int32_t M, K;             /* > 0 (not necessarily multiples of 64: zero-padded GroupTiles) */
     int32_t gt_h, gt_w;       /* must be 64, 64 */
     int64_t nnz;              /* true non-zeros (informational) */
     int64_t n_values;         /* == gtile_offset[NGT] (padded count), < 2^31 */
@@ -127,8 +129,9 @@ SPINFER_API int spinfer_spmm_ex(const spinfer_tca *T, const uint16_t *X, uint16_
                                 const uint16_t *bias, int act, void *workspace, size_t ws_bytes, void *stream);
 
 /* Tensor-parallel row partition: rank `rank` of `world` owns rows
- * [*row_begin, *row_begin + *row_count) — contiguous, multiples of 64, sizes
- * differ by at most 64 (host only). */
+ * [*row_begin, *row_begin + *row_count) — contiguous, whole GroupTile rows (multiples of 64;
+ * the ragged tail of an M that is not a multiple of 64 goes to the rank owning the last GT
+ * row), sizes differ by at most 64; ranks beyond the GT-row count get 0 rows (host only). */
 SPINFER_API int spinfer_tp_rows(int M, int world, int rank, int *row_begin /* host */, int *row_count /* host */);
 
 /* Row-partitioned SpMM: T_shard encodes W[row_begin : row_begin+row_count, :]

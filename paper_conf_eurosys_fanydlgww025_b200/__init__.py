@@ -119,10 +119,10 @@ class TCA:
     def shard(self, row_begin: int, row_count: int) -> "TCA":
         """Zero-copy row shard: GT rows [a, b) are a contiguous slice of all three
         arrays; GTileOffset is rebased (on device) by the shard's first offset."""
-        if row_begin % GT or row_count % GT:
-            raise ValueError("shard rows must be multiples of 64")
-        KG = self.K // GT
-        a, b = row_begin // GT, (row_begin + row_count) // GT
+        if row_begin % GT or (row_count % GT and row_begin + row_count != self.M):
+            raise ValueError("shard rows must be multiples of 64 (except a ragged tail ending at M)")
+        KG = -(-self.K // GT)
+        a, b = row_begin // GT, -(-(row_begin + row_count) // GT)
         off = self.gtile_offset[a * KG: b * KG + 1]
         base = int(off[0].item())
         end = int(off[-1].item())
@@ -136,7 +136,8 @@ class TCA:
 
 def storage_bytes(M: int, K: int, n_values: int) -> int:
     """Buffer bytes of a TCA-BME matrix: eq. (9) with the padded value count."""
-    return 4 * ((M // GT) * (K // GT) + 1) + 8 * (M * K // 64) + 2 * n_values
+    ngt = (-(-M // GT)) * (-(-K // GT))   # zero-padded to whole GroupTiles (reading A8)
+    return 4 * (ngt + 1) + 8 * 64 * ngt + 2 * n_values
 
 
 def algorithmic_bytes(T: TCA, N: int) -> int:
@@ -155,12 +156,12 @@ def encode(W: torch.Tensor, stream=None) -> TCA:
     L = lib()
     st = _stream(stream)
     with torch.cuda.device(W.device):
-        off = torch.empty((M // GT) * (K // GT) + 1 if M % GT == 0 and K % GT == 0 else 1, dtype=torch.int32,
+        off = torch.empty((-(-M // GT)) * (-(-K // GT)) + 1, dtype=torch.int32,
                           device=W.device)
         nv, nz, mx = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int32()
         _check(L.spinfer_encode_count(W.data_ptr(), M, K, off.data_ptr(), ctypes.byref(nv), ctypes.byref(nz),
                                       ctypes.byref(mx), st), "spinfer_encode_count")
-        bm = torch.empty(M * K // 64, dtype=torch.int64, device=W.device)
+        bm = torch.empty(64 * (off.numel() - 1), dtype=torch.int64, device=W.device)   # NBT = 64 NGT
         vals = torch.empty(max(nv.value, 8), dtype=torch.float16, device=W.device)
         T = TCA(M, K, off, bm, vals, int(nv.value), int(nz.value), int(mx.value))
         cs = T.c_struct()

@@ -17,7 +17,8 @@ int check_device() {
     return (major == 10 && minor == 0) ? SPINFER_OK : SPINFER_ENODEV;   // built for sm_100a only
 }
 
-static bool shape_ok(int M, int K) { return M > 0 && K > 0 && M % kGT == 0 && K % kGT == 0; }
+// any M, K > 0: shapes that are not multiples of 64 are zero-padded to whole GroupTiles (A8)
+static bool shape_ok(int M, int K) { return M > 0 && K > 0; }
 
 int validate_tca(const spinfer_tca *T, int M, int K) {
     if (!T || !T->gtile_offset || !T->bitmap || !T->values) return SPINFER_EINVAL;
@@ -100,11 +101,15 @@ int spinfer_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, in
 }
 
 int spinfer_tp_rows(int M, int world, int rank, int *row_begin, int *row_count) {
-    if (!row_begin || !row_count || M <= 0 || M % kGT || world <= 0 || rank < 0 || rank >= world)
+    if (!row_begin || !row_count || M <= 0 || world <= 0 || rank < 0 || rank >= world)
         return SPINFER_EINVAL;
-    const int MG = M / kGT, q = MG / world, rem = MG % world;
-    *row_begin = (rank * q + (rank < rem ? rank : rem)) * kGT;
-    *row_count = (q + (rank < rem ? 1 : 0)) * kGT;
+    const int MG = (M + kGT - 1) / kGT, q = MG / world, rem = MG % world;
+    int b = (rank * q + (rank < rem ? rank : rem)) * kGT;
+    int c = (q + (rank < rem ? 1 : 0)) * kGT;
+    if (b > M) b = M;                  // A8: the ragged tail belongs to the rank owning the last GT row
+    if (b + c > M) c = M - b;
+    *row_begin = b;
+    *row_count = c;
     return SPINFER_OK;
 }
 

@@ -47,13 +47,22 @@ __device__ __forceinline__ uint32_t nz_byte(uint4 v) {
     return m;
 }
 
-__device__ __forceinline__ uint64_t bt_bitmap(const uint16_t *__restrict__ W, int K, int row0, int col0) {
+// 8 consecutive halves W[r][c0 .. c0+7] of the zero-padded matrix (reading A8): one 16-byte
+// load when the row segment is inside W and 16-byte aligned (K % 8 == 0), else element-wise.
+__device__ __forceinline__ uint4 row8(const uint16_t *__restrict__ W, int M, int K, int r, int c0) {
+    if (r >= M) return make_uint4(0u, 0u, 0u, 0u);
+    if ((K & 7) == 0 && c0 + 8 <= K) return __ldg(reinterpret_cast<const uint4 *>(W + (size_t)r * K + c0));
+    uint32_t w[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+        if (c0 + j < K) w[j >> 1] |= (uint32_t)__ldg(W + (size_t)r * K + c0 + j) << (16 * (j & 1));
+    return make_uint4(w[0], w[1], w[2], w[3]);
+}
+
+__device__ __forceinline__ uint64_t bt_bitmap(const uint16_t *__restrict__ W, int M, int K, int row0, int col0) {
     uint64_t bm = 0;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) {
-        uint4 v = __ldg(reinterpret_cast<const uint4 *>(W + (size_t)(row0 + i) * K + col0));
-        bm |= (uint64_t)nz_byte(v) << (8 * i);
-    }
+    for (int i = 0; i < 8; ++i) bm |= (uint64_t)nz_byte(row8(W, M, K, row0 + i, col0)) << (8 * i);
     return bm;
 }
 
@@ -75,12 +84,12 @@ __device__ __forceinline__ int gt_exclusive_scan(int c, int *total) {
     return excl;
 }
 
-__global__ void __launch_bounds__(kThreads) k_encode_count(const uint16_t *__restrict__ W, int K, int KG,
+__global__ void __launch_bounds__(kThreads) k_encode_count(const uint16_t *__restrict__ W, int M, int K, int KG,
                                                            int64_t NGT, int32_t *__restrict__ padcount,
                                                            unsigned long long *__restrict__ stats) {
     BtPos p = bt_pos(KG);
     int c = 0;
-    if (p.g < NGT) c = __popcll(bt_bitmap(W, K, p.row0, p.col0));
+    if (p.g < NGT) c = __popcll(bt_bitmap(W, M, K, p.row0, p.col0));
     int total;
     (void)gt_exclusive_scan(c, &total);
     __shared__ unsigned long long blk_nnz;
@@ -140,13 +149,13 @@ __global__ void __launch_bounds__(1024) k_scan_offsets(int32_t *__restrict__ a, 
     }
 }
 
-__global__ void __launch_bounds__(kThreads) k_encode_fill(const uint16_t *__restrict__ W, int K, int KG, int64_t NGT,
+__global__ void __launch_bounds__(kThreads) k_encode_fill(const uint16_t *__restrict__ W, int M, int K, int KG, int64_t NGT,
                                                           const int32_t *__restrict__ off,
                                                           uint64_t *__restrict__ bitmap,
                                                           uint16_t *__restrict__ values) {
     BtPos p = bt_pos(KG);
     bool live = p.g < NGT;
-    uint64_t bm = live ? bt_bitmap(W, K, p.row0, p.col0) : 0ull;
+    uint64_t bm = live ? bt_bitmap(W, M, K, p.row0, p.col0) : 0ull;
     int c = __popcll(bm);
     int total;
     int excl = gt_exclusive_scan(c, &total);
@@ -156,7 +165,7 @@ __global__ void __launch_bounds__(kThreads) k_encode_fill(const uint16_t *__rest
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
         if (((bm >> (8 * i)) & 0xFFu) == 0) continue;
-        uint4 v = __ldg(reinterpret_cast<const uint4 *>(W + (size_t)(p.row0 + i) * K + p.col0));
+        uint4 v = row8(W, M, K, p.row0 + i, p.col0);
         uint32_t w[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
@@ -172,7 +181,7 @@ __global__ void __launch_bounds__(kThreads) k_encode_fill(const uint16_t *__rest
 
 __global__ void __launch_bounds__(kThreads) k_decode(const int32_t *__restrict__ off,
                                                      const uint64_t *__restrict__ bitmap,
-                                                     const uint16_t *__restrict__ values, int K, int KG,
+                                                     const uint16_t *__restrict__ values, int M, int K, int KG,
                                                      int64_t NGT, uint16_t *__restrict__ W) {
     BtPos p = bt_pos(KG);
     bool live = p.g < NGT;
@@ -188,7 +197,15 @@ __global__ void __launch_bounds__(kThreads) k_decode(const int32_t *__restrict__
         for (int j = 0; j < 8; ++j) {
             if ((bm >> (8 * i + j)) & 1ull) w[j >> 1] |= (uint32_t)values[pos++] << (16 * (j & 1));
         }
-        *reinterpret_cast<uint4 *>(W + (size_t)(p.row0 + i) * K + p.col0) = make_uint4(w[0], w[1], w[2], w[3]);
+        const int r = p.row0 + i;
+        if (r >= M) continue;                                  // zero padding is not written (A8)
+        if ((K & 7) == 0 && p.col0 + 8 <= K) {
+            *reinterpret_cast<uint4 *>(W + (size_t)r * K + p.col0) = make_uint4(w[0], w[1], w[2], w[3]);
+        } else {
+#pragma unroll
+            for (int j = 0; j < 8; ++j)
+                if (p.col0 + j < K) W[(size_t)r * K + p.col0 + j] = (uint16_t)(w[j >> 1] >> (16 * (j & 1)));
+        }
     }
 }
 
@@ -196,28 +213,28 @@ __global__ void __launch_bounds__(kThreads) k_decode(const int32_t *__restrict__
 
 int launch_encode_count(const uint16_t *W, int M, int K, int32_t *gtile_offset, int64_t *stats_dev,
                         cudaStream_t st) {
-    int KG = K / kGT;
-    int64_t NGT = (int64_t)(M / kGT) * KG;
+    int KG = (K + kGT - 1) / kGT;
+    int64_t NGT = (int64_t)((M + kGT - 1) / kGT) * KG;   // zero-padded to whole GroupTiles (A8)
     int64_t blocks = (NGT + kGTPerBlock - 1) / kGTPerBlock;
-    k_encode_count<<<(unsigned)blocks, kThreads, 0, st>>>(W, K, KG, NGT, gtile_offset,
+    k_encode_count<<<(unsigned)blocks, kThreads, 0, st>>>(W, M, K, KG, NGT, gtile_offset,
                                                           reinterpret_cast<unsigned long long *>(stats_dev));
     k_scan_offsets<<<1, 1024, 0, st>>>(gtile_offset, NGT, reinterpret_cast<unsigned long long *>(stats_dev));
     return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
 }
 
 int launch_encode_fill(const uint16_t *W, const spinfer_tca *T, cudaStream_t st) {
-    int KG = T->K / kGT;
-    int64_t NGT = (int64_t)(T->M / kGT) * KG;
+    int KG = (T->K + kGT - 1) / kGT;
+    int64_t NGT = (int64_t)((T->M + kGT - 1) / kGT) * KG;
     int64_t blocks = (NGT + kGTPerBlock - 1) / kGTPerBlock;
-    k_encode_fill<<<(unsigned)blocks, kThreads, 0, st>>>(W, T->K, KG, NGT, T->gtile_offset, T->bitmap, T->values);
+    k_encode_fill<<<(unsigned)blocks, kThreads, 0, st>>>(W, T->M, T->K, KG, NGT, T->gtile_offset, T->bitmap, T->values);
     return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
 }
 
 int launch_decode(const spinfer_tca *T, uint16_t *W_out, cudaStream_t st) {
-    int KG = T->K / kGT;
-    int64_t NGT = (int64_t)(T->M / kGT) * KG;
+    int KG = (T->K + kGT - 1) / kGT;
+    int64_t NGT = (int64_t)((T->M + kGT - 1) / kGT) * KG;
     int64_t blocks = (NGT + kGTPerBlock - 1) / kGTPerBlock;
-    k_decode<<<(unsigned)blocks, kThreads, 0, st>>>(T->gtile_offset, T->bitmap, T->values, T->K, KG, NGT, W_out);
+    k_decode<<<(unsigned)blocks, kThreads, 0, st>>>(T->gtile_offset, T->bitmap, T->values, T->M, T->K, KG, NGT, W_out);
     return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
 }
 

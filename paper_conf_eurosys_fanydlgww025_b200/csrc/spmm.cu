@@ -142,6 +142,7 @@ struct Params {
     uint32_t o_desc, o_tbl, o_stage;            // region offsets from the smem base
     long long *trace;   // experiments only (SPINFER_TRACE): [kTraceCTAs][kTraceStages][8] clock64 stamps
     float avg_gt;       // n_values / NGT: predicts where a CTA's first value range lies (start-up page prefetch)
+    int M;              // real rows of Y (M need not be a multiple of 64: rows >= M are padding, A8)
     int dbg;            // experiments only (SPINFER_DEBUG_MODE): bit0 = consumers skip decode/MMA, bit1 = scan skips work
 };
 
@@ -321,6 +322,8 @@ __device__ __forceinline__ float epi_act(float v, float b, int act) {
 
 // prm.N = the caller's column count (row stride of Y); the kernel computes NT * 8 >= N columns
 // (X zero-padded to a multiple of 8) and drops the padding columns here.
+// EPI: the general path — fused bias / activation (spinfer_spmm_ex) and the padding rows of a
+// ragged M (A8); the plain path (EPI = false) is only launched for M % 64 == 0 without epilogue.
 template <int NT, bool EPI>
 __device__ __forceinline__ void store_y(const Params &prm, int row_base, float (&acc)[4][NT][4], int lane) {
     uint16_t *const Y = prm.Y;
@@ -328,7 +331,7 @@ __device__ __forceinline__ void store_y(const Params &prm, int row_base, float (
 #pragma unroll
     for (int tr = 0; tr < 4; ++tr) {
         const int r0 = row_base + tr * 16 + (lane >> 2);
-        if (EPI) {   // fused epilogue: a separate kernel instantiation, so the plain path pays nothing
+        if (EPI && (prm.bias || prm.act)) {   // fused epilogue (general instantiation only)
             const float b0 = prm.bias ? __half2float(__ushort_as_half(prm.bias[r0])) : 0.f;
             const float b1 = prm.bias ? __half2float(__ushort_as_half(prm.bias[r0 + 8])) : 0.f;
 #pragma unroll
@@ -344,7 +347,14 @@ __device__ __forceinline__ void store_y(const Params &prm, int row_base, float (
             int col = nt * 8 + 2 * (lane & 3);
             __half2 lo = __floats2half2_rn(acc[tr][nt][0], acc[tr][nt][1]);   // one RNE per output (A11)
             __half2 hi = __floats2half2_rn(acc[tr][nt][2], acc[tr][nt][3]);
-            if (N == NT * 8) {
+            if (EPI && r0 + 8 >= prm.M) {   // last GT row of a ragged M (A8): padding rows are not stored
+                __half *y0 = reinterpret_cast<__half *>(Y + (size_t)r0 * N);
+                __half *y1 = reinterpret_cast<__half *>(Y + (size_t)(r0 + 8) * N);
+                if (r0 < prm.M && col < N) y0[col] = __low2half(lo);
+                if (r0 < prm.M && col + 1 < N) y0[col + 1] = __high2half(lo);
+                if (r0 + 8 < prm.M && col < N) y1[col] = __low2half(hi);
+                if (r0 + 8 < prm.M && col + 1 < N) y1[col + 1] = __high2half(hi);
+            } else if (N == NT * 8) {
                 *reinterpret_cast<__half2 *>(Y + (size_t)r0 * N + col) = lo;
                 *reinterpret_cast<__half2 *>(Y + (size_t)(r0 + 8) * N + col) = hi;
             } else {
@@ -1117,6 +1127,7 @@ template <int NB>
 __device__ __forceinline__ void store_y_row(const Params &prm, size_t grow, float (&v)[NB]) {
     uint16_t *const Y = prm.Y;
     const int N = prm.N;
+    if (grow >= (size_t)prm.M) return;   // padding row of a ragged M (A8)
     if (prm.bias || prm.act) {   // fused epilogue (spinfer_spmm_ex)
         const float b = prm.bias ? __half2float(__ushort_as_half(prm.bias[grow])) : 0.f;
 #pragma unroll
@@ -1699,7 +1710,7 @@ int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int bo
 }
 
 bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl, bool tc) {
-    const int MG = M / kGT, KG = K / kGT;
+    const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;   // zero-padded to whole GTs (A8)
     const int nRB = (MG + kR - 1) / kR;
     const long long U = (long long)nRB * KG;
     pl->P = choose_P(U);
@@ -1783,8 +1794,8 @@ int launch_tc(const Plan &pl, cudaStream_t st) {
 }  // namespace
 
 size_t spmm_workspace_bytes(int M, int K, int N) {
-    if (M <= 0 || K <= 0 || M % kGT || K % kGT || N <= 0 || N > 32 || M / kGT > kMaxCounters) return 0;
-    const int MG = M / kGT, KG = K / kGT;
+    if (M <= 0 || K <= 0 || N <= 0 || N > 32 || (M + kGT - 1) / kGT > kMaxCounters) return 0;
+    const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;
     const long long U = (long long)((MG + kR - 1) / kR) * KG;
     const int P = choose_P(U);
     const int Np = (N + 7) & ~7;   // computed columns (X zero-padded to a multiple of 8)
@@ -1809,7 +1820,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     if (ke && ke[0] == 't') tc = true;
     if (ke && ke[0] == 'm') tc = false;
     // the tcgen05 kernel's fix-up keeps one counter per rowblock and TMEM lane quarter
-    if (tc && 4LL * ((M / kGT + kR - 1) / kR) > kMaxCounters) tc = false;
+    if (tc && 4LL * (((M + kGT - 1) / kGT + kR - 1) / kR) > kMaxCounters) tc = false;
     if (!make_plan(M, K, Np, T->max_gt_values, &pl, tc)) return SPINFER_EINVAL;
     const size_t need = spmm_workspace_bytes(M, K, N);
     if (need == 0) return SPINFER_EINVAL;
@@ -1833,11 +1844,14 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     q.Y = Y;
     q.bias = bias;
     q.act = act;
-    const bool epi = bias != nullptr || act != SPINFER_ACT_NONE;
+    // the general store path (fused bias / activation, padding rows of a ragged M) is a separate
+    // instantiation, so the plain aligned path carries none of it
+    const bool epi = bias != nullptr || act != SPINFER_ACT_NONE || (M % kGT) != 0;
     q.ws_cnt = reinterpret_cast<int32_t *>(ws);
     q.ws_part = reinterpret_cast<float *>(reinterpret_cast<uint8_t *>(ws) + kCounterBytes);
     q.ws_epi = q.ws_part + (size_t)pl.P * 2 * kR * 64 * Np;
-    q.avg_gt = (float)((double)T->n_values / ((double)(M / kGT) * (double)(K / kGT)));
+    q.avg_gt = (float)((double)T->n_values / ((double)q.MG * (double)q.KG));
+    q.M = M;
     q.dbg = 0;
     if (const char *e = getenv("SPINFER_DEBUG_MODE")) q.dbg = atoi(e);
     q.trace = nullptr;

@@ -30,11 +30,13 @@ GT = 64
 
 def tp_rows(M: int, world: int, rank: int):
     """Same partition as spinfer_tp_rows (host logic, no device needed)."""
-    if M <= 0 or M % GT or world <= 0 or not (0 <= rank < world):
+    if M <= 0 or world <= 0 or not (0 <= rank < world):
         raise ValueError("bad tp_rows arguments")
-    MG = M // GT
+    MG = -(-M // GT)                      # ragged M: zero-padded to whole GroupTiles (reading A8)
     q, rem = divmod(MG, world)
-    return (rank * q + min(rank, rem)) * GT, (q + (1 if rank < rem else 0)) * GT
+    b, c = (rank * q + min(rank, rem)) * GT, (q + (1 if rank < rem else 0)) * GT
+    b = min(b, M)
+    return b, min(c, M - b)               # the ragged tail belongs to the rank owning the last GT row
 
 
 @dataclass

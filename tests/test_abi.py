@@ -55,12 +55,14 @@ def test_status_strings_and_version(sp):
 
 def test_tp_rows_host_logic(sp):
     import oracle
-    for M in (64, 1152, 9216, 28672, 36864):
-        for world in (1, 2, 4, 8):
-            for r in range(world):
-                assert sp.tp_rows(M, world, r) == oracle.tp_rows(M, world, r)
+    for M in (64, 100, 1000, 1152, 9216, 28672, 36864):      # 100, 1000: ragged tail (reading A8)
+        for world in (1, 2, 3, 4, 8):
+            spans = [sp.tp_rows(M, world, r) for r in range(world)]
+            assert spans == [oracle.tp_rows(M, world, r) for r in range(world)]
+            assert sum(c for _, c in spans) == M
+            assert all(b % 64 == 0 or c == 0 for b, c in spans)
     with pytest.raises(sp.SpinferError):
-        sp.tp_rows(100, 2, 0)
+        sp.tp_rows(0, 2, 0)
     with pytest.raises(sp.SpinferError):
         sp.tp_rows(128, 2, 2)
 

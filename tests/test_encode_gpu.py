@@ -71,9 +71,8 @@ def test_encode_config2_full_size():
 
 
 def test_encode_invalid_shape():
+    """Ragged shapes are valid (zero-padded, reading A8; tests/test_ragged_gpu.py); an empty W is not."""
     import torch
     sp = _sp()
     with pytest.raises(sp.SpinferError):
-        sp.encode(torch.zeros((96, 64), dtype=torch.float16, device="cuda"))
-    with pytest.raises(sp.SpinferError):
-        sp.encode(torch.zeros((64, 100), dtype=torch.float16, device="cuda"))
+        sp.encode(torch.zeros((0, 64), dtype=torch.float16, device="cuda"))
