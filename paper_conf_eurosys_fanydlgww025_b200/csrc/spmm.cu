@@ -1111,17 +1111,6 @@ struct Ring {
     uint32_t b = 0, ph = 0;
     __device__ __forceinline__ void next() { if (++b == NBUF) { b = 0; ph ^= 1u; } }
 };
-// per-stage segment flags, computed identically by every role from the StageIter
-struct SegFlags {
-    bool full_start = false;
-    bool zero = false, seg_end = false, complete = false;
-    __device__ __forceinline__ void at(const StageIter &sg, const Params &prm) {
-        zero = sg.seg_first();
-        if (zero) full_start = (sg.gc == 0);
-        seg_end = sg.seg_last(prm);
-        complete = seg_end && full_start && (sg.gc + sg.g == prm.KG);
-    }
-};
 
 template <int NB>
 __device__ __forceinline__ void store_y_row(const Params &prm, size_t grow, float (&v)[NB]) {
@@ -1159,6 +1148,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
     constexpr int ABufs = TmemTC<NB>::ABufs;
     constexpr uint32_t DCol = TmemTC<NB>::DCol;
     constexpr uint32_t kEndBar = 1, kTeamBar = 2;   // named barriers: decode warps at the end; 2 + kt: k-team kt
+    constexpr uint32_t kDescBarTC = 6;              // stage descriptors written (scan warp 1 -> decode warps)
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *const smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     const uint32_t sbase = smem_u32(smem);
@@ -1330,6 +1320,28 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
                 }
             }
         };
+        if (sw == 1) {
+            // stage descriptors for the decode warps (same encoding as k_spmm's StageDesc)
+            if (lane == 0) {
+                StageIter d;
+                int n = 0;
+                bool full_start = false;
+                for (d.init(u0, u1, prm); d.valid(); d.next(prm), ++n) {
+                    const bool zero = d.seg_first();
+                    if (zero) full_start = (d.gc == 0);
+                    const bool seg_end = d.seg_last(prm);
+                    const bool complete = seg_end && full_start && (d.gc + d.g == KG);
+                    const uint32_t w0 = (uint32_t)d.rb | ((uint32_t)d.slot << 20) | (d.ph << 24) | ((uint32_t)zero << 25) |
+                                        ((uint32_t)seg_end << 26) | ((uint32_t)complete << 27) |
+                                        ((uint32_t)(d.rows - 1) << 28);
+                    sts_v4(sbase + prm.o_desc + 16u * (uint32_t)n,
+                           make_uint4(w0, (uint32_t)d.gc | ((uint32_t)d.g << 16), 0u, 0u));
+                }
+                reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3] = (uint32_t)n;
+            }
+            __syncwarp();
+            named_bar_arrive(6u, 32u * (CfgTC::CW + 1));
+        }
         StageIter it;
         it.init(u0, u1, prm);
         if (sw == 1) it.next(prm);
@@ -1526,8 +1538,11 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
     constexpr uint32_t idesc = (1u << 4) | (1u << 16) | ((uint32_t)(NB >> 3) << 17) | ((128u >> 4) << 24);
     constexpr uint64_t kDescHi = ((uint64_t)((8 * NB * 2) >> 4) << 32) | (1ull << 46) |
                                  ((uint64_t)(NB == 16 ? 6 : 4) << 61) | (1ull << 16);
+    auto tc_rd = [&](int si) {
+        const uint4 v = lds_v4(sbase + prm.o_desc + 16u * (uint32_t)si);
+        return StageDesc{v.x, v.y, v.z, v.w};
+    };
     Ring<ABufs> ar;
-    SegFlags sf;
     int seg = -1;
     uint32_t dpar = 1, dph = 1;     // D parity of the current segment and its phase (advanced at segment start)
     bool first = false;             // team: the next MMA starts the segment's accumulation
@@ -1536,10 +1551,14 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
     uint32_t pend_db = 0, pend_dph = 0;
     int pend_rb = 0, pend_rows = 0, pend_nt = 0;
     bool pend_complete = false;
-    StageIter it;
-    for (it.init(u0, u1, prm); it.valid(); it.next(prm), ar.next()) {
-        const int i = it.i, slot = it.slot;
-        sf.at(it, prm);
+    // per-stage descriptors (built once by scan warp 1): one 16-byte shared load per stage instead
+    // of every warp walking the StageIter and the segment flags
+    named_bar_sync(kDescBarTC, 32u * (kCW + 1));
+    const int nst = (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3];
+    for (int i = 0; i < nst; ++i, ar.next()) {
+        const StageDesc d = tc_rd(i);
+        const int slot = d.slot();
+        struct { bool zero, seg_end, complete; } sf = {d.zero(), d.seg_end(), d.complete()};
         if (sf.zero) {
             ++seg;
             dpar ^= 1u;
@@ -1547,18 +1566,18 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
             first = true;
             maxg = 0;
         }
-        maxg = max(maxg, it.g);
+        maxg = max(maxg, d.g());
         if (lane == 0) trace_ev(prm, p, i, warp, 0);
         const bool reuse0 = (dbg_mode(prm) & 4) != 0;   // experiment: stage 0's data for every stage
         if (!reuse0 || i == 0) {
-            mbar_wait_sleep(bar_scan + 8 * slot, it.par());   // table written (the scan runs ahead)
-            mbar_wait_sleep(bar_full + 8 * slot, it.par());   // values and X landed
+            mbar_wait_sleep(bar_scan + 8 * slot, d.par());   // table written (the scan runs ahead)
+            mbar_wait_sleep(bar_full + 8 * slot, d.par());   // values and X landed
         }
         if (lane == 0) trace_ev(prm, p, i, warp, 1);
         const uint32_t ab = (uint32_t)(kt * ABufs) + ar.b;
         if (i >= ABufs) mbar_wait(bar_ae + 8u * ab, ar.ph ^ 1u);
         tm_fence_after();
-        if (r < it.rows && kt < it.g && !(dbg_mode(prm) & 1)) {
+        if (r < d.rows() && kt < d.g() && !(dbg_mode(prm) & 1)) {
             const uint32_t tb = sbase + prm.o_tbl + (uint32_t)(reuse0 ? 0 : slot) * prm.tbl_bytes +
                                 (uint32_t)(r * G + kt) * 1024u + tbl_lane;
             const uint32_t acol = ab * 32u;
@@ -1579,7 +1598,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         tm_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(bar_empty + 8 * slot);   // this warp is done with the slot's values/table
-        const bool mm = kt < it.g;
+        const bool mm = kt < d.g();
 #if SPINFER_TC_LAST
         // the last of the team's 4 lane-quarter warps to finish its A tiles multiplies
         bool issuer = false;
@@ -1629,7 +1648,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         }
         if (sf.seg_end && (seg & 3) == kt) {
             pend = true;
-            pend_db = dpar; pend_dph = dph; pend_rb = it.rb; pend_rows = it.rows; pend_complete = sf.complete;
+            pend_db = dpar; pend_dph = dph; pend_rb = d.rb(); pend_rows = d.rows(); pend_complete = sf.complete;
             pend_nt = min(maxg, 4);
         }
         if (lane == 0) trace_ev(prm, p, i, warp, 3);
@@ -1739,7 +1758,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl, bool tc) {
         // stage descriptors: at most one per unit, and no more than ceil(units/G) + rowblock splits
         const uint32_t desc_bytes = align_up((uint32_t)(16 * std::min<long long>(upc, upc / G + upc / KG + 3)), 128);
         uint32_t fixed = o_desc + desc_bytes + 128 + 2048;   // +slack: t1 over-read, base and ring alignment
-        if (tc) fixed = 1024 + 128 + 1024;   // tcgen05 path: no descriptor table
+        if (tc) fixed = 1024 + align_up(desc_bytes, 1024) + 128 + 1024;   // tcgen05 path: descriptors (tables 1024-aligned)
         stage += tbl;                                     // k_spmm: each ring slot carries its table
         if ((long long)fixed + 2LL * stage > smem_max) continue;
         int S = (int)std::min<long long>(smax, ((long long)smem_max - fixed) / stage);
@@ -1753,7 +1772,7 @@ bool make_plan(int M, int K, int N, int max_gt_values, Plan *pl, bool tc) {
         q.tbl_bytes = tbl;
         q.o_desc = o_desc;
         q.o_tbl = q.o_desc + desc_bytes;
-        if (tc) q.o_tbl = 1024;
+        if (tc) q.o_tbl = q.o_desc + align_up(desc_bytes, 1024);
         q.o_stage = align_up(q.o_tbl + (uint32_t)S * tbl, 1024);
         pl->smem = (size_t)q.o_stage + (size_t)S * stage + 128 + 1024;   // +1024: runtime base alignment
         return true;

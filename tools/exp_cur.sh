@@ -1,1 +1,2 @@
-bash tools/ab.sh "base:libspinfer_base.so:" "base2:libspinfer_base2.so:" "rag:libspinfer_rag.so:" "rag2:libspinfer_rag2.so:"
+timeout 900 python -m pytest tests -m gpu -x -q --timeout 300 2>&1 | tail -3
+BENCH_ARGS="--N 32" bash tools/ab.sh "base32:libspinfer_base.so:" "desc32:libspinfer_tcdesc.so:"
