@@ -1099,6 +1099,9 @@ constexpr uint32_t kTcScan = 512;      // [S]: the slot's SMBD table is written
 constexpr uint32_t kTcTeamCnt = 960;   // int [k-team][A buffer]: A tiles written (last of 4 writers issues the MMA)
 // k-team MMA issue by the last of the team's 4 lane-quarter warps to finish its A tiles (a shared
 // atomic count per A buffer) instead of a named barrier of the 4 warps: no warp waits for another
+#ifndef SPINFER_TC_SCANFULL
+#define SPINFER_TC_SCANFULL 1
+#endif
 #ifndef SPINFER_TC_WARPFIX
 #define SPINFER_TC_WARPFIX 1
 #endif
@@ -1402,6 +1405,11 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
                 rel[rr] += (int)(((t & 0xFFFFu) + (t >> 16) + 7u) & ~7u);
             }
             __syncwarp();
+#if SPINFER_TC_SCANFULL
+            // publish the table only once the slot's values and X have landed too, so the decode
+            // warps wait on one barrier per stage
+            mbar_wait_sleep(bar_full + 8 * slot, sg.par());
+#endif
             if (lane == 0) mbar_arrive(bar_scan + 8 * slot);
             if (lane == 0) trace_ev(prm, p, sg.i, warp, 3);
             skip2(it);
@@ -1571,7 +1579,9 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         const bool reuse0 = (dbg_mode(prm) & 4) != 0;   // experiment: stage 0's data for every stage
         if (!reuse0 || i == 0) {
             mbar_wait_sleep(bar_scan + 8 * slot, d.par());   // table written (the scan runs ahead)
+#if !SPINFER_TC_SCANFULL
             mbar_wait_sleep(bar_full + 8 * slot, d.par());   // values and X landed
+#endif
         }
         if (lane == 0) trace_ev(prm, p, i, warp, 1);
         const uint32_t ab = (uint32_t)(kt * ABufs) + ar.b;
