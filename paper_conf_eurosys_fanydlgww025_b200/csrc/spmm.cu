@@ -1444,16 +1444,20 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
 #pragma unroll
         for (int j = 0; j < NB; ++j) v[j] = 0.f;
 #pragma unroll
+        // NB = 32: a team's two x16 loads in flight per wait (measured -0.5 %); NB = 16: one load and
+        // wait per team (batching two teams measured +1.8 %). Summed in team order: deterministic.
+#pragma unroll
         for (int tt = 0; tt < 4; ++tt) {
             if (tt < nteams) {
+                float x[NB / 16][16];
 #pragma unroll
-                for (int h = 0; h < NB / 16; ++h) {
-                    float x[16];
-                    tm_ld_32x32b_x16(t_q + DCol + ((uint32_t)tt * 2u + db) * NB + 16u * h, x);
-                    tm_wait_ld();
+                for (int h = 0; h < NB / 16; ++h)
+                    tm_ld_32x32b_x16(t_q + DCol + ((uint32_t)tt * 2u + db) * NB + 16u * h, x[h]);
+                tm_wait_ld();
 #pragma unroll
-                    for (int j = 0; j < 16; ++j) v[16 * h + j] += x[j];
-                }
+                for (int h = 0; h < NB / 16; ++h)
+#pragma unroll
+                    for (int j = 0; j < 16; ++j) v[16 * h + j] += x[h][j];
             }
         }
         tm_fence_before();
