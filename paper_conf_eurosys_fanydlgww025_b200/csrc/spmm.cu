@@ -1095,6 +1095,7 @@ struct TmemTC {
 // barrier / scalar region (bytes from the aligned smem base); per-warp tables from 1024
 constexpr uint32_t kTcFull = 0, kTcEmpty = 64, kTcEmptyX = 128, kTcTmemSlot = 208;
 constexpr uint32_t kTcAEmpty = 256, kTcDFull = 352, kTcDEmpty = 368, kTcFix = 384;   // aempty [4][3]
+constexpr uint32_t kTcAFull = 400;     // [k-team][A buffer]: the team's 4 lane-quarter warps wrote their A tiles
 constexpr uint32_t kTcScan = 512;      // [S]: the slot's SMBD table is written
 constexpr uint32_t kTcTeamCnt = 960;   // int [k-team][A buffer]: A tiles written (last of 4 writers issues the MMA)
 // k-team MMA issue by the last of the team's 4 lane-quarter warps to finish its A tiles (a shared
@@ -1104,6 +1105,9 @@ constexpr uint32_t kTcTeamCnt = 960;   // int [k-team][A buffer]: A tiles writte
 #endif
 #ifndef SPINFER_TC_WARPFIX
 #define SPINFER_TC_WARPFIX 1
+#endif
+#ifndef SPINFER_TC_AFULL
+#define SPINFER_TC_AFULL 0
 #endif
 #ifndef SPINFER_TC_LAST
 #define SPINFER_TC_LAST 0
@@ -1175,6 +1179,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
             mbar_init(bar_scan + 8 * s, 1);                // the stage's scan warp
         }
         for (int k = 0; k < 4 * ABufs; ++k) mbar_init(bar_ae + 8 * k, 1);   // [k-team][buffer]: team MMA commit
+        for (int k = 0; k < 4 * ABufs; ++k) mbar_init(sbase + kTcAFull + 8 * k, 4);   // [k-team][buffer]: A written
         for (int k = 0; k < 2; ++k) {
             mbar_init(bar_df + 8 * k, 4);                  // [segment parity]: the 4 k-teams' commits
             mbar_init(bar_de + 8 * k, 4);                  // the 4 warps of the finishing k-team
@@ -1625,6 +1630,13 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
             }
             issuer = (__shfl_sync(0xffffffffu, old, 0) & 3) == 3;
         }
+#elif SPINFER_TC_AFULL
+        // the team's 4 lane-quarter warps arrive on the A buffer's mbarrier (release: their TMEM
+        // stores, fenced above); only the team leader waits for it and multiplies — the other
+        // three go on to the next stage
+        if (lane == 0) mbar_arrive(sbase + kTcAFull + 8u * ab);
+        const bool issuer = (q == 0);
+        if (issuer) mbar_wait(sbase + kTcAFull + 8u * ab, ar.ph);
 #else
         // the team's 4 lane-quarter warps have written their A tiles: the team leader multiplies
         named_bar_sync(kTeamBar + (uint32_t)kt, 128);
