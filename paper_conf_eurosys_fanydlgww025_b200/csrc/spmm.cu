@@ -105,6 +105,10 @@ constexpr int kMaxStages = 8;
 #ifndef SPINFER_RELCNT
 #define SPINFER_RELCNT 0
 #endif
+// scan warps walk the per-CTA stage descriptors instead of their own StageIter
+#ifndef SPINFER_SCANDESC
+#define SPINFER_SCANDESC 0
+#endif
 #ifndef SPINFER_EPREF
 #define SPINFER_EPREF 0
 #endif
@@ -684,23 +688,36 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
                 reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3] = (uint32_t)n;
             }
             __syncwarp();
-            named_bar_arrive(kDescBar, 32u * (kCW + 1));
+            named_bar_arrive(kDescBar, 32u * (kCW + 1 + SPINFER_SCANDESC));
         }
+#if SPINFER_SCANDESC
+        // walk the stage descriptors (scan warp 0 wrote them above) instead of the StageIter
+        if (r != 0) named_bar_sync(kDescBar, 32u * (kCW + 2));
+        const int nst_s = (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3];
+        for (int i = 0; i < nst_s; ++i) {
+            const uint4 dv = lds_v4(sbase + prm.o_desc + 16u * (uint32_t)i);
+            const StageDesc dd{dv.x, dv.y, dv.z, dv.w};
+            const int slot = dd.slot();
+            const uint32_t spar = dd.par();
+            const struct { int rows, g; } sg = {dd.rows(), dd.g()};
+#else
         StageIter it;
         for (it.init(u0, u1, prm); it.valid(); it.next(prm)) {
             const StageIter &sg = it;
             const int i = it.i, slot = it.slot;
+            const uint32_t spar = it.par();
+#endif
             if ((dbg_mode(prm) & 4) && i > 0) break;
             // suspend (not spin) while waiting: these warps have the highest scheduling
             // priority and would otherwise steal issue slots from the consumers
             if (lane == 0) trace_ev(prm, p, i, warp, 0);
 #if SPINFER_SCANSPIN
-            mbar_wait(bar_full + 8 * slot, it.par());
+            mbar_wait(bar_full + 8 * slot, spar);
 #else
 #if SPINFER_BMBAR
-            mbar_wait_sleep(bar_bm + 8 * slot, it.par());   // the scan reads only the bitmaps
+            mbar_wait_sleep(bar_bm + 8 * slot, spar);   // the scan reads only the bitmaps
 #else
-            mbar_wait_sleep(bar_full + 8 * slot, it.par());
+            mbar_wait_sleep(bar_full + 8 * slot, spar);
 #endif
 #endif
             if (lane == 0) trace_ev(prm, p, i, warp, 1);
@@ -873,7 +890,7 @@ __global__ void __launch_bounds__(Cfg<NT>::Threads, 1) k_spmm(const __grid_const
             load_E(tb, 2 * q + 1);
         }
     };
-    named_bar_sync(kDescBar, 32u * (kCW + 1));
+    named_bar_sync(kDescBar, 32u * (kCW + 1 + SPINFER_SCANDESC));
     const int nst = (dbg_mode(prm) & 16) ? 0 : (int)reinterpret_cast<volatile uint32_t *>(smem)[kConstWord + 3];
     if (kPipe && nst > 0) begin_stage(rd(0), 0);
     // the next stage's descriptor is fetched during the current stage's decode (a shared load
