@@ -1,2 +1,3 @@
-timeout 900 python -m pytest tests -m gpu -x -q --timeout 300 2>&1 | tail -3
-BENCH_ARGS="--N 32" bash tools/ab.sh "base32:libspinfer_base.so:" "desc32:libspinfer_tcdesc.so:"
+timeout 900 python -m pytest tests -m gpu -q --timeout 300 2>&1 | tail -2
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -1
+timeout 300 python bench.py 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.readline()); print(d['us_per_spmm'], d['value'], d['roofline']['frac'], d['cublas_fp16']['us'], d['clocks'])"
