@@ -50,12 +50,21 @@ def run(env_extra, args, lib):
         return None, None
 
 
+def build_variants():
+    """The variant libraries some rows need (experiment builds of the same sources)."""
+    kq1 = os.path.join(PKG, "libspinfer_kq1.so")
+    subprocess.check_call(["bash", os.path.join(ROOT, "tools", "mkvar.sh"), "kq1", "-DSPINFER_FORCE_KQ1=1"], cwd=ROOT)
+    return kq1
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--out", default=None)
     a = ap.parse_args()
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
+    if not os.path.exists(os.path.join(PKG, "libspinfer_kq1.so")):
+        build_variants()
     res = {v[0]: [] for v in VARIANTS}
     for _ in range(a.reps):
         for tag, _, env, args, lib in VARIANTS:
