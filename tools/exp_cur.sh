@@ -1,1 +1,1 @@
-bash tools/ab.sh "base:libspinfer_base.so:" "scanspin:libspinfer_scanspin.so:" "consspin:libspinfer_consspin.so:"
+timeout 2400 python tools/ablation.py --reps 3 --out gpurun_out/r1h_ablation.jsonl > gpurun_out/ablation_r1h.txt 2>&1; cat gpurun_out/ablation_r1h.txt
