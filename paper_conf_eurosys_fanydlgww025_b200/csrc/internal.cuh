@@ -1,5 +1,6 @@
 // internal.cuh — declarations shared by the library's translation units.
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <cstdint>
 #include "spinfer.h"
@@ -19,9 +20,23 @@ int launch_encode_count(const uint16_t *W, int M, int K, int32_t *gtile_offset, 
 int launch_encode_fill(const uint16_t *W, const spinfer_tca *T, cudaStream_t st);
 int launch_decode(const spinfer_tca *T, uint16_t *W_out, cudaStream_t st);
 
+// Workspace head shared by the SpMM kernels: int32 GT-row counters [0, kErrWord) and, at word
+// kErrWord, the error word (non-zero after a call that met corrupt TCA-BME input).
+constexpr size_t kCounterRegion = 65536;
+constexpr int kErrWord = 16383;
+
 // spmm.cu
+int sm_count();                          // SMs of the current device (cached per device)
+int choose_grid(long long units);        // persistent grid size: min(SMs, units)
+int make_x_tmap(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows, bool swizzle);
+int launch_pad_x(const uint16_t *X, uint16_t *Xp, int K, int N, int Np, cudaStream_t st);
 size_t spmm_workspace_bytes(int M, int K, int N);
 int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias, int act, void *ws,
                 size_t ws_bytes, cudaStream_t st);
+
+// spmm_dw.cu (decoupled-warp kernel, N <= 16)
+size_t spmm_dw_workspace_bytes(int M, int K, int N);
+int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias,
+                   int act, void *ws, size_t ws_bytes, cudaStream_t st);
 
 }  // namespace spinfer

@@ -1745,7 +1745,7 @@ using EncodeTiledFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_
                                    const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
-int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows) {
+int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows, bool swizzle = true) {
     static EncodeTiledFn fn = nullptr;
     if (!fn) {
         void *f = nullptr;
@@ -1763,7 +1763,8 @@ int encode_x_map(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int bo
     // TMA fills with zeros (X padded to the MMA's N = 16 / 32 without a copy)
     const cuuint32_t box[2] = {(cuuint32_t)NX, (cuuint32_t)box_rows};
     const cuuint32_t estr[2] = {1u, 1u};
-    const CUtensorMapSwizzle sw = NX == 16 ? CU_TENSOR_MAP_SWIZZLE_32B : NX == 32 ? CU_TENSOR_MAP_SWIZZLE_64B
+    const CUtensorMapSwizzle sw = !swizzle ? CU_TENSOR_MAP_SWIZZLE_NONE
+                                  : NX == 16 ? CU_TENSOR_MAP_SWIZZLE_32B : NX == 32 ? CU_TENSOR_MAP_SWIZZLE_64B
                                                                                  : CU_TENSOR_MAP_SWIZZLE_NONE;
     CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, const_cast<uint16_t *>(X), dims, strides, box, estr,
                     CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
@@ -1855,8 +1856,29 @@ int launch_tc(const Plan &pl, cudaStream_t st) {
 
 }  // namespace
 
+int sm_count() {
+    static int cached[64] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) { cudaGetLastError(); return num_sms(); }
+    if (!cached[dev]) cached[dev] = num_sms();
+    return cached[dev];
+}
+int choose_grid(long long units) {
+    long long cap = sm_count();
+    if (const char *e = getenv("SPINFER_MAX_CTAS")) { long long v = atoll(e); if (v > 0 && v < cap) cap = v; }
+    return (int)std::max(1LL, std::min(cap, units));
+}
+int make_x_tmap(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows, bool swizzle) {
+    return encode_x_map(m, X, K, N, NX, box_rows, swizzle);
+}
+int launch_pad_x(const uint16_t *X, uint16_t *Xp, int K, int N, int Np, cudaStream_t st) {
+    const long long tot = (long long)K * Np;
+    k_pad_x<<<(int)std::min<long long>((tot + 255) / 256, 4096), 256, 0, st>>>(X, Xp, K, N, Np);
+    return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
+}
+
 size_t spmm_workspace_bytes(int M, int K, int N) {
-    if (M <= 0 || K <= 0 || N <= 0 || N > 32 || (M + kGT - 1) / kGT > kMaxCounters) return 0;
+    if (M <= 0 || K <= 0 || N <= 0 || N > 32 || (M + kGT - 1) / kGT >= kErrWord) return 0;
     const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;
     const long long U = (long long)((MG + kR - 1) / kR) * KG;
     const int P = choose_P(U);
@@ -1864,7 +1886,8 @@ size_t spmm_workspace_bytes(int M, int K, int N) {
     size_t part = (size_t)P * 2 * kR * 64 * Np * 4;
     size_t epi = SPINFER_AEPI ? (size_t)P * 2 * kR * 8 * 64 * Np * 4 : 0;   // asynchronous epilogue partials
     size_t xpad = (N % 8) ? align_up_sz((size_t)K * Np * 2, 256) : 0;      // zero-padded copy of X
-    return kCounterBytes + part + epi + xpad;
+    const size_t old = kCounterBytes + part + epi + xpad;
+    return std::max(old, N <= 16 ? spmm_dw_workspace_bytes(M, K, N) : (size_t)0);
 }
 
 int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias, int act,
@@ -1878,11 +1901,14 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     // copy of X in the workspace (k_pad_x) and store only the N real columns of Y
     const int Np = (N + 7) & ~7;
     const char *ke = getenv("SPINFER_KERNEL");
+    // N <= 16: the decoupled-warp kernel (spmm_dw.cu); SPINFER_KERNEL=mma keeps the round-1 kernel
+    if (Np <= 16 && !(ke && (ke[0] == 't' || ke[0] == 'm')))   // SPINFER_KERNEL=dw or unset
+        return launch_spmm_dw(T, X, Y, M, K, N, bias, act, ws, ws_bytes, st);
     bool tc = Np >= 24;
     if (ke && ke[0] == 't') tc = true;
     if (ke && ke[0] == 'm') tc = false;
     // the tcgen05 kernel's fix-up keeps one counter per rowblock and TMEM lane quarter
-    if (tc && 4LL * (((M + kGT - 1) / kGT + kR - 1) / kR) > kMaxCounters) tc = false;
+    if (tc && 4LL * (((M + kGT - 1) / kGT + kR - 1) / kR) >= kErrWord) tc = false;
     if (!make_plan(M, K, Np, T->max_gt_values, &pl, tc)) return SPINFER_EINVAL;
     const size_t need = spmm_workspace_bytes(M, K, N);
     if (need == 0) return SPINFER_EINVAL;

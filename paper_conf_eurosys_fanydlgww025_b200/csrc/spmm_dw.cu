@@ -1,0 +1,1022 @@
+// spmm_dw.cu — decoupled-warp TCA-BME SpMM Y = W x X for N <= 16 (sm_100a; §4.3,
+// P:214-301). The library's kernel for N <= 16 (the decode regime of the paper's Fig. 1 shape).
+//
+// Why this design: in the round-1 kernel all consumer warps walked the ring in
+// lockstep behind two scan warps and met at named barriers at every segment epilogue; the decode
+// ran only 69 % of the time. Here the warps are independent:
+//   * producer warp: per stage (up to G GroupTile columns x 2 GT rows) one warp instruction issues
+//     the bulk copies of both rows' bitmaps and packed values from different lanes (a thread's
+//     successive bulk copies serialise at ~310 ns each, tools/tma_sweep2.sh) plus the X slab's
+//     tensor copy, into an S-slot ring; a small per-slot header carries the per-GT value offsets
+//     (GTileOffset). The slot's empty barrier counts only the warps that own a GT of the
+//     stage (the producer pre-arrives for the rest).
+//   * 16 consumer warps: warp (r, m) owns GT row r of each rowblock and every unit u (a GT column
+//     of the CTA's stream-K range) with u % 8 == m. Every warp walks the stage sequence itself and
+//     waits only for the stages that hold its GTs. Per GroupTile it computes the PopCount base of
+//     every BitmapTile with a 32-lane shuffle scan into its own 1 KB table, then decodes
+//     the 16 TCTiles (MaskedPopCount, Alg. 2) into mma.m16n8k16 A fragments (X via
+//     ldmatrix.trans, fp32 accumulators in registers, Listing 1).
+//   * segment ends (the end of the CTA's part of a rowblock, the paper's ReductionWorkspace P:231,
+//     P:263): a consumer parks its fp32 partial in the workspace and signals the reducer warp,
+//     which sums the row's partials in warp order and writes Y (complete rowblock) or the CTA's
+//     partial; the last CTA of a split rowblock sums the CTA partials in CTA order. The CTA's
+//     final segment is reduced by the 16 consumers together through shared memory. Every sum
+//     runs in a fixed order: results do not depend on timing.
+// Corrupt or stale TCA-BME input (offsets not monotone / not 16-byte aligned / past n_values, a
+// GT with more values than a stage slot holds, bitmaps with more set bits than the GT's values)
+// never reads or writes outside the caller's buffers: the stage or GT is skipped and the
+// workspace's error word is set (include/spinfer.h).
+#include <cuda.h>
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include "internal.cuh"
+#include "ptx.cuh"
+
+namespace spinfer {
+namespace {
+
+constexpr int kRd = 2;                    // GT rows per rowblock (128 output rows)
+constexpr int kCWd = 16;                  // consumer warps: r = w >> 3, m = w & 7
+constexpr int kProdWarp0 = kCWd;          // producer warps kCWd, kCWd + 2 (SMSPs 0 and 2)
+constexpr int kNProd = 2;                 // stage i is issued by producer i % 2
+constexpr int kRedWarp = kCWd + 1;        // reducer warp (SMSP 1)
+#ifndef SPINFER_DW_PIPE
+#define SPINFER_DW_PIPE 0
+#endif
+#ifndef SPINFER_DW_REG
+#define SPINFER_DW_REG 0
+#endif
+// register split (setmaxnreg, per warpgroup of 4 warps): with 20 warps each SM sub-partition
+// holds 4 consumer warps + 1 role warp; setmaxnreg.inc is served only from what the role
+// warpgroup released, so consumers get 96 + 32 / 4 = 104
+constexpr int kRegCons = SPINFER_DW_REG ? 104 : 96, kRegRole = 64;   // pool: 16 x (104 - 96) = 4 x (96 - 64)
+constexpr int kWarpsD = kCWd + 4;         // + warp 19 (idle: completes the role warpgroup)
+constexpr int kThreadsD = 32 * kWarpsD;
+constexpr int kMaxSd = 8;
+constexpr int kMaxGd = 4;
+constexpr int kNSeg = 4;                  // segment slots between consumers and the reducer
+constexpr uint32_t kHdrBytes = 64;        // per-slot stage header: value offsets, poison flag
+constexpr uint32_t kTblBytes = 1024;      // one GroupTile's SMBD table (64 BTs x 2 halves x 8 B)
+// shared-memory map (bytes from the 1024-aligned base)
+constexpr uint32_t kBarFull = 0, kBarEmpty = 64, kBarSegFull = 128, kBarSegFree = 192, kSegMask = 224;
+#ifndef SPINFER_DW_XTMA
+#define SPINFER_DW_XTMA 1
+#endif
+// X slab: tensor copy with the 32B swizzle (conflict-free ldmatrix) or a plain bulk copy issued
+// with the stage's other copies (2-way bank conflicts on the ldmatrix reads)
+constexpr bool kXTma = SPINFER_DW_XTMA != 0;
+constexpr uint32_t kHdrStop = 1u << 16, kHdrBad = 1u << 17;   // header word 1: g | rows << 8 | flags
+constexpr uint32_t kOffHdr = 1024;
+constexpr uint32_t kOffTbl = kOffHdr + kMaxSd * kHdrBytes;   // per-warp SMBD tables
+constexpr uint32_t kOffRing = (kOffTbl + kCWd * kTblBytes + 1023) / 1024 * 1024;
+
+struct DParams {
+    CUtensorMap tmap_x;           // X [K][Np] fp16, box {Np, 64 G}, no swizzle (ragged-K tail stages only)
+    const int32_t *off;
+    const uint64_t *bm;
+    const uint16_t *vals;
+    const uint16_t *X;            // X [K][Np] fp16 (or its zero-padded copy), the bulk-copy source
+    uint16_t *Y;
+    const uint16_t *bias;         // fused epilogue: fp16 [M] or null
+    int act;
+    float *ws_seg;                // [P][kNSeg][2][8] warp partials (m16n8k16 D layout), 64 x Np fp32 each
+    float *ws_cta;                // [MG][cslots] CTA partials of split rowblocks (row-major 64 x Np)
+    int32_t *ws_cnt;              // [MG] CTA counters of split rowblocks (zero between calls)
+    int32_t *ws_err;              // error word (non-zero: corrupt TCA-BME input was skipped)
+    int KG, MG, M, N, K;
+    int n_values;                 // values[] length: value ranges past it are rejected
+    uint32_t U;                   // units = rowblocks x KG; U * P < 2^32
+    int P, G, S;
+    int cslots;                   // CTA partial slots per GT row (max CTAs one rowblock overlaps)
+    uint32_t slot_bytes, st_bm, st_v0, st_v1, vcap;   // slot: X slab | bitmaps | values row 0 | row 1
+    float avg_gt;                 // n_values / NGT (start-up page prefetch hint)
+    long long *prof;              // experiments only (SPINFER_INSTRUMENT)
+};
+
+#ifndef SPINFER_INSTRUMENT
+#define SPINFER_INSTRUMENT 0
+#endif
+// Per-warp cycle accounting (instrumented build only): consumers k0 waiting for data, k1 scan,
+// k2 decode, k3 segment hand-off, k4 GTs decoded, k5 first data seen, k6 exit, k7 other;
+// producer k0 waiting for a free slot, k1 issuing; reducer k0 waiting, k1 reducing.
+constexpr int kProfW = 20;
+constexpr size_t kTraceOff = 1024 * kProfW * 8;   // stage trace of CTA 0 after the counters
+constexpr size_t kEvOff = kTraceOff + 256 * 4;      // per-warp event trace of CTA 0: [16 warps][64 stages][6]
+struct Prof {
+#if SPINFER_INSTRUMENT
+    long long c[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    long long t = 0, t0 = 0;
+    __device__ __forceinline__ void start() { t0 = t = clock64(); }
+    __device__ __forceinline__ void lap(int k) { const long long n = clock64(); c[k] += n - t; t = n; }
+    __device__ __forceinline__ void mark(int k) { c[k] = clock64() - t0; }
+    __device__ __forceinline__ void count(int k) { ++c[k]; }
+    __device__ __forceinline__ void dump(long long *prof, int p, int w, int lane) {
+        if (prof && lane == 0 && p < 1024)
+            for (int k = 0; k < 8; ++k) prof[((size_t)p * kProfW + w) * 8 + k] = c[k];
+    }
+    // CTA 0 stage trace: [i][k] k0 producer issue, k1 first owner wake (min), k2 last release, k3 producer wait start
+    __device__ __forceinline__ void st(long long *prof, int p, int i, int k, bool mx) {
+        if (!prof || p != 0 || i >= 256) return;
+        unsigned long long *q = reinterpret_cast<unsigned long long *>(prof) + kTraceOff + (size_t)i * 4 + k;
+        const unsigned long long v = (unsigned long long)(clock64() - t0 + 1);
+        atomicMax(q, mx ? v : ~v);   // min fields hold the complement
+    }
+    __device__ __forceinline__ void ev(long long *prof, int p, int w, int i, int k) {
+        if (prof && p == 0 && w < 16 && i < 64) prof[kEvOff + ((size_t)w * 64 + i) * 6 + k] = clock64() - t0;
+    }
+#else
+    __device__ __forceinline__ void ev(long long *, int, int, int, int) {}
+    __device__ __forceinline__ void start() {}
+    __device__ __forceinline__ void lap(int) {}
+    __device__ __forceinline__ void mark(int) {}
+    __device__ __forceinline__ void count(int) {}
+    __device__ __forceinline__ void dump(long long *, int, int, int) {}
+    __device__ __forceinline__ void st(long long *, int, int, int, bool) {}
+#endif
+};
+
+__device__ __forceinline__ int ustart(int p, uint32_t U, int P) { return (int)((uint32_t)p * U / (uint32_t)P); }
+__device__ __forceinline__ int uowner(int u, uint32_t U, int P) { return (int)(((uint32_t)(u + 1) * (uint32_t)P - 1u) / U); }
+
+// The CTA's stage walk (every warp runs its own copy). A CTA's unit range [u0, u1) runs in the
+// order A = tail of the rowblock it starts inside (split with CTA p-1), C = head of the rowblock
+// it ends inside (split with CTA p+1), then the full rowblocks: split rowblocks finish early, so
+// their cross-CTA sums do not trail the kernel. A stage = up to G consecutive units of one
+// rowblock; a segment = the stages of one part inside one rowblock.
+struct Stages {
+    int u, ue, us;
+    int ns0, ne0, ns1, ne1;
+    int rb, gc, g, rows;
+    __device__ __forceinline__ void init(int u0, int u1, int KG, int G, int MG) {
+        const int a_end = (u0 % KG) ? min(u1, (u0 / KG + 1) * KG) : u0;
+        const int c_beg = (u1 % KG) ? max(a_end, (u1 / KG) * KG) : u1;
+        int q0s = u1, q0e = u1, q1s = u1, q1e = u1, q2s = u1, q2e = u1, k = 0;
+        auto push = [&](int s_, int e_) {
+            if (s_ >= e_) return;
+            if (k == 0) { q0s = s_; q0e = e_; } else if (k == 1) { q1s = s_; q1e = e_; } else { q2s = s_; q2e = e_; }
+            ++k;
+        };
+        push(u0, a_end);
+        push(c_beg, u1);
+        push(a_end, c_beg);
+        ns0 = q1s; ne0 = q1e; ns1 = q2s; ne1 = q2e;
+        part(q0s, q0e, KG, G, MG);
+    }
+    __device__ __forceinline__ void part(int s0, int e0, int KG, int G, int MG) {
+        u = s0; us = s0; ue = e0;
+        rb = (int)((uint32_t)u / (uint32_t)KG);
+        gc = u - rb * KG;
+        shape(KG, G, MG);
+    }
+    __device__ __forceinline__ void shape(int KG, int G, int MG) {
+        g = min(min(G, KG - gc), ue - u);
+        rows = min(kRd, MG - kRd * rb);
+    }
+    __device__ __forceinline__ bool valid() const { return u < ue; }
+    __device__ __forceinline__ bool seg_first() const { return u == us || gc == 0; }
+    __device__ __forceinline__ bool seg_last(int KG) const { return gc + g == KG || u + g == ue; }
+    __device__ __forceinline__ void next(int KG, int G, int MG) {
+        u += g;
+        gc += g;
+        if (gc == KG) { gc = 0; ++rb; }
+        if (u == ue && ns0 < ne0) {
+            const int s0 = ns0, e0 = ne0;
+            ns0 = ns1; ne0 = ne1; ns1 = ne1;
+            part(s0, e0, KG, G, MG);
+        } else {
+            shape(KG, G, MG);
+        }
+    }
+};
+
+// SMBD selector: PRMT of the two zero-extended u16 loads {V[c2-2], V[c2-1]} with selector
+// y (kSelA + kSelB y) + kSelC for the lane's bit pair y (found by exhaustive search,
+// tools/selector_search.py; pinned in tests/test_host_logic.py).
+constexpr uint32_t kSelA = 0x7f62u, kSelB = 0x4cbfu, kSelC = 0x2333u;
+
+__device__ __forceinline__ float epi_act(float v, float b, int act) {
+    v += b;
+    return act == SPINFER_ACT_RELU ? fmaxf(v, 0.f) : v;
+}
+
+// Y rows [row_base, row_base + 64) from accumulators in the m16n8k16 D layout. EPI: fused
+// bias/activation, padding rows of a ragged M (A8), N not a multiple of 8.
+template <int NT, bool EPI>
+__device__ __forceinline__ void store_frag(const DParams &prm, int row_base, float (&acc)[4][NT][4], int lane) {
+    uint16_t *const Y = prm.Y;
+    const int N = prm.N;
+#pragma unroll
+    for (int tr = 0; tr < 4; ++tr) {
+        const int r0 = row_base + tr * 16 + (lane >> 2);
+        if (EPI && (prm.bias || prm.act)) {
+            // rows past M (padding of a ragged M) read no bias
+            const float b0 = (prm.bias && r0 < prm.M) ? __half2float(__ushort_as_half(prm.bias[r0])) : 0.f;
+            const float b1 = (prm.bias && r0 + 8 < prm.M) ? __half2float(__ushort_as_half(prm.bias[r0 + 8])) : 0.f;
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) {
+                acc[tr][nt][0] = epi_act(acc[tr][nt][0], b0, prm.act);
+                acc[tr][nt][1] = epi_act(acc[tr][nt][1], b0, prm.act);
+                acc[tr][nt][2] = epi_act(acc[tr][nt][2], b1, prm.act);
+                acc[tr][nt][3] = epi_act(acc[tr][nt][3], b1, prm.act);
+            }
+        }
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt) {
+            const int col = nt * 8 + 2 * (lane & 3);
+            const __half2 lo = __floats2half2_rn(acc[tr][nt][0], acc[tr][nt][1]);   // one RNE per output (A11)
+            const __half2 hi = __floats2half2_rn(acc[tr][nt][2], acc[tr][nt][3]);
+            if (!EPI) {
+                *reinterpret_cast<__half2 *>(Y + (size_t)r0 * N + col) = lo;
+                *reinterpret_cast<__half2 *>(Y + (size_t)(r0 + 8) * N + col) = hi;
+            } else {
+                __half *y0 = reinterpret_cast<__half *>(Y + (size_t)r0 * N);
+                __half *y1 = reinterpret_cast<__half *>(Y + (size_t)(r0 + 8) * N);
+                const bool v0 = r0 < prm.M, v1 = r0 + 8 < prm.M;
+                if (N == NT * 8 && v0) *reinterpret_cast<__half2 *>(y0 + col) = lo;
+                if (N == NT * 8 && v1) *reinterpret_cast<__half2 *>(y1 + col) = hi;
+                if (N != NT * 8) {
+                    if (v0 && col < N) y0[col] = __low2half(lo);
+                    if (v0 && col + 1 < N) y0[col + 1] = __high2half(lo);
+                    if (v1 && col < N) y1[col] = __low2half(hi);
+                    if (v1 && col + 1 < N) y1[col + 1] = __high2half(hi);
+                }
+            }
+        }
+    }
+}
+
+// NC consecutive outputs Y[row][col0 .. col0 + NC) (NC = 2 or 4, col0 a multiple of NC).
+template <int NT, bool EPI, int NC>
+__device__ __forceinline__ void store_cols(const DParams &prm, int row, int col0, const float (&v)[NC]) {
+    const int N = prm.N;
+    if (EPI && row >= prm.M) return;   // padding row of a ragged M (A8)
+    float w[NC];
+    const float b = (EPI && prm.bias) ? __half2float(__ushort_as_half(prm.bias[row])) : 0.f;
+#pragma unroll
+    for (int c = 0; c < NC; ++c) w[c] = EPI ? epi_act(v[c], b, prm.act) : v[c];
+    __half *y = reinterpret_cast<__half *>(prm.Y + (size_t)row * N);
+    if (!EPI || N == NT * 8) {
+        if constexpr (NC == 4) {
+            const __half2 a = __floats2half2_rn(w[0], w[1]), c2 = __floats2half2_rn(w[2], w[3]);
+            uint2 u;
+            u.x = *reinterpret_cast<const uint32_t *>(&a);
+            u.y = *reinterpret_cast<const uint32_t *>(&c2);
+            *reinterpret_cast<uint2 *>(y + col0) = u;
+        } else {
+            *reinterpret_cast<__half2 *>(y + col0) = __floats2half2_rn(w[0], w[1]);
+        }
+    } else {
+#pragma unroll
+        for (int c = 0; c < NC; ++c)
+            if (col0 + c < N) y[col0 + c] = __float2half_rn(w[c]);
+    }
+}
+
+__device__ __forceinline__ void stg_f4(float4 *p, float4 v) {
+    asm volatile("st.global.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w) : "memory");
+}
+__device__ __forceinline__ void stg_f2(float *p, float x, float y) {
+    asm volatile("st.global.v2.f32 [%0], {%1, %2};" ::"l"(p), "f"(x), "f"(y) : "memory");
+}
+__device__ __forceinline__ float4 ldg_cg4(const float4 *p) {
+    float4 v;
+    asm volatile("ld.global.cg.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p)
+                 : "memory");
+    return v;
+}
+// Drop an L2 line without writing it back: every partial is read exactly once.
+__device__ __forceinline__ void discard_l2(const void *p) {
+    asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_cnt(uint32_t bar, uint32_t n) {
+    asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0], %1;\n\t}" ::"r"(bar), "r"(n) : "memory");
+}
+
+// The CTA partial of GT row `grow` (row-major 64 x Np fp32) is parked; count the CTA and, as the
+// last of the CTAs overlapping the rowblock, sum all CTA partials in CTA order and write Y.
+// Called by one whole warp after every lane's stores are ordered before it (syncwarp/barrier).
+template <int NT, bool EPI>
+__device__ __forceinline__ void cta_count_and_sum(const DParams &prm, int rb, int grow, int lane) {
+    constexpr int Np = NT * 8, kF4 = 64 * Np / 4;
+    const int pf = uowner(rb * prm.KG, prm.U, prm.P), pl = uowner((rb + 1) * prm.KG - 1, prm.U, prm.P);
+    __threadfence();
+    int old = 0;
+    if (lane == 0) old = atomicAdd(prm.ws_cnt + grow, 1);
+    old = __shfl_sync(0xffffffffu, old, 0);
+    if (old != pl - pf) return;
+    __threadfence();   // acquire: every CTA partial is visible
+    const float4 *base = reinterpret_cast<const float4 *>(prm.ws_cta) + (size_t)grow * prm.cslots * kF4;
+    constexpr int kPer = kF4 / 32;   // float4 per lane
+    float4 s[kPer];
+#pragma unroll
+    for (int t = 0; t < kPer; ++t) s[t] = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int q = 0; q <= pl - pf; ++q) {
+#pragma unroll
+        for (int t = 0; t < kPer; ++t) {
+            const float4 v = ldg_cg4(base + (size_t)q * kF4 + t * 32 + lane);
+            s[t].x += v.x; s[t].y += v.y; s[t].z += v.z; s[t].w += v.w;
+        }
+    }
+#pragma unroll
+    for (int t = 0; t < kPer; ++t) {
+        const int e = 4 * (t * 32 + lane);   // element index in the row-major 64 x Np block
+        const float v[4] = {s[t].x, s[t].y, s[t].z, s[t].w};
+        store_cols<NT, EPI, 4>(prm, grow * 64 + e / Np, e % Np, v);
+    }
+    for (int q = 0; q <= pl - pf; ++q)
+        if (lane < kF4 / 8) discard_l2(base + (size_t)q * kF4 + 8 * lane);
+    if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed for the next call
+}
+
+template <int NT, bool EPI>
+__global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant__ DParams prm) {
+    constexpr int Np = NT * 8;
+    constexpr int kF4 = 64 * Np / 4;   // float4 per 64 x Np partial
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *const smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+    const uint32_t sbase = smem_u32(smem);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int p = blockIdx.x;
+    const int KG = prm.KG, G = prm.G, S = prm.S, MG = prm.MG;
+    const uint32_t bar_full = sbase + kBarFull, bar_empty = sbase + kBarEmpty;
+    const uint32_t bar_sfull = sbase + kBarSegFull, bar_sfree = sbase + kBarSegFree;
+    const uint32_t seg_mask = sbase + kSegMask;
+    const uint32_t ring = sbase + kOffRing;
+    const int u0 = ustart(p, prm.U, prm.P), u1 = ustart(p + 1, prm.U, prm.P);
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(bar_full + 8 * s, 1);              // the producer's arrive.expect_tx (+ TMA bytes)
+            mbar_init(bar_empty + 8 * s, kRd * kMaxGd);  // the stage's GT owners + the producer's pre-arrival
+        }
+        for (int k = 0; k < kNSeg; ++k) {
+            mbar_init(bar_sfull + 16 * k, 8);             // row 0: its 8 consumer warps
+            mbar_init(bar_sfull + 16 * k + 8, 8);         // row 1
+            mbar_init(bar_sfree + 8 * k, 1);              // the reducer has read the slot
+            sts_u32(seg_mask + 8 * k, 0u);
+            sts_u32(seg_mask + 8 * k + 4, 0u);
+        }
+        fence_barrier_init();
+    }
+    __syncthreads();
+    Prof pf;
+    pf.start();
+    // role warps (warpgroup 4): give registers back, then split into producers / reducer / idle.
+    // Each branch below ends in a return, so ptxas compiles each region for its own budget.
+    if (warp >= kCWd) {
+#if SPINFER_DW_REG
+    setmaxnreg_dec<kRegRole>();
+#endif
+    if (warp == kCWd + 3) return;   // the idle warp (completes the warpgroup)
+
+    if (warp == kProdWarp0 || warp == kProdWarp0 + 2) {
+        // ------------------------------------------------------------------ producers (2 warps)
+        // Producer q issues the stages i with i % 2 == q. Lanes 0-4 / 8-12 hold the GTileOffset
+        // entries j = 0..4 of GT row 0 / 1 of a stage, loaded two own stages ahead with one load
+        // instruction. All of a stage's copies go out in ONE bulk-copy instruction from different
+        // lanes (lane 0 / 8: packed values of row 0 / 1, lane 1: the X slab, lanes 2, 3: the
+        // bitmaps of rows 0, 1): a thread's successive bulk copies serialise at ~310 ns each
+        // (tools/tma_sweep2.sh: 4 KB chunks from one thread 1.97 TB/s, 8 lanes x 4 KB per
+        // instruction 5.7 TB/s).
+        const int q = (warp - kProdWarp0) >> 1;
+        const int orow = lane >> 3, oj = lane & 7;
+        if (lane == 0) prefetch_tmap(&prm.tmap_x);
+        Stages it;
+        it.init(u0, u1, KG, G, MG);
+        int nseg = 0, i = 0;
+        uint32_t pslot = 0, pph = 0;   // ring position of stage i
+        auto step = [&](Stages &s, int &ns, int &ii) {   // one stage forward (segment count, index)
+            if (s.seg_last(KG)) ++ns;
+            s.next(KG, G, MG);
+            ++ii;
+        };
+        if (q == 1 && it.valid()) { step(it, nseg, i); pslot = 1; }
+        Stages ia = it;   // two own stages ahead of `it`: the offset prefetch
+        int nsa = nseg, ia_i = i;
+        // start-up: touch the predicted first value line of each GT row (page translation
+        // overlaps the GTileOffset loads the first copies wait for; a hint only)
+        if (it.valid() && lane < it.rows)
+            prefetch_l2(prm.vals + (long long)((double)((long long)(kRd * it.rb + lane) * KG + it.gc) * prm.avg_gt));
+        auto ld_off = [&](const Stages &sg) -> int {
+            return (sg.valid() && orow < sg.rows && oj <= sg.g)
+                       ? __ldg(prm.off + (long long)(kRd * sg.rb + orow) * KG + sg.gc + oj) : 0;
+        };
+        auto skip2 = [&](Stages &s, int &ns, int &ii) {
+            for (int k = 0; k < kNProd && s.valid(); ++k) step(s, ns, ii);
+        };
+        int oc = ld_off(ia);
+        skip2(ia, nsa, ia_i);
+        int on = ld_off(ia);
+        skip2(ia, nsa, ia_i);
+
+        const uint64_t pol = policy_evict_first();
+        while (it.valid()) {
+            const uint32_t slot = pslot, ph = pph;
+            pf.lap(1);
+            if (lane == 0) pf.st(prm.prof, p, i, 3, true);
+            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, ph ^ 1u);
+            pf.lap(0);
+            if (lane == 0) pf.st(prm.prof, p, i, 0, true);
+            const uint32_t st = ring + slot * prm.slot_bytes, fb = bar_full + 8 * slot;
+            const uint32_t hb = sbase + kOffHdr + slot * kHdrBytes;
+            const int g = it.g, rows = it.rows;
+            // validate the stage's value ranges (never trust the caller's max_gt_values)
+            const int obeg = __shfl_sync(0xffffffffu, oc, lane & 8);
+            const int oend = __shfl_sync(0xffffffffu, oc, (lane & 8) + g);
+            const int onxt = __shfl_down_sync(0xffffffffu, oc, 1);
+            bool badl = false;
+            if (orow < rows && oj < g) badl = onxt < oc;
+            if (orow < rows && oj == 0)
+                badl |= (oc & 7) != 0 || oc < 0 || oend > prm.n_values || 2LL * (oend - oc) > (long long)prm.vcap;
+            const uint32_t badm = __ballot_sync(0xffffffffu, badl);   // lanes 0-7: row 0, 8-15: row 1
+            const bool bad0 = (badm & 0xFFu) != 0, bad1 = (badm & 0xFF00u) != 0;
+            const bool bad = orow ? bad1 : bad0;
+            pf.lap(2);
+            // header: stage shape, segment index, per-GT value offsets (bytes from the row's value region)
+            if (orow < kRd && oj <= kMaxGd) sts_u32(hb + 16u + 20u * orow + 4u * oj, 2u * (uint32_t)(oc - obeg));
+            if (lane == 31)
+                sts_v4(hb, make_uint4((uint32_t)it.rb, (uint32_t)g | ((uint32_t)rows << 8) | ((bad0 || bad1) ? kHdrBad : 0u),
+                                      (uint32_t)nseg, 0u));
+            const uint32_t vbl = (oj == 0 && orow < rows && !bad) ? 2u * (uint32_t)(oend - oc) : 0u;   // lanes 0, 8
+            const uint32_t vb1 = __shfl_sync(0xffffffffu, vbl, 8);
+            // the X slab: a plain bulk copy of g GT columns, or (ragged K, last column) the tensor
+            // copy that zero-fills the rows past K
+            const bool xt = kXTma || (it.gc + g) * 64 > prm.K;
+            const uint32_t xbytes = xt ? (uint32_t)G * 64u * Np * 2u : (uint32_t)g * 64u * Np * 2u;
+            const uint32_t bmb = (uint32_t)g * 512u;
+            __syncwarp();
+            if (lane == 0) {
+                if (badm) atomicOr(prm.ws_err, 1);
+                // one arrival with every transaction byte registered up front: the phase completes
+                // only when all copies of the stage have landed (release: the header stores above)
+                mbar_arrive_expect_tx(fb, (uint32_t)rows * bmb + xbytes + vbl + vb1);
+                // the empty barrier expects kRd * kMaxGd arrivals: one per GT owner of the stage, the rest now
+                const uint32_t owners = (uint32_t)(rows * g);
+                if (owners < (uint32_t)(kRd * kMaxGd)) mbar_arrive_cnt(bar_empty + 8 * slot, (uint32_t)(kRd * kMaxGd) - owners);
+            }
+            pf.lap(3);
+            uint32_t dst = 0, bytes = 0;
+            const void *src = nullptr;
+            if (oj == 0) {                                  // lanes 0, 8: packed values of row orow
+                dst = st + (orow ? prm.st_v1 : prm.st_v0); src = prm.vals + oc; bytes = vbl;
+            } else if (lane == 1 && !xt) {                  // X rows [64 gc, 64 (gc + g))
+                dst = st; src = prm.X + (size_t)64 * it.gc * Np; bytes = xbytes;
+            } else if (lane == 2 || lane == 3) {            // bitmaps of row lane - 2
+                const int r = lane - 2;
+                dst = st + prm.st_bm + (uint32_t)(r * G) * 512u;
+                src = prm.bm + ((size_t)(kRd * it.rb + r) * KG + it.gc) * 64;
+                bytes = r < rows ? bmb : 0u;
+            }
+            if (bytes) bulk_g2s(dst, src, bytes, fb, pol);
+            if (xt && lane == 1) tma_2d_g2s(st, &prm.tmap_x, 0, 64 * it.gc, fb);
+            pf.lap(4);
+
+            skip2(it, nseg, i);
+            pslot += 2;
+            if (pslot >= (uint32_t)S) { pslot -= (uint32_t)S; pph ^= 1u; }
+            oc = on;
+            on = ld_off(ia);   // two own stages ahead: in flight while this warp issues the next stages
+            skip2(ia, nsa, ia_i);
+            pf.lap(5);
+        }
+        // stop sentinel in the slot of the first stage index >= the stage count with this parity;
+        // its header carries the CTA's segment count
+        {
+            if ((i & 1) != q) ++i;   // the loop can stop one index short of this producer's parity
+            const uint32_t slot = (uint32_t)(i % S), ph = (uint32_t)(i / S) & 1u;
+            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, ph ^ 1u);
+            if (lane == 0) {
+                sts_v4(sbase + kOffHdr + slot * kHdrBytes, make_uint4(0u, kHdrStop, (uint32_t)nseg, 0u));
+                mbar_arrive(bar_full + 8 * slot);
+            }
+        }
+        pf.mark(6);
+        pf.dump(prm.prof, p, warp, lane);
+        return;
+    }
+
+    if (warp == kRedWarp) {
+        // ------------------------------------------------------------------ reducer (one warp)
+        // Non-final segments of the CTA, in order: sum the GT row's warp partials (warp order),
+        // then write Y (the CTA holds the whole rowblock) or park the CTA partial for the
+        // cross-CTA sum.
+        Stages it;
+        it.init(u0, u1, KG, G, MG);
+        int nseg = 0, sstart = 0;
+        while (it.valid()) {
+            if (it.seg_first()) sstart = it.u;
+            const bool seg_end = it.seg_last(KG);
+            const int rb = it.rb, rows = it.rows, send = it.u + it.g;
+            it.next(KG, G, MG);
+            if (!seg_end) continue;
+            if (!it.valid()) break;   // the final segment: the consumers reduce it in shared memory
+            const int k = nseg % kNSeg;
+            const uint32_t par = (uint32_t)(nseg / kNSeg) & 1u;
+            const bool complete = sstart == rb * KG && send == (rb + 1) * KG;
+            for (int r = 0; r < rows; ++r) {
+                pf.lap(1);
+                mbar_wait_sleep(bar_sfull + 16 * k + 8 * r, par);
+                pf.lap(0);
+                const uint32_t cmask = lds_u32(seg_mask + 8 * k + 4 * r);   // warps that own a GT of the segment
+                if (lane == 0) sts_u32(seg_mask + 8 * k + 4 * r, 0u);
+                const float4 *src = reinterpret_cast<const float4 *>(prm.ws_seg) + ((((size_t)p * kNSeg + k) * kRd + r) * 8) * kF4;
+                float acc[4][NT][4];
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+#pragma unroll
+                    for (int b = 0; b < NT; ++b)
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
+                for (int m = 0; m < 8; ++m) {
+                    if (!((cmask >> m) & 1u)) continue;
+#pragma unroll
+                    for (int tr = 0; tr < 4; ++tr) {
+                        float4 v[NT];
+#pragma unroll
+                        for (int nt = 0; nt < NT; ++nt) v[nt] = ldg_cg4(src + (size_t)m * kF4 + (tr * NT + nt) * 32 + lane);
+#pragma unroll
+                        for (int nt = 0; nt < NT; ++nt) {
+                            const float4 w = v[nt];
+                            acc[tr][nt][0] += w.x; acc[tr][nt][1] += w.y; acc[tr][nt][2] += w.z; acc[tr][nt][3] += w.w;
+                        }
+                    }
+                }
+                for (int m = 0; m < 8; ++m)
+                    if (((cmask >> m) & 1u) && lane < kF4 / 8) discard_l2(src + (size_t)m * kF4 + 8 * lane);
+                const int grow = kRd * rb + r;
+                if (complete) {
+                    store_frag<NT, EPI>(prm, grow * 64, acc, lane);
+                } else {
+                    const int pfirst = uowner(rb * KG, prm.U, prm.P);
+                    float *dst = prm.ws_cta + ((size_t)grow * prm.cslots + (p - pfirst)) * (64 * Np);
+#pragma unroll
+                    for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                        for (int nt = 0; nt < NT; ++nt) {
+                            const int row = tr * 16 + (lane >> 2), col = nt * 8 + 2 * (lane & 3);
+                            stg_f2(dst + row * Np + col, acc[tr][nt][0], acc[tr][nt][1]);
+                            stg_f2(dst + (row + 8) * Np + col, acc[tr][nt][2], acc[tr][nt][3]);
+                        }
+                    __syncwarp();
+                    cta_count_and_sum<NT, EPI>(prm, rb, grow, lane);
+                }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar_sfree + 8 * k);   // the slot's partials may be overwritten
+            ++nseg;
+        }
+        pf.lap(1);
+        pf.mark(6);
+        pf.dump(prm.prof, p, warp, lane);
+        return;
+    }
+
+    }   // role warps
+#if SPINFER_DW_REG
+    setmaxnreg_inc<kRegCons>();
+#endif
+
+    // ---------------------------------------------------------------------- consumers
+    // Warp (r, m) owns GT j = m % 4 of GT row r in every stage i with i % 2 == m / 4; it reads the
+    // stage's shape and segment index from the slot header.
+    const int r = warp >> 3, m = warp & 7, jw = m & 3;
+    const uint32_t mulc = opaque_u32(1u << (30u - 2u * (uint32_t)(lane & 15)));   // z = w << (30 - sh) on the FMA pipe
+    const uint32_t selA = opaque_u32(kSelA), selB = opaque_u32(kSelB), selC = opaque_u32(kSelC);
+    constexpr uint32_t cpr = Np / 8;   // 16-byte chunks per X row
+    const uint32_t rr = lane & 7, mk = (lane >> 3) & 1, mn = (lane >> 4) & 1;
+    // X slab row-major; with the tensor copy the 32B swizzle XORs the 16-byte chunk with row bit 2
+    const uint32_t x_lane = (mk * 8u + rr) * cpr * 16u + ((mn ^ (kXTma && NT == 2 ? (rr >> 2) & 1u : 0u)) * 16u);
+    float acc[4][NT][4];
+#pragma unroll
+    for (int a = 0; a < 4; ++a)
+#pragma unroll
+        for (int b = 0; b < NT; ++b)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
+
+    uint4 E[4];
+    auto load_E = [&](uint32_t tb) {   // entries of 8 consecutive BTs, this lane's half
+#pragma unroll
+        for (int k = 0; k < 4; ++k) E[k] = lds_v4(tb + 16u * k);
+    };
+    auto issue_to = [&](uint32_t (&u0)[8], uint32_t (&u1)[8], uint32_t (&sl)[8]) {   // SMBD value loads into a set
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
+            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;
+            const uint32_t z = w * mulc;
+            const uint32_t a = A + 2u * __popc(z);
+            const uint32_t y = z >> 30;
+            sl[k] = y * (y * selB + selA) + selC;
+            u0[k] = lds_u16(a);
+            u1[k] = lds_u16(a + 2u);
+        }
+    };
+    auto assemble_from = [&](const uint32_t (&u0)[8], const uint32_t (&u1)[8], const uint32_t (&sl)[8], int trb,
+                             const uint32_t (&bfr)[NT][2]) {
+#pragma unroll
+        for (int tt = 0; tt < 2; ++tt) {
+            uint32_t afr[4];
+#pragma unroll
+            for (int b = 0; b < 4; ++b) afr[b] = prmt(u0[tt * 4 + b], u1[tt * 4 + b], sl[tt * 4 + b]);
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) mma_16816(acc[trb + tt][nt], afr, bfr[nt][0], bfr[nt][1]);
+        }
+    };
+    // segment hand-off to the reducer (non-final segments): park the partial if this warp owned a
+    // GT of the segment, then arrive; `own` = false arrives for a segment without a GT of this warp
+    auto seg_close = [&](int sg, bool own) {
+        const int k = sg % kNSeg;
+        if (sg >= kNSeg) mbar_wait_sleep(bar_sfree + 8 * k, (uint32_t)((sg / kNSeg) - 1) & 1u);
+        if (own) {
+            float4 *dst = reinterpret_cast<float4 *>(prm.ws_seg) + ((((size_t)p * kNSeg + k) * kRd + r) * 8 + m) * kF4;
+#pragma unroll
+            for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                for (int nt = 0; nt < NT; ++nt)
+                    stg_f4(dst + (tr * NT + nt) * 32 + lane, make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]));
+            if (lane == 0) atomicOr(reinterpret_cast<uint32_t *>(smem + kSegMask + 8 * k + 4 * r), 1u << m);
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(bar_sfull + 16 * k + 8 * r);   // release: the stores above
+    };
+
+    const uint32_t tbl = sbase + kOffTbl + (uint32_t)warp * kTblBytes;
+    const uint32_t tbl_lane = tbl + (uint32_t)(lane >> 4) * 512u;
+    // PopCount bases of a GT's 64 BitmapTiles into the table at `tb`: lane l pops BTs l and
+    // l + 32, one 32-lane shuffle scan; false if the GT is poisoned or its bitmaps hold more set
+    // bits than its value range (corrupt input: never read past the stage's values)
+    auto scan_gt = [&](uint32_t st_, uint32_t voff_, uint32_t vend_, uint2 ba_, uint2 bb_, uint32_t flags_,
+                       uint32_t tb) -> bool {
+        const uint32_t vsm = st_ + (r ? prm.st_v1 : prm.st_v0) + voff_;
+        const uint32_t pax = __popc(ba_.x), pbx = __popc(bb_.x);
+        const uint32_t packed = (pax + __popc(ba_.y)) | ((pbx + __popc(bb_.y)) << 16);
+        uint32_t incl = packed;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+            incl += (lane >= o) ? y : 0u;
+        }
+        const uint32_t tot = __shfl_sync(0xffffffffu, incl, 31);
+        const uint32_t tot_a = tot & 0xFFFFu;
+        if ((flags_ & kHdrBad) || 2u * (tot_a + (tot >> 16)) > vend_ - voff_) return false;
+        const uint32_t excl = incl - packed;
+        const uint32_t Aa = vsm + 2u * (excl & 0xFFFFu) - 4u;
+        const uint32_t Ab = vsm + 2u * (tot_a + (excl >> 16)) - 4u;
+        const uint32_t te = tb + 8u * lane;
+        sts_v2(te, ba_.x, Aa);
+        sts_v2(te + 512u, ba_.y, Aa + 2u * pax);
+        sts_v2(te + 256u, bb_.x, Ab);
+        sts_v2(te + 768u, bb_.y, Ab + 2u * pbx);
+        __syncwarp();
+        return true;
+    };
+
+    int i = m >> 2;                 // stage index
+    uint32_t slot = (uint32_t)(i % S), ph = 0;   // ring position of stage i (S >= 2)
+    int cur = -1;                   // open segment of this warp (-1: none)
+    bool contrib = false, seen = false;
+    int nseg_total = 0, f_rb = 0, f_rows = 0;
+    while (true) {
+        pf.lap(7);
+        if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 0);
+        mbar_wait_sleep(bar_full + 8 * slot, ph);
+        if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 1);
+        if (!seen) { seen = true; pf.mark(5); }
+        pf.lap(0);
+        if (lane == 0) pf.st(prm.prof, p, i, 1, false);
+        const uint32_t hb = sbase + kOffHdr + slot * kHdrBytes;
+        const uint32_t st = ring + slot * prm.slot_bytes;
+        // everything this stage needs from shared memory, in one round trip: header, this GT's
+        // value range, its 64 bitmaps (lane l: BTs l and l + 32)
+        const uint4 h = lds_v4(hb);
+        const uint32_t voff = lds_u32(hb + 16u + 20u * (uint32_t)r + 4u * (uint32_t)jw);
+        const uint32_t vend = lds_u32(hb + 20u + 20u * (uint32_t)r + 4u * (uint32_t)jw);
+        const uint32_t bms = st + prm.st_bm + (uint32_t)(r * G + jw) * 512u;
+        const uint2 ba = lds_v2(bms + 8u * lane), bb = lds_v2(bms + 256u + 8u * lane);
+        if (h.y & kHdrStop) { nseg_total = (int)h.z; break; }
+        const int sg = (int)h.z, g = (int)(h.y & 0xFFu), rows = (int)((h.y >> 8) & 3u);
+        if (sg != cur) {   // this stage opens a new segment
+            if (cur >= 0 && r < f_rows) seg_close(cur, contrib);
+            for (int s2 = cur + 1; s2 < sg; ++s2) seg_close(s2, false);   // segments with no stage of this parity
+            cur = sg;
+#pragma unroll
+            for (int a = 0; a < 4; ++a)
+#pragma unroll
+                for (int b = 0; b < NT; ++b)
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
+            contrib = false;
+        }
+        f_rb = (int)h.x; f_rows = rows;
+        pf.lap(3);
+        if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 2);
+        if (r < rows && jw < g) {
+            contrib = true;
+            const bool ok = scan_gt(st, voff, vend, ba, bb, h.y, tbl);
+            pf.lap(1);
+            if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 3);
+            if (ok) {
+#if SPINFER_DW_PIPE
+                // --- decode the 16 TCTiles: 8 steps of 8 BitmapTiles (TCTile column tc = s / 2, TCTile
+                // rows 2 (s % 2), 2 (s % 2) + 1), two deep: while step s is assembled and multiplied, the
+                // value loads of step s + 1 and the table entries of step s + 2 are in flight
+                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
+                uint32_t bfr[2][NT][2];
+                auto load_x = [&](int tc, uint32_t (&b)[NT][2]) {
+                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+                    if constexpr (NT == 1) {
+                        ldsm_x2_trans(xk, b[0][0], b[0][1]);
+                    } else {
+                        ldsm_x4_trans(xk, b[0][0], b[0][1], b[1][0], b[1][1]);
+                    }
+                };
+                uint32_t tA0[8], tA1[8], sA[8], tB0[8], tB1[8], sB[8];
+                load_x(0, bfr[0]);
+                load_E(tbl_lane);
+                issue_to(tA0, tA1, sA);
+                load_E(tbl_lane + 64u);
+#pragma unroll
+                for (int s = 0; s < 8; ++s) {
+                    if (s + 1 < 8) {
+                        if (s & 1) issue_to(tA0, tA1, sA); else issue_to(tB0, tB1, sB);
+                    }
+                    if (s + 2 < 8) load_E(tbl_lane + (uint32_t)(s + 2) * 64u);
+                    if ((s & 1) && s + 1 < 8) load_x((s + 1) >> 1, bfr[((s + 1) >> 1) & 1]);
+                    if (s & 1) assemble_from(tB0, tB1, sB, 2, bfr[(s >> 1) & 1]);
+                    else assemble_from(tA0, tA1, sA, 0, bfr[(s >> 1) & 1]);
+                }
+#else
+                // --- decode the 16 TCTiles: TCTile column tc, row pairs (0,1), (2,3)
+                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
+                uint32_t t0[8], t1[8], s1[8];
+#pragma unroll 1
+                for (int tc = 0; tc < 4; ++tc) {
+                    uint32_t bfr[NT][2];
+                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+                    if constexpr (NT == 1) {
+                        ldsm_x2_trans(xk, bfr[0][0], bfr[0][1]);
+                    } else {
+                        ldsm_x4_trans(xk, bfr[0][0], bfr[0][1], bfr[1][0], bfr[1][1]);
+                    }
+#pragma unroll
+                    for (int hh = 0; hh < 2; ++hh) {
+                        load_E(tbl_lane + (uint32_t)(tc * 16 + hh * 8) * 8u);
+                        issue_to(t0, t1, s1);
+                        assemble_from(t0, t1, s1, 2 * hh, bfr);
+                    }
+                }
+#endif
+                __syncwarp();   // table reads done before the next GT's scan rewrites it
+                pf.lap(2);
+                if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 4);
+                pf.count(4);
+            } else if (lane == 0) {
+                atomicOr(prm.ws_err, 2);   // corrupt GT (or poisoned stage): skipped, Y is not valid
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
+            if (lane == 0) pf.st(prm.prof, p, i, 2, true);
+            if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 5);
+        }
+        i += 2;
+        slot += 2;
+        if (slot >= (uint32_t)S) { slot -= (uint32_t)S; ph ^= 1u; }
+    }
+    // segments after this warp's last stage: close the non-final ones it did not see
+    pf.lap(7);
+    const int fseg = nseg_total - 1;   // the final segment (reduced below in shared memory)
+    if (cur >= 0 && cur < fseg && r < f_rows) seg_close(cur, contrib);
+    for (int s2 = cur + 1; s2 < fseg; ++s2) seg_close(s2, false);
+    if (cur != fseg) {   // this warp holds nothing of the final segment
+#pragma unroll
+        for (int a = 0; a < 4; ++a)
+#pragma unroll
+            for (int b = 0; b < NT; ++b)
+#pragma unroll
+                for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
+    }
+    pf.lap(3);
+
+    // ---------------------------------------------------------------------- final segment
+    // All consumer warps are past their last stage, so the ring is free: the 8 warps of each GT
+    // row put their partials (row-major) into shared memory and warp m sums rows [8m, 8m + 8)
+    // over the 8 partials in warp order. Its shape comes from the reducer-free walk below.
+    named_bar_sync(1, 32 * kCWd);
+    int frb = 0, frows = 0;
+    bool fcomplete = false;
+    if (fseg >= 0) {   // the final segment's rowblock and extent: the CTA's last part
+        Stages it;
+        it.init(u0, u1, KG, G, MG);
+        int sstart = it.u;
+        while (it.valid()) {
+            if (it.seg_first()) sstart = it.u;
+            frb = it.rb; frows = it.rows;
+            const int send = it.u + it.g;
+            fcomplete = sstart == frb * KG && send == (frb + 1) * KG;
+            it.next(KG, G, MG);
+        }
+    }
+    if (fseg >= 0 && r < frows) {
+        const uint32_t mine = ring + (uint32_t)(r * 8 + m) * (64u * Np * 4u);
+#pragma unroll
+        for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) {
+                const uint32_t row = tr * 16 + (lane >> 2), col = nt * 8 + 2 * (lane & 3);
+                sts_v2(mine + (row * Np + col) * 4u, __float_as_uint(acc[tr][nt][0]), __float_as_uint(acc[tr][nt][1]));
+                sts_v2(mine + ((row + 8) * Np + col) * 4u, __float_as_uint(acc[tr][nt][2]), __float_as_uint(acc[tr][nt][3]));
+            }
+    }
+    named_bar_sync(1, 32 * kCWd);
+    if (fseg >= 0 && r < frows) {
+        constexpr int NC = Np / 4;   // outputs per lane: 8 rows x Np columns per warp
+        const int row = 8 * m + (lane >> 2), col0 = NC * (lane & 3);
+        float v[NC];
+#pragma unroll
+        for (int c = 0; c < NC; ++c) v[c] = 0.f;
+        for (int m2 = 0; m2 < 8; ++m2) {   // warp order; warps without a GT of the segment hold +0
+            const uint32_t a = ring + (uint32_t)(r * 8 + m2) * (64u * Np * 4u) + (uint32_t)(row * Np + col0) * 4u;
+            if constexpr (NC == 4) {
+                const float4 w = lds_f4(a);
+                v[0] += w.x; v[1] += w.y; v[2] += w.z; v[3] += w.w;
+            } else {
+                const uint2 w = lds_v2(a);
+                v[0] += __uint_as_float(w.x); v[1] += __uint_as_float(w.y);
+            }
+        }
+        const int grow = kRd * frb + r;
+        if (fcomplete) {
+            store_cols<NT, EPI, NC>(prm, grow * 64 + row, col0, v);
+        } else {
+            const int pfirst = uowner(frb * KG, prm.U, prm.P);
+            float *dst = prm.ws_cta + ((size_t)grow * prm.cslots + (p - pfirst)) * (64 * Np) + row * Np + col0;
+            if constexpr (NC == 4) stg_f4(reinterpret_cast<float4 *>(dst), make_float4(v[0], v[1], v[2], v[3]));
+            else stg_f2(dst, v[0], v[1]);
+        }
+    }
+    if (fseg >= 0 && !fcomplete) {
+        named_bar_sync(2, 32 * kCWd);   // every warp's slice of the CTA partial is stored
+        if (m == 0 && r < frows) cta_count_and_sum<NT, EPI>(prm, frb, kRd * frb + r, lane);
+    }
+    pf.lap(3);
+    pf.mark(6);
+    pf.dump(prm.prof, p, warp, lane);
+}
+
+inline uint32_t al(uint32_t x, uint32_t a) { return (x + a - 1) / a * a; }
+
+struct DPlan {
+    int P, G, S;
+    size_t smem;
+    DParams prm;
+};
+
+// CTA partial slots per GT row: the most CTAs one rowblock can overlap.
+int cta_slots(long long U, int P, int KG) {
+    const long long upc_min = std::max(1LL, U / P);
+    return (int)((KG + upc_min - 1) / upc_min + 1);
+}
+
+// Ring sizing: each slot holds the X slab (1024-aligned for the swizzle), both GT rows'
+// bitmaps and value capacity G * max_gt_values; prefer G = 4 with >= 4 slots.
+bool make_dplan(int M, int K, int Np, int max_gt_values, DPlan *pl) {
+    const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;
+    if (KG > 65535 || MG >= kErrWord) return false;
+    const long long U = (long long)((MG + kRd - 1) / kRd) * KG;
+    const int P = choose_grid(U);
+    if ((unsigned long long)U * (unsigned long long)P >= (1ull << 32)) return false;
+    int dev = 0, smem_max = 232448;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    cudaGetLastError();
+    int maxv = max_gt_values > 0 ? max_gt_values : 4096;
+    maxv = std::min(4096, (maxv + 7) & ~7);
+    int gmax = kMaxGd, smax = kMaxSd;
+    if (const char *e = getenv("SPINFER_G")) gmax = std::max(1, std::min(kMaxGd, atoi(e)));
+    if (const char *e = getenv("SPINFER_S")) smax = std::max(2, std::min(kMaxSd, atoi(e)));
+    const uint32_t final_scratch = 2u * 8u * 64u * Np * 4u;   // the final segment's partials reuse the ring
+    int bestG = 0, bestS = 0;   // the largest G with >= 4 slots, else the deepest ring with >= 2
+    for (int G = gmax; G >= 1; --G) {
+        const uint32_t st_bm = al((uint32_t)G * 64 * Np * 2, 128);
+        const uint32_t vcap = al((uint32_t)G * maxv * 2, 128);
+        const uint32_t slot = al(st_bm + kRd * G * 512 + 2 * vcap, 1024);
+        const int S = (int)std::min<long long>(smax, ((long long)smem_max - kOffRing - 1024) / slot);
+        if ((uint32_t)S * slot < final_scratch) continue;
+        if (S >= 4) { bestG = G; bestS = S; break; }
+        if (S >= 2 && S > bestS) { bestG = G; bestS = S; }
+    }
+    if (bestG == 0) return false;
+    const int G = bestG, S = bestS;
+    DParams &q = pl->prm;
+    q.KG = KG; q.MG = MG; q.M = M; q.U = (uint32_t)U; q.P = P; q.G = G; q.S = S;
+    q.st_bm = al((uint32_t)G * 64 * Np * 2, 128);
+    q.vcap = al((uint32_t)G * maxv * 2, 128);
+    q.st_v0 = q.st_bm + kRd * G * 512;
+    q.st_v1 = q.st_v0 + q.vcap;
+    q.slot_bytes = al(q.st_v1 + q.vcap, 1024);
+    q.cslots = cta_slots(U, P, KG);
+    pl->P = P; pl->G = G; pl->S = S;
+    pl->smem = (size_t)kOffRing + (size_t)S * q.slot_bytes + 1024;
+    return true;
+}
+
+template <int NT, bool EPI>
+int launch_dw(const DPlan &pl, cudaStream_t st) {
+    static int configured[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if ((int)pl.smem > configured[dev]) {
+        if (cudaFuncSetAttribute(k_spmm_dw<NT, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem) != cudaSuccess)
+            return SPINFER_ECUDA;
+        configured[dev] = (int)pl.smem;
+    }
+    k_spmm_dw<NT, EPI><<<pl.P, kThreadsD, pl.smem, st>>>(pl.prm);
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess && getenv("SPINFER_VERBOSE"))
+        fprintf(stderr, "spinfer: k_spmm_dw launch (P=%d smem=%zu): %s\n", pl.P, pl.smem, cudaGetErrorString(e));
+    return e == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
+}
+
+struct DwLayout {
+    size_t seg, cta, xpad, total;
+};
+DwLayout dw_layout(int M, int K, int N) {
+    const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;
+    const long long U = (long long)((MG + kRd - 1) / kRd) * KG;
+    const int P = choose_grid(U);
+    const int Np = (N + 7) & ~7;
+    DwLayout l;
+    l.seg = (size_t)P * kNSeg * kRd * 8 * 64 * Np * 4;
+    l.cta = (size_t)MG * cta_slots(U, P, KG) * 64 * Np * 4;
+    l.xpad = (N % 8) ? ((size_t)K * Np * 2 + 255) / 256 * 256 : 0;
+    l.total = kCounterRegion + l.seg + l.cta + l.xpad;
+    return l;
+}
+
+}  // namespace
+
+// Workspace of the decoupled-warp kernel: [CTA counters + error word][warp partials]
+// [CTA partials][padded X].
+size_t spmm_dw_workspace_bytes(int M, int K, int N) { return dw_layout(M, K, N).total; }
+
+int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias,
+                   int act, void *ws, size_t ws_bytes, cudaStream_t st) {
+    const int Np = (N + 7) & ~7;
+    if (Np > 16) return SPINFER_EINVAL;
+    DPlan pl;
+    if (!make_dplan(M, K, Np, T->max_gt_values, &pl)) return SPINFER_EINVAL;
+    const DwLayout lay = dw_layout(M, K, N);
+    if (ws == nullptr || ws_bytes < lay.total) return SPINFER_ENOSPC;
+    DParams &q = pl.prm;
+    uint8_t *w8 = reinterpret_cast<uint8_t *>(ws);
+    const uint16_t *Xk = X;
+    if (N % 8) {
+        uint16_t *Xp = reinterpret_cast<uint16_t *>(w8 + kCounterRegion + lay.seg + lay.cta);
+        if (int rc = launch_pad_x(X, Xp, K, N, Np, st)) return rc;
+        Xk = Xp;
+    }
+    if (int rc = make_x_tmap(&q.tmap_x, Xk, K, Np, Np, 64 * pl.G, kXTma)) return rc;
+    q.X = Xk;
+    q.K = K;
+    q.off = T->gtile_offset;
+    q.bm = T->bitmap;
+    q.vals = T->values;
+    q.Y = Y;
+    q.bias = bias;
+    q.act = act;
+    q.N = N;
+    q.ws_cnt = reinterpret_cast<int32_t *>(w8);
+    q.ws_err = reinterpret_cast<int32_t *>(w8) + kErrWord;
+    q.ws_seg = reinterpret_cast<float *>(w8 + kCounterRegion);
+    q.ws_cta = reinterpret_cast<float *>(w8 + kCounterRegion + lay.seg);
+    q.n_values = (int)T->n_values;
+    q.avg_gt = (float)((double)T->n_values / ((double)q.MG * (double)q.KG));
+    q.prof = nullptr;
+    const bool epi = bias != nullptr || act != SPINFER_ACT_NONE || (M % kGT) != 0 || (N % 8) != 0;
+    auto go = [&]() {
+        if (Np == 8) return epi ? launch_dw<1, true>(pl, st) : launch_dw<1, false>(pl, st);
+        return epi ? launch_dw<2, true>(pl, st) : launch_dw<2, false>(pl, st);
+    };
+#if SPINFER_INSTRUMENT
+    if (const char *path = getenv("SPINFER_PROF")) {   // experiments: dump per-warp cycle counters
+        static long long *prof_buf = nullptr;
+        const size_t n = kEvOff + 16 * 64 * 6;
+        if (!prof_buf && cudaMalloc(&prof_buf, n * 8) != cudaSuccess) return SPINFER_ECUDA;
+        cudaMemsetAsync(prof_buf, 0, n * 8, st);
+        q.prof = prof_buf;
+        const int rc = go();
+        long long *host = (long long *)malloc(n * 8);
+        cudaMemcpyAsync(host, prof_buf, n * 8, cudaMemcpyDeviceToHost, st);
+        cudaStreamSynchronize(st);
+        if (FILE *f = fopen(path, "wb")) { fwrite(host, 8, n, f); fclose(f); }
+        free(host);
+        return rc;
+    }
+#endif
+    return go();
+}
+
+}  // namespace spinfer

@@ -33,3 +33,15 @@ def assert_within(Y_gpu_bits: np.ndarray, Y_ref: np.ndarray, bound: np.ndarray, 
         raise AssertionError(f"{what}: {int(bad.sum())} outputs out of tolerance, e.g. "
                              + ", ".join(f"{tuple(i)} gpu={y[tuple(i)]} ref={Y_ref[tuple(i)]} bound={bound[tuple(i)]:.3g}"
                                          for i in idx))
+
+
+def use_kernel(kernel: str, N: int, monkeypatch):
+    """Select the SpMM kernel for this test (SPINFER_KERNEL): "default" = the library's choice,
+    "dw" = the decoupled-warp kernel (N <= 16), "mma" = the round-1 mma.sync kernel, "tc" =
+    the tcgen05 kernel."""
+    import pytest
+    if kernel == "default":
+        return
+    if kernel == "dw" and N > 16:
+        pytest.skip("the decoupled-warp kernel serves N <= 16")
+    monkeypatch.setenv("SPINFER_KERNEL", kernel)
