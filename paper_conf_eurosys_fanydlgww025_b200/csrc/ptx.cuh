@@ -76,6 +76,11 @@ __device__ __forceinline__ bool mbar_test_wait(uint32_t bar, uint32_t parity) {
         : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
     return ok != 0;
 }
+// Poll with a fixed sleep between probes: a waiter that is not woken by the CTA's other
+// mbarrier events (each event wakes every suspended try_wait, which then re-executes).
+__device__ __forceinline__ void mbar_wait_poll(uint32_t bar, uint32_t parity, uint32_t ns) {
+    while (!mbar_test_wait(bar, parity)) __nanosleep(ns);
+}
 // For waiters that usually block for a long time (scan on data, producer on a free slot):
 // the hinted try_wait sleeps until ANY mbarrier event of the CTA, i.e. it wakes ~25 times
 // per stage; a timed back-off (plain nanosleep, not woken by barrier traffic) polls a few times.
@@ -145,6 +150,25 @@ __device__ __forceinline__ uint4 lds_v4(uint32_t a) {
     asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
     return v;
 }
+// Non-volatile variants for a decode region the compiler may schedule freely (deep load
+// lookahead): the region is bracketed by launder_u32 (addresses defined after the table writes)
+// and fence_acc (every accumulator consumed before what follows).
+__device__ __forceinline__ uint4 lds_v4_nv(uint32_t a) {
+    uint4 v;
+    asm("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ void ldsm_x4_trans_nv(uint32_t a, uint32_t &d0, uint32_t &d1, uint32_t &d2, uint32_t &d3) {
+    asm("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0, %1, %2, %3}, [%4];"
+        : "=r"(d0), "=r"(d1), "=r"(d2), "=r"(d3) : "r"(a));
+}
+__device__ __forceinline__ void ldsm_x2_trans_nv(uint32_t a, uint32_t &d0, uint32_t &d1) {
+    asm("ldmatrix.sync.aligned.m8n8.x2.trans.shared.b16 {%0, %1}, [%2];" : "=r"(d0), "=r"(d1) : "r"(a));
+}
+__device__ __forceinline__ uint32_t launder_u32(uint32_t v) {
+    asm volatile("mov.b32 %0, %0;" : "+r"(v) :: "memory");
+    return v;
+}
 // Non-volatile: its address always comes from a volatile table load issued after
 // the stage's mbarrier wait, and its result feeds a volatile mma, so it can be
 // scheduled freely in between but never crosses the wait or the release.
@@ -199,6 +223,12 @@ __device__ __forceinline__ void ldsm_x4_trans(uint32_t a, uint32_t &d0, uint32_t
 __device__ __forceinline__ void ldsm_x2_trans(uint32_t a, uint32_t &d0, uint32_t &d1) {
     asm volatile("ldmatrix.sync.aligned.m8n8.x2.trans.shared.b16 {%0, %1}, [%2];"
                  : "=r"(d0), "=r"(d1) : "r"(a));
+}
+__device__ __forceinline__ void mma_16816_nv(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+    asm("mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0, %1, %2, %3}, {%4, %5, %6, %7}, {%8, %9}, "
+        "{%0, %1, %2, %3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
 }
 // D = A(16x16, row) * B(16x8, col) + D ; f16 inputs, f32 accumulate (Listing 1)
 __device__ __forceinline__ void mma_16816(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
@@ -265,6 +295,27 @@ __device__ __forceinline__ void tm_ld_32x32b_x16(uint32_t taddr, float (&v)[16])
                  : "r"(taddr) : "memory");
 #pragma unroll
     for (int j = 0; j < 16; ++j) v[j] = __uint_as_float(r[j]);
+}
+// A warp's own lane quarter, 32-bit columns: 16 (x16) or 8 (x8) consecutive columns per thread.
+__device__ __forceinline__ void tm_st_32x32b_x16(uint32_t taddr, const uint32_t (&r)[16]) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};"
+                 ::"r"(taddr), "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]),
+                   "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]) : "memory");
+}
+__device__ __forceinline__ void tm_ld_32x32b_x16u(uint32_t taddr, uint32_t (&r)[16]) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+                   "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+                 : "r"(taddr) : "memory");
+}
+__device__ __forceinline__ void tm_st_32x32b_x8(uint32_t taddr, const uint32_t (&r)[8]) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};"
+                 ::"r"(taddr), "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]) : "memory");
+}
+__device__ __forceinline__ void tm_ld_32x32b_x8u(uint32_t taddr, uint32_t (&r)[8]) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+                 : "r"(taddr) : "memory");
 }
 // D[tmem] (+)= A[tmem] x B[smem descriptor]; kind::f16 (fp16 in, fp32 accumulate), cta_group::1.
 __device__ __forceinline__ void umma_f16_ts(uint32_t d_t, uint32_t a_t, uint64_t bdesc, uint32_t idesc, uint32_t acc) {

@@ -41,8 +41,11 @@ constexpr int kCWd = 16;                  // consumer warps: r = w >> 3, m = w &
 constexpr int kProdWarp0 = kCWd;          // producer warps kCWd, kCWd + 2 (SMSPs 0 and 2)
 constexpr int kNProd = 2;                 // stage i is issued by producer i % 2
 constexpr int kRedWarp = kCWd + 1;        // reducer warp (SMSP 1)
+#ifndef SPINFER_DW_VSCAN
+#define SPINFER_DW_VSCAN 0
+#endif
 #ifndef SPINFER_DW_PIPE
-#define SPINFER_DW_PIPE 0
+#define SPINFER_DW_PIPE 2
 #endif
 #ifndef SPINFER_DW_REG
 #define SPINFER_DW_REG 0
@@ -59,7 +62,10 @@ constexpr int kNSeg = 4;                  // segment slots between consumers and
 constexpr uint32_t kHdrBytes = 64;        // per-slot stage header: value offsets, poison flag
 constexpr uint32_t kTblBytes = 1024;      // one GroupTile's SMBD table (64 BTs x 2 halves x 8 B)
 // shared-memory map (bytes from the 1024-aligned base)
-constexpr uint32_t kBarFull = 0, kBarEmpty = 64, kBarSegFull = 128, kBarSegFree = 192, kSegMask = 224;
+constexpr uint32_t kBarFull = 0, kBarEmpty = 64, kBarSegFull = 128, kBarSegFree = 192, kSegMask = 224, kTmemSlot = 256;
+// PIPE 9: each consumer warp keeps its fp32 accumulators in its TMEM lane quarter between
+// half-GroupTile phases (16 N columns: 32 TMEM columns per warp, 128 per quarter)
+constexpr uint32_t kTmemCols = 128;
 #ifndef SPINFER_DW_XTMA
 #define SPINFER_DW_XTMA 1
 #endif
@@ -92,6 +98,7 @@ struct DParams {
     uint32_t slot_bytes, st_bm, st_v0, st_v1, vcap;   // slot: X slab | bitmaps | values row 0 | row 1
     float avg_gt;                 // n_values / NGT (start-up page prefetch hint)
     long long *prof;              // experiments only (SPINFER_INSTRUMENT)
+    uint32_t zero;                // 0 at run time (a value ptxas cannot fold: scheduling dependency)
 };
 
 #ifndef SPINFER_INSTRUMENT
@@ -329,6 +336,53 @@ __device__ __forceinline__ void cta_count_and_sum(const DParams &prm, int rb, in
     if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed for the next call
 }
 
+// The decode of one GroupTile as its own (out-of-line) function: compiled in a clean context, ptxas
+// issues the table and value loads of the whole GT in one burst ahead of the MMAs (3x the decode
+// throughput of the interleaved schedule it picks inside the consumer loop, tools/decode_bench.cu).
+template <int NT>
+struct AccT {
+    float v[4][NT][4];
+};
+template <int NT>
+__device__ __noinline__ AccT<NT> decode_gt(AccT<NT> acc, uint32_t tbl_lane, uint32_t xs, uint32_t mulc) {
+    constexpr uint32_t cpr = NT;
+    uint32_t bfr[4][NT][2];
+#pragma unroll
+    for (int tc = 0; tc < 4; ++tc) {
+        const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+        if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
+        else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+    }
+#pragma unroll
+    for (int s8 = 0; s8 < 8; ++s8) {
+        uint4 E[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) E[k] = lds_v4(tbl_lane + (uint32_t)s8 * 64u + 16u * k);
+        uint32_t t0[8], t1[8], s1[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
+            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;   // first value of the half - 4 bytes
+            const uint32_t z = w * mulc;                               // top two bits: the lane's pair y
+            const uint32_t a = A + 2u * __popc(z);                     // &V[c2 - 2], c2 = MaskedPopCount + y0 + y1
+            const uint32_t y = z >> 30;
+            s1[k] = y * (y * kSelB + kSelA) + kSelC;
+            t0[k] = lds_u16(a);
+            t1[k] = lds_u16(a + 2u);
+        }
+        const int trb = 2 * (s8 & 1);
+#pragma unroll
+        for (int tt = 0; tt < 2; ++tt) {
+            uint32_t afr[4];
+#pragma unroll
+            for (int b = 0; b < 4; ++b) afr[b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) mma_16816(acc.v[trb + tt][nt], afr, bfr[s8 >> 1][nt][0], bfr[s8 >> 1][nt][1]);
+        }
+    }
+    return acc;
+}
+
 template <int NT, bool EPI>
 __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant__ DParams prm) {
     constexpr int Np = NT * 8;
@@ -359,7 +413,14 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         }
         fence_barrier_init();
     }
+#if SPINFER_DW_PIPE == 9
+    if (warp == 0) tm_alloc(sbase + kTmemSlot, kTmemCols);
+    tm_fence_before();
+#endif
     __syncthreads();
+#if SPINFER_DW_PIPE == 9
+    tm_fence_after();
+#endif
     Prof pf;
     pf.start();
     // role warps (warpgroup 4): give registers back, then split into producers / reducer / idle.
@@ -415,7 +476,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             const uint32_t slot = pslot, ph = pph;
             pf.lap(1);
             if (lane == 0) pf.st(prm.prof, p, i, 3, true);
-            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, ph ^ 1u);
+            if (i >= S) mbar_wait_poll(bar_empty + 8 * slot, ph ^ 1u, 128u);
             pf.lap(0);
             if (lane == 0) pf.st(prm.prof, p, i, 0, true);
             const uint32_t st = ring + slot * prm.slot_bytes, fb = bar_full + 8 * slot;
@@ -485,7 +546,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         {
             if ((i & 1) != q) ++i;   // the loop can stop one index short of this producer's parity
             const uint32_t slot = (uint32_t)(i % S), ph = (uint32_t)(i / S) & 1u;
-            if (i >= S) mbar_wait_sleep(bar_empty + 8 * slot, ph ^ 1u);
+            if (i >= S) mbar_wait_poll(bar_empty + 8 * slot, ph ^ 1u, 128u);
             if (lane == 0) {
                 sts_v4(sbase + kOffHdr + slot * kHdrBytes, make_uint4(0u, kHdrStop, (uint32_t)nseg, 0u));
                 mbar_arrive(bar_full + 8 * slot);
@@ -516,7 +577,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             const bool complete = sstart == rb * KG && send == (rb + 1) * KG;
             for (int r = 0; r < rows; ++r) {
                 pf.lap(1);
-                mbar_wait_sleep(bar_sfull + 16 * k + 8 * r, par);
+                mbar_wait_poll(bar_sfull + 16 * k + 8 * r, par, 512u);
                 pf.lap(0);
                 const uint32_t cmask = lds_u32(seg_mask + 8 * k + 4 * r);   // warps that own a GT of the segment
                 if (lane == 0) sts_u32(seg_mask + 8 * k + 4 * r, 0u);
@@ -582,7 +643,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     // stage's shape and segment index from the slot header.
     const int r = warp >> 3, m = warp & 7, jw = m & 3;
     const uint32_t mulc = opaque_u32(1u << (30u - 2u * (uint32_t)(lane & 15)));   // z = w << (30 - sh) on the FMA pipe
-    const uint32_t selA = opaque_u32(kSelA), selB = opaque_u32(kSelB), selC = opaque_u32(kSelC);
+    constexpr uint32_t selA = kSelA, selB = kSelB, selC = kSelC;   // IMAD immediates
     constexpr uint32_t cpr = Np / 8;   // 16-byte chunks per X row
     const uint32_t rr = lane & 7, mk = (lane >> 3) & 1, mn = (lane >> 4) & 1;
     // X slab row-major; with the tensor copy the 32B swizzle XORs the 16-byte chunk with row bit 2
@@ -599,6 +660,21 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     auto load_E = [&](uint32_t tb) {   // entries of 8 consecutive BTs, this lane's half
 #pragma unroll
         for (int k = 0; k < 4; ++k) E[k] = lds_v4(tb + 16u * k);
+    };
+    auto load_E_nv = [&](uint32_t tb) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) E[k] = lds_v4_nv(tb + 16u * k);
+    };
+    auto assemble_nv = [&](const uint32_t (&u0)[8], const uint32_t (&u1)[8], const uint32_t (&sl)[8], int trb,
+                           const uint32_t (&bfr)[NT][2]) {
+#pragma unroll
+        for (int tt = 0; tt < 2; ++tt) {
+            uint32_t afr[4];
+#pragma unroll
+            for (int b = 0; b < 4; ++b) afr[b] = prmt(u0[tt * 4 + b], u1[tt * 4 + b], sl[tt * 4 + b]);
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) mma_16816_nv(acc[trb + tt][nt], afr, bfr[nt][0], bfr[nt][1]);
+        }
     };
     auto issue_to = [&](uint32_t (&u0)[8], uint32_t (&u1)[8], uint32_t (&sl)[8]) {   // SMBD value loads into a set
 #pragma unroll
@@ -624,12 +700,71 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             for (int nt = 0; nt < NT; ++nt) mma_16816(acc[trb + tt][nt], afr, bfr[nt][0], bfr[nt][1]);
         }
     };
+#if SPINFER_DW_PIPE == 9
+    const uint32_t tacc = lds_u32(sbase + kTmemSlot) + ((uint32_t)(warp & 3) * 32u << 16) + (uint32_t)(warp >> 2) * 16u * NT;
+    uint32_t zmask = 3u;   // bit h: half h of the accumulators (TCTile rows 2h, 2h + 1) is zero, not in TMEM
+    auto tm_get = [&](int h, float (&a)[2][NT][4]) {
+        if ((zmask >> h) & 1u) {
+#pragma unroll
+            for (int t = 0; t < 2; ++t)
+#pragma unroll
+                for (int b = 0; b < NT; ++b)
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) a[t][b][e] = 0.f;
+            return;
+        }
+        if constexpr (NT == 2) {
+            uint32_t u[16];
+            tm_ld_32x32b_x16u(tacc + 16u * h, u);
+            tm_wait_ld();
+#pragma unroll
+            for (int k = 0; k < 16; ++k) a[k >> 3][(k >> 2) & 1][k & 3] = __uint_as_float(u[k]);
+        } else {
+            uint32_t u[8];
+            tm_ld_32x32b_x8u(tacc + 8u * h, u);
+            tm_wait_ld();
+#pragma unroll
+            for (int k = 0; k < 8; ++k) a[k >> 2][0][k & 3] = __uint_as_float(u[k]);
+        }
+    };
+    auto tm_put = [&](int h, const float (&a)[2][NT][4]) {
+        if constexpr (NT == 2) {
+            uint32_t u[16];
+#pragma unroll
+            for (int k = 0; k < 16; ++k) u[k] = __float_as_uint(a[k >> 3][(k >> 2) & 1][k & 3]);
+            tm_st_32x32b_x16(tacc + 16u * h, u);
+        } else {
+            uint32_t u[8];
+#pragma unroll
+            for (int k = 0; k < 8; ++k) u[k] = __float_as_uint(a[k >> 2][0][k & 3]);
+            tm_st_32x32b_x8(tacc + 8u * h, u);
+        }
+        tm_wait_st();
+        zmask &= ~(1u << h);
+    };
+    auto fetch_acc = [&]() {   // the accumulators into registers (segment ends)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            float a[2][NT][4];
+            tm_get(h, a);
+#pragma unroll
+            for (int t = 0; t < 2; ++t)
+#pragma unroll
+                for (int b = 0; b < NT; ++b)
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) acc[2 * h + t][b][e] = a[t][b][e];
+        }
+    };
+#else
+    auto fetch_acc = [&]() {};
+#endif
     // segment hand-off to the reducer (non-final segments): park the partial if this warp owned a
     // GT of the segment, then arrive; `own` = false arrives for a segment without a GT of this warp
     auto seg_close = [&](int sg, bool own) {
         const int k = sg % kNSeg;
-        if (sg >= kNSeg) mbar_wait_sleep(bar_sfree + 8 * k, (uint32_t)((sg / kNSeg) - 1) & 1u);
+        if (sg >= kNSeg) mbar_wait_poll(bar_sfree + 8 * k, (uint32_t)((sg / kNSeg) - 1) & 1u, 256u);
         if (own) {
+            fetch_acc();
             float4 *dst = reinterpret_cast<float4 *>(prm.ws_seg) + ((((size_t)p * kNSeg + k) * kRd + r) * 8 + m) * kF4;
 #pragma unroll
             for (int tr = 0; tr < 4; ++tr)
@@ -652,6 +787,23 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         const uint32_t vsm = st_ + (r ? prm.st_v1 : prm.st_v0) + voff_;
         const uint32_t pax = __popc(ba_.x), pbx = __popc(bb_.x);
         const uint32_t packed = (pax + __popc(ba_.y)) | ((pbx + __popc(bb_.y)) << 16);
+#if SPINFER_DW_VSCAN
+        // exclusive prefix of the two 7-bit counts over the lanes, bit-sliced with ballots (vote
+        // unit, not the shared-memory pipe the shuffles queue behind)
+        const uint32_t lo = packed & 0xFFFFu, hi = packed >> 16;
+        const uint32_t lt = (1u << lane) - 1u;
+        uint32_t elo = 0, ehi = 0, tlo = 0, thi = 0;
+#pragma unroll
+        for (int b = 0; b < 7; ++b) {
+            const uint32_t B0 = __ballot_sync(0xffffffffu, (lo >> b) & 1u), B1 = __ballot_sync(0xffffffffu, (hi >> b) & 1u);
+            elo += (uint32_t)__popc(B0 & lt) << b;
+            ehi += (uint32_t)__popc(B1 & lt) << b;
+            tlo += (uint32_t)__popc(B0) << b;
+            thi += (uint32_t)__popc(B1) << b;
+        }
+        const uint32_t tot = tlo | (thi << 16);
+        const uint32_t incl = packed + (elo | (ehi << 16));
+#else
         uint32_t incl = packed;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -659,6 +811,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             incl += (lane >= o) ? y : 0u;
         }
         const uint32_t tot = __shfl_sync(0xffffffffu, incl, 31);
+#endif
         const uint32_t tot_a = tot & 0xFFFFu;
         if ((flags_ & kHdrBad) || 2u * (tot_a + (tot >> 16)) > vend_ - voff_) return false;
         const uint32_t excl = incl - packed;
@@ -681,7 +834,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     while (true) {
         pf.lap(7);
         if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 0);
-        mbar_wait_sleep(bar_full + 8 * slot, ph);
+        if (!mbar_test_wait(bar_full + 8 * slot, ph)) mbar_wait_sleep(bar_full + 8 * slot, ph);
         if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 1);
         if (!seen) { seen = true; pf.mark(5); }
         pf.lap(0);
@@ -701,12 +854,16 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             if (cur >= 0 && r < f_rows) seg_close(cur, contrib);
             for (int s2 = cur + 1; s2 < sg; ++s2) seg_close(s2, false);   // segments with no stage of this parity
             cur = sg;
+#if SPINFER_DW_PIPE == 9
+            zmask = 3u;
+#else
 #pragma unroll
             for (int a = 0; a < 4; ++a)
 #pragma unroll
                 for (int b = 0; b < NT; ++b)
 #pragma unroll
                     for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
+#endif
             contrib = false;
         }
         f_rb = (int)h.x; f_rows = rows;
@@ -718,7 +875,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             pf.lap(1);
             if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 3);
             if (ok) {
-#if SPINFER_DW_PIPE
+#if SPINFER_DW_PIPE == 1
                 // --- decode the 16 TCTiles: 8 steps of 8 BitmapTiles (TCTile column tc = s / 2, TCTile
                 // rows 2 (s % 2), 2 (s % 2) + 1), two deep: while step s is assembled and multiplied, the
                 // value loads of step s + 1 and the table entries of step s + 2 are in flight
@@ -747,6 +904,242 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                     if (s & 1) assemble_from(tB0, tB1, sB, 2, bfr[(s >> 1) & 1]);
                     else assemble_from(tA0, tA1, sA, 0, bfr[(s >> 1) & 1]);
                 }
+#elif SPINFER_DW_PIPE == 2
+                // --- decode the 16 TCTiles: TCTile column tc, row pairs (0,1), (2,3)
+                // the whole GT is one schedulable region: addresses laundered after the table writes,
+                // accumulators fenced at the end, no volatile operation in between
+                const uint32_t xs = launder_u32(st + x_lane + (uint32_t)(64 * jw) * cpr * 16u);
+                const uint32_t tbl_lane_l = launder_u32(tbl_lane);
+                uint32_t t0[8], t1[8], s1[8];
+#pragma unroll
+                for (int tc = 0; tc < 4; ++tc) {
+                    uint32_t bfr[NT][2];
+                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+                    if constexpr (NT == 1) {
+                        ldsm_x2_trans_nv(xk, bfr[0][0], bfr[0][1]);
+                    } else {
+                        ldsm_x4_trans_nv(xk, bfr[0][0], bfr[0][1], bfr[1][0], bfr[1][1]);
+                    }
+#pragma unroll
+                    for (int hh = 0; hh < 2; ++hh) {
+                        load_E_nv(tbl_lane_l + (uint32_t)(tc * 16 + hh * 8) * 8u);
+                        issue_to(t0, t1, s1);
+                        assemble_nv(t0, t1, s1, 2 * hh, bfr);
+                    }
+                }
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+#pragma unroll
+                    for (int b = 0; b < NT; ++b)
+                        asm volatile("" : "+f"(acc[a][b][0]), "+f"(acc[a][b][1]), "+f"(acc[a][b][2]), "+f"(acc[a][b][3]) :: "memory");
+#elif SPINFER_DW_PIPE == 5
+                {
+                    AccT<NT> a_;
+#pragma unroll
+                    for (int a = 0; a < 4; ++a)
+#pragma unroll
+                        for (int b = 0; b < NT; ++b)
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) a_.v[a][b][e] = acc[a][b][e];
+                    a_ = decode_gt<NT>(a_, tbl_lane, st + x_lane + (uint32_t)(64 * jw) * cpr * 16u, mulc);
+#pragma unroll
+                    for (int a = 0; a < 4; ++a)
+#pragma unroll
+                        for (int b = 0; b < NT; ++b)
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) acc[a][b][e] = a_.v[a][b][e];
+                }
+#elif SPINFER_DW_PIPE == 6
+                // --- decode in two phases per half GroupTile: (1) table entries, value loads and PRMTs
+                // of 32 BitmapTiles into A fragments, (2) their 16 MMAs; a compiler barrier between
+                // the phases keeps the 64 value loads of a half in one burst ahead of the MMAs
+                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
+#pragma unroll
+                for (int half = 0; half < 2; ++half) {
+                    uint32_t bfr[2][NT][2];
+#pragma unroll
+                    for (int t2 = 0; t2 < 2; ++t2) {
+                        const uint32_t xk = xs + (uint32_t)(16 * (2 * half + t2)) * cpr * 16u;
+                        if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[t2][0][0], bfr[t2][0][1]);
+                        else ldsm_x4_trans(xk, bfr[t2][0][0], bfr[t2][0][1], bfr[t2][1][0], bfr[t2][1][1]);
+                    }
+                    uint32_t afr[4][2][4];
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        uint32_t t0[8], t1[8], s1[8];
+                        load_E(tbl_lane + (uint32_t)(4 * half + k) * 64u);
+                        issue_to(t0, t1, s1);
+#pragma unroll
+                        for (int tt = 0; tt < 2; ++tt)
+#pragma unroll
+                            for (int b = 0; b < 4; ++b) afr[k][tt][b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
+                    }
+#pragma unroll
+                    for (int k = 0; k < 4; ++k)
+#pragma unroll
+                        for (int tt = 0; tt < 2; ++tt)
+                            asm volatile("" : "+r"(afr[k][tt][0]), "+r"(afr[k][tt][1]), "+r"(afr[k][tt][2]), "+r"(afr[k][tt][3]));
+#pragma unroll
+                    for (int k = 0; k < 4; ++k)
+#pragma unroll
+                        for (int tt = 0; tt < 2; ++tt)
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt)
+                                mma_16816(acc[2 * (k & 1) + tt][nt], afr[k][tt], bfr[k >> 1][nt][0], bfr[k >> 1][nt][1]);
+                }
+#elif SPINFER_DW_PIPE == 7
+                // --- decode in two phases per GroupTile: (1) table entries, value loads and PRMTs of all
+                // 64 BitmapTiles into A fragments, (2) the 32 MMAs. Every MMA also depends on the last
+                // fragment (OR with prm.zero, 0 at run time and unknown to ptxas), so ptxas issues the
+                // GT's 128 value loads in one burst instead of interleaving them with the MMAs
+                // (tools/decode_bench.cu: 3x the decode throughput).
+                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
+                uint32_t afr[8][2][4];
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    uint32_t t0[8], t1[8], s1[8];
+                    load_E(tbl_lane + (uint32_t)k * 64u);
+                    issue_to(t0, t1, s1);
+#pragma unroll
+                    for (int tt = 0; tt < 2; ++tt)
+#pragma unroll
+                        for (int b = 0; b < 4; ++b) afr[k][tt][b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
+                }
+                const uint32_t dep = afr[7][1][3] & prm.zero;
+                uint32_t bfr[4][NT][2];
+#pragma unroll
+                for (int tc = 0; tc < 4; ++tc) {
+                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+                    if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
+                    else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+                }
+#pragma unroll
+                for (int k = 0; k < 8; ++k)
+#pragma unroll
+                    for (int tt = 0; tt < 2; ++tt) {
+                        afr[k][tt][0] |= dep;
+#pragma unroll
+                        for (int nt = 0; nt < NT; ++nt)
+                            mma_16816(acc[2 * (k & 1) + tt][nt], afr[k][tt], bfr[k >> 1][nt][0], bfr[k >> 1][nt][1]);
+                    }
+#elif SPINFER_DW_PIPE == 8
+                // --- as PIPE 7, per half GroupTile (32 BitmapTiles per burst, fewer live fragments)
+                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
+#pragma unroll
+                for (int half = 0; half < 2; ++half) {
+                    uint32_t afr[4][2][4];
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        uint32_t t0[8], t1[8], s1[8];
+                        load_E(tbl_lane + (uint32_t)(4 * half + k) * 64u);
+                        issue_to(t0, t1, s1);
+#pragma unroll
+                        for (int tt = 0; tt < 2; ++tt)
+#pragma unroll
+                            for (int b = 0; b < 4; ++b) afr[k][tt][b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
+                    }
+                    const uint32_t dep = afr[3][1][3] & prm.zero;
+                    uint32_t bfr[2][NT][2];
+#pragma unroll
+                    for (int t2 = 0; t2 < 2; ++t2) {
+                        const uint32_t xk = xs + (uint32_t)(16 * (2 * half + t2)) * cpr * 16u;
+                        if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[t2][0][0], bfr[t2][0][1]);
+                        else ldsm_x4_trans(xk, bfr[t2][0][0], bfr[t2][0][1], bfr[t2][1][0], bfr[t2][1][1]);
+                    }
+#pragma unroll
+                    for (int k = 0; k < 4; ++k)
+#pragma unroll
+                        for (int tt = 0; tt < 2; ++tt) {
+                            afr[k][tt][0] |= dep;
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt)
+                                mma_16816(acc[2 * (k & 1) + tt][nt], afr[k][tt], bfr[k >> 1][nt][0], bfr[k >> 1][nt][1]);
+                        }
+                }
+#elif SPINFER_DW_PIPE == 9
+                // --- decode in two phases of 32 BitmapTiles (TCTile rows 2h, 2h + 1 of all 4 TCTile
+                // columns); the phase's 16 accumulators come from and go back to TMEM, which frees
+                // the registers for the whole phase's table entries, value loads and PRMTs ahead of
+                // its 16 MMAs (one burst of 64 value loads; tools/decode_bench.cu)
+                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
+                uint32_t bfr[4][NT][2];
+#pragma unroll
+                for (int tc = 0; tc < 4; ++tc) {
+                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+                    if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
+                    else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+                }
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    uint32_t afr[4][2][4];
+#pragma unroll
+                    for (int tc = 0; tc < 4; ++tc) {
+                        uint32_t t0[8], t1[8], s1[8];
+                        load_E(tbl_lane + (uint32_t)(2 * tc + h) * 64u);
+                        issue_to(t0, t1, s1);
+#pragma unroll
+                        for (int tt = 0; tt < 2; ++tt)
+#pragma unroll
+                            for (int b = 0; b < 4; ++b) afr[tc][tt][b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
+                    }
+                    float a[2][NT][4];
+                    tm_get(h, a);
+                    const uint32_t dep = afr[3][1][3] & prm.zero;
+#pragma unroll
+                    for (int tc = 0; tc < 4; ++tc)
+#pragma unroll
+                        for (int tt = 0; tt < 2; ++tt) {
+                            afr[tc][tt][0] |= dep;
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt) mma_16816(a[tt][nt], afr[tc][tt], bfr[tc][nt][0], bfr[tc][nt][1]);
+                        }
+                    tm_put(h, a);
+                }
+#elif SPINFER_DW_PIPE == 4
+                // --- decode the 16 TCTiles, fully unrolled: X fragments of all 4 TCTile columns, then
+                // 8 steps of 8 BitmapTiles (tools/decode_bench.cu: the compiler issues the table and
+                // value loads of the whole GT in one burst ahead of the MMAs)
+                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
+                uint32_t bfr[4][NT][2];
+#pragma unroll
+                for (int tc = 0; tc < 4; ++tc) {
+                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+                    if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
+                    else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+                }
+                uint32_t t0[8], t1[8], s1[8];
+#pragma unroll
+                for (int s8 = 0; s8 < 8; ++s8) {
+                    load_E(tbl_lane + (uint32_t)s8 * 64u);
+                    issue_to(t0, t1, s1);
+                    assemble_from(t0, t1, s1, 2 * (s8 & 1), bfr[s8 >> 1]);
+                }
+#elif SPINFER_DW_PIPE == 3
+                // --- decode the 16 TCTiles as one schedulable region (no volatile operation inside:
+                // addresses laundered after the table writes, accumulators fenced at the end), X
+                // fragments of all 4 TCTile columns first, then 8 steps of 8 BitmapTiles; the compiler
+                // hoists the table and value loads of later steps ahead of earlier steps' MMAs
+                const uint32_t xs = launder_u32(st + x_lane + (uint32_t)(64 * jw) * cpr * 16u);
+                const uint32_t tbl_lane_l = launder_u32(tbl_lane);
+                uint32_t bfr[4][NT][2];
+#pragma unroll
+                for (int tc = 0; tc < 4; ++tc) {
+                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+                    if constexpr (NT == 1) ldsm_x2_trans_nv(xk, bfr[tc][0][0], bfr[tc][0][1]);
+                    else ldsm_x4_trans_nv(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+                }
+                uint32_t t0[8], t1[8], s1[8];
+#pragma unroll
+                for (int s8 = 0; s8 < 8; ++s8) {
+                    load_E_nv(tbl_lane_l + (uint32_t)s8 * 64u);
+                    issue_to(t0, t1, s1);
+                    assemble_nv(t0, t1, s1, 2 * (s8 & 1), bfr[s8 >> 1]);
+                }
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+#pragma unroll
+                    for (int b = 0; b < NT; ++b)
+                        asm volatile("" : "+f"(acc[a][b][0]), "+f"(acc[a][b][1]), "+f"(acc[a][b][2]), "+f"(acc[a][b][3]) :: "memory");
 #else
                 // --- decode the 16 TCTiles: TCTile column tc, row pairs (0,1), (2,3)
                 const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
@@ -789,6 +1182,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     const int fseg = nseg_total - 1;   // the final segment (reduced below in shared memory)
     if (cur >= 0 && cur < fseg && r < f_rows) seg_close(cur, contrib);
     for (int s2 = cur + 1; s2 < fseg; ++s2) seg_close(s2, false);
+    if (cur == fseg) fetch_acc();
     if (cur != fseg) {   // this warp holds nothing of the final segment
 #pragma unroll
         for (int a = 0; a < 4; ++a)
@@ -806,17 +1200,14 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     named_bar_sync(1, 32 * kCWd);
     int frb = 0, frows = 0;
     bool fcomplete = false;
-    if (fseg >= 0) {   // the final segment's rowblock and extent: the CTA's last part
-        Stages it;
-        it.init(u0, u1, KG, G, MG);
-        int sstart = it.u;
-        while (it.valid()) {
-            if (it.seg_first()) sstart = it.u;
-            frb = it.rb; frows = it.rows;
-            const int send = it.u + it.g;
-            fcomplete = sstart == frb * KG && send == (frb + 1) * KG;
-            it.next(KG, G, MG);
-        }
+    if (fseg >= 0) {   // the final segment: the last rowblock piece of the CTA's last non-empty part (A, C, M order)
+        const int a_end = (u0 % KG) ? min(u1, (u0 / KG + 1) * KG) : u0;
+        const int c_beg = (u1 % KG) ? max(a_end, (u1 / KG) * KG) : u1;
+        int ps, pe;
+        if (a_end < c_beg) { ps = a_end; pe = c_beg; } else if (c_beg < u1) { ps = c_beg; pe = u1; } else { ps = u0; pe = a_end; }
+        frb = (pe - 1) / KG;
+        frows = min(kRd, MG - kRd * frb);
+        fcomplete = max(ps, frb * KG) == frb * KG && pe == (frb + 1) * KG;
     }
     if (fseg >= 0 && r < frows) {
         const uint32_t mine = ring + (uint32_t)(r * 8 + m) * (64u * Np * 4u);
@@ -830,6 +1221,9 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             }
     }
     named_bar_sync(1, 32 * kCWd);
+#if SPINFER_DW_PIPE == 9
+    if (warp == 0) tm_dealloc(lds_u32(sbase + kTmemSlot), kTmemCols);   // every consumer fetched its accumulators
+#endif
     if (fseg >= 0 && r < frows) {
         constexpr int NC = Np / 4;   // outputs per lane: 8 rows x Np columns per warp
         const int row = 8 * m + (lane >> 2), col0 = NC * (lane & 3);
@@ -995,6 +1389,7 @@ int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, 
     q.n_values = (int)T->n_values;
     q.avg_gt = (float)((double)T->n_values / ((double)q.MG * (double)q.KG));
     q.prof = nullptr;
+    q.zero = 0;
     const bool epi = bias != nullptr || act != SPINFER_ACT_NONE || (M % kGT) != 0 || (N % 8) != 0;
     auto go = [&]() {
         if (Np == 8) return epi ? launch_dw<1, true>(pl, st) : launch_dw<1, false>(pl, st);

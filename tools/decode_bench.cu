@@ -1,0 +1,405 @@
+// decode_bench.cu — microbenchmark of the SMBD decode loop alone (experiment tool, not product):
+// W warps per CTA, one CTA per SM, each warp decodes a synthetic GroupTile held in shared memory
+// (table + packed values + X slab) ITER times. Reports SM-cycles per BitmapTile (all warps) for
+// variants: 0 = simple (load_E -> issue -> assemble per 8-BT step), 1 = two-deep software
+// pipeline, 2 = 4-BT steps, 3 = simple without the value loads (table + MMA only),
+// 4 = simple without MMA.
+#include <cstdio>
+#include <cstdlib>
+#include <cstdint>
+#include <cuda_runtime.h>
+#include <cuda_fp16.h>
+#include "../paper_conf_eurosys_fanydlgww025_b200/csrc/ptx.cuh"
+using namespace spinfer;
+
+constexpr uint32_t kSelA = 0x7f62u, kSelB = 0x4cbfu, kSelC = 0x2333u;
+
+template <int NT>
+struct AccT {
+    float v[4][NT][4];
+};
+template <int NT>
+__device__ __noinline__ AccT<NT> decode_gt(AccT<NT> acc, uint32_t tbl_lane, uint32_t xs, uint32_t mulc) {
+    constexpr uint32_t cpr = NT;
+    uint32_t bfr[4][NT][2];
+#pragma unroll
+    for (int tc = 0; tc < 4; ++tc) {
+        const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+        if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
+        else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+    }
+#pragma unroll
+    for (int s8 = 0; s8 < 8; ++s8) {
+        uint4 E[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) E[k] = lds_v4(tbl_lane + (uint32_t)s8 * 64u + 16u * k);
+        uint32_t t0[8], t1[8], s1[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
+            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;   // first value of the half - 4 bytes
+            const uint32_t z = w * mulc;                               // top two bits: the lane's pair y
+            const uint32_t a = A + 2u * __popc(z);                     // &V[c2 - 2], c2 = MaskedPopCount + y0 + y1
+            const uint32_t y = z >> 30;
+            s1[k] = y * (y * kSelB + kSelA) + kSelC;
+            t0[k] = lds_u16(a);
+            t1[k] = lds_u16(a + 2u);
+        }
+        const int trb = 2 * (s8 & 1);
+#pragma unroll
+        for (int tt = 0; tt < 2; ++tt) {
+            uint32_t afr[4];
+#pragma unroll
+            for (int b = 0; b < 4; ++b) afr[b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) mma_16816(acc.v[trb + tt][nt], afr, bfr[s8 >> 1][nt][0], bfr[s8 >> 1][nt][1]);
+        }
+    }
+    return acc;
+}
+template <int NT>
+__device__ __noinline__ AccT<NT> decode_gt2(AccT<NT> acc, uint32_t tbl_lane, uint32_t xs, uint32_t mulc) {
+    constexpr uint32_t cpr = NT;
+    const uint32_t sA = opaque_u32(kSelA), sB = opaque_u32(kSelB), sC = opaque_u32(kSelC);
+    uint32_t bfr[4][NT][2];
+#pragma unroll
+    for (int tc = 0; tc < 4; ++tc) {
+        const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+        if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
+        else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+    }
+#pragma unroll
+    for (int s8 = 0; s8 < 8; ++s8) {
+        uint4 E[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) E[k] = lds_v4(tbl_lane + (uint32_t)s8 * 64u + 16u * k);
+        uint32_t t0[8], t1[8], s1[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
+            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;   // first value of the half - 4 bytes
+            const uint32_t z = w * mulc;                               // top two bits: the lane's pair y
+            const uint32_t a = A + 2u * __popc(z);                     // &V[c2 - 2], c2 = MaskedPopCount + y0 + y1
+            const uint32_t y = z >> 30;
+            s1[k] = y * (y * sB + sA) + sC;
+            t0[k] = lds_u16(a);
+            t1[k] = lds_u16(a + 2u);
+        }
+        const int trb = 2 * (s8 & 1);
+#pragma unroll
+        for (int tt = 0; tt < 2; ++tt) {
+            uint32_t afr[4];
+#pragma unroll
+            for (int b = 0; b < 4; ++b) afr[b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) mma_16816(acc.v[trb + tt][nt], afr, bfr[s8 >> 1][nt][0], bfr[s8 >> 1][nt][1]);
+        }
+    }
+    return acc;
+}
+template <int NT>
+__device__ __noinline__ AccT<NT> decode_gt3(AccT<NT> acc, uint32_t tbl_lane, uint32_t xs, uint32_t mulc) {
+    constexpr uint32_t cpr = NT;
+    uint32_t bfr[4][NT][2];
+    uint4 E[4];
+    uint32_t t0[8], t1[8], s1[8];
+#pragma unroll
+    for (int tc = 0; tc < 4; ++tc) {
+        const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
+        if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
+        else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+    }
+#pragma unroll
+    for (int s8 = 0; s8 < 8; ++s8) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) E[k] = lds_v4(tbl_lane + (uint32_t)s8 * 64u + 16u * k);
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
+            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;   // first value of the half - 4 bytes
+            const uint32_t z = w * mulc;                               // top two bits: the lane's pair y
+            const uint32_t a = A + 2u * __popc(z);                     // &V[c2 - 2], c2 = MaskedPopCount + y0 + y1
+            const uint32_t y = z >> 30;
+            s1[k] = y * (y * kSelB + kSelA) + kSelC;
+            t0[k] = lds_u16(a);
+            t1[k] = lds_u16(a + 2u);
+        }
+        const int trb = 2 * (s8 & 1);
+#pragma unroll
+        for (int tt = 0; tt < 2; ++tt) {
+            uint32_t afr[4];
+#pragma unroll
+            for (int b = 0; b < 4; ++b) afr[b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) mma_16816(acc.v[trb + tt][nt], afr, bfr[s8 >> 1][nt][0], bfr[s8 >> 1][nt][1]);
+        }
+    }
+    return acc;
+}
+
+
+__device__ volatile int g_stop;
+template <int VAR, int TB>
+__global__ void __launch_bounds__(TB, 1) k_dec(int iters, float *out, long long *cyc, const uint8_t *src, int tma) {
+    extern __shared__ __align__(1024) uint8_t sm[];
+    const uint32_t sb = smem_u32(sm);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    // layout: [0, 32K) values (random fp16), [32K, 64K) 2 tables per warp (16 warps), bitmaps at 58K, X at 60K (2 KB)
+    const uint32_t vals = sb, tblbase = sb + 24576, xs0 = sb + 61440;
+    // fill: values, X, and per-warp tables of a random 50 % GT
+    for (int i = threadIdx.x; i < 16384 + 1024; i += blockDim.x)
+        reinterpret_cast<uint16_t *>(sm)[i < 12288 ? i : 30720 + (i - 16384)] = (uint16_t)(0x3C00 | (i & 0x1FF));
+    __syncthreads();
+    {
+        // each warp builds its table from pseudo-random bitmaps (50 % density)
+        uint32_t h = 0x9E3779B9u * (warp + 1) + lane * 0x85EBCA6Bu;
+        auto rnd = [&]() { h ^= h << 13; h ^= h >> 17; h ^= h << 5; return h; };
+        const uint32_t a0 = rnd(), a1 = rnd(), b0 = rnd(), b1 = rnd();
+        const uint32_t pa = __popc(a0) + __popc(a1), pb = __popc(b0) + __popc(b1);
+        uint32_t packed = pa | (pb << 16), incl = packed;
+        for (int o = 1; o < 32; o <<= 1) { uint32_t y = __shfl_up_sync(~0u, incl, o); incl += lane >= o ? y : 0u; }
+        const uint32_t tot = __shfl_sync(~0u, incl, 31), excl = incl - packed;
+        const uint32_t vsm = vals + (warp * 2048) % 16384;
+        const uint32_t Aa = vsm + 2u * (excl & 0xFFFFu) - 4u + 8, Ab = vsm + 2u * ((tot & 0xFFFF) + (excl >> 16)) - 4u + 8;
+        for (int bsel = 0; bsel < 2; ++bsel) {
+            const uint32_t te = tblbase + (warp * 2 + bsel) * 1024 + 8 * lane;
+            sts_v2(te, a0, Aa); sts_v2(te + 512, a1, Aa + 2 * __popc(a0));
+            sts_v2(te + 256, b0, Ab); sts_v2(te + 768, b1, Ab + 2 * __popc(b0));
+        }
+        if (warp < 8) { sts_v2(sb + 59392 + warp * 512 + 8 * lane, a0, a1); sts_v2(sb + 59392 + warp * 512 + 256 + 8 * lane, b0, b1); }
+    }
+    __syncthreads();
+    const int nw = blockDim.x >> 5;
+    if (tma && warp == nw - 1) {   // background bulk-copy stream (the producer's smem write traffic)
+        if (lane == 0) {
+            const uint32_t bars = sb + 65536 + 4 * 32768;
+            for (int s2 = 0; s2 < 4; ++s2) mbar_init(bars + 8 * s2, 1);
+            fence_barrier_init();
+            const uint8_t *base = src + (size_t)blockIdx.x * (256u << 10);
+            for (int i = 0; i < 100000; ++i) {
+                const int sl = i & 3;
+                if (i >= 4) mbar_wait(bars + 8 * sl, ((i >> 2) - 1) & 1);
+                if (*(volatile int *)&g_stop) break;
+                mbar_arrive_expect_tx(bars + 8 * sl, 32768);
+                bulk_g2s(sb + 65536 + sl * 32768, base + (size_t)(i % 8) * 32768, 32768, bars + 8 * sl, policy_evict_first());
+            }
+        }
+        return;
+    }
+    const uint32_t tbl_lane = tblbase + warp * 2048 + (lane >> 4) * 512;
+    const uint32_t mulc = opaque_u32(1u << (30u - 2u * (uint32_t)(lane & 15)));
+    const uint32_t selA = opaque_u32(kSelA), selB = opaque_u32(kSelB), selC = opaque_u32(kSelC);
+    const uint32_t rr = lane & 7, mk = (lane >> 3) & 1, mn = (lane >> 4) & 1;
+    const uint32_t xs = xs0 + (mk * 8u + rr) * 32u + ((mn ^ ((rr >> 2) & 1u)) * 16u);
+    float acc[4][2][4];
+    for (int a = 0; a < 4; ++a) for (int b = 0; b < 2; ++b) for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
+    uint4 E[4];
+    auto load_E = [&](uint32_t tb) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) E[k] = lds_v4(tb + 16u * k);
+    };
+    auto issue_to = [&](uint32_t (&u0)[8], uint32_t (&u1)[8], uint32_t (&sl)[8]) {
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
+            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;
+            const uint32_t z = w * mulc;
+            const uint32_t a = A + 2u * __popc(z);
+            const uint32_t y = z >> 30;
+            sl[k] = y * (y * selB + selA) + selC;
+            if (VAR == 3) { u0[k] = a; u1[k] = z; }
+            else { u0[k] = lds_u16(a); u1[k] = lds_u16(a + 2u); }
+        }
+    };
+    auto assemble_from = [&](const uint32_t (&u0)[8], const uint32_t (&u1)[8], const uint32_t (&sl)[8], int trb,
+                             const uint32_t (&bfr)[2][2]) {
+#pragma unroll
+        for (int tt = 0; tt < 2; ++tt) {
+            uint32_t afr[4];
+#pragma unroll
+            for (int b = 0; b < 4; ++b) afr[b] = prmt(u0[tt * 4 + b], u1[tt * 4 + b], sl[tt * 4 + b]);
+            if (VAR == 4) { acc[trb + tt][0][0] += __uint_as_float(afr[0] ^ afr[1] ^ afr[2] ^ afr[3]); continue; }
+#pragma unroll
+            for (int nt = 0; nt < 2; ++nt) mma_16816(acc[trb + tt][nt], afr, bfr[nt][0], bfr[nt][1]);
+        }
+    };
+    __syncthreads();
+    const long long t0 = clock64();
+    for (int it = 0; it < iters; ++it) {
+        if constexpr (VAR == 1) {
+            uint32_t bfr[2][2][2];
+            uint32_t tA0[8], tA1[8], sA[8], tB0[8], tB1[8], sB[8];
+            ldsm_x4_trans(xs, bfr[0][0][0], bfr[0][0][1], bfr[0][1][0], bfr[0][1][1]);
+            load_E(tbl_lane);
+            issue_to(tA0, tA1, sA);
+            load_E(tbl_lane + 64u);
+#pragma unroll
+            for (int s = 0; s < 8; ++s) {
+                if (s + 1 < 8) { if (s & 1) issue_to(tA0, tA1, sA); else issue_to(tB0, tB1, sB); }
+                if (s + 2 < 8) load_E(tbl_lane + (uint32_t)(s + 2) * 64u);
+                if ((s & 1) && s + 1 < 8) { const int tc = (s + 1) >> 1; ldsm_x4_trans(xs + tc * 512, bfr[tc & 1][0][0], bfr[tc & 1][0][1], bfr[tc & 1][1][0], bfr[tc & 1][1][1]); }
+                if (s & 1) assemble_from(tB0, tB1, sB, 2, bfr[(s >> 1) & 1]);
+                else assemble_from(tA0, tA1, sA, 0, bfr[(s >> 1) & 1]);
+            }
+        } else if constexpr (VAR == 50) {
+            AccT<2> a_;
+            for (int a = 0; a < 4; ++a) for (int b = 0; b < 2; ++b) for (int e = 0; e < 4; ++e) a_.v[a][b][e] = acc[a][b][e];
+            a_ = decode_gt<2>(a_, tbl_lane, xs, mulc);
+            for (int a = 0; a < 4; ++a) for (int b = 0; b < 2; ++b) for (int e = 0; e < 4; ++e) acc[a][b][e] = a_.v[a][b][e];
+        } else if constexpr (VAR == 51 || VAR == 52) {
+            AccT<2> a_;
+            for (int a = 0; a < 4; ++a) for (int b = 0; b < 2; ++b) for (int e = 0; e < 4; ++e) a_.v[a][b][e] = acc[a][b][e];
+            if (VAR == 51) a_ = decode_gt2<2>(a_, tbl_lane, xs, mulc); else a_ = decode_gt3<2>(a_, tbl_lane, xs, mulc);
+            for (int a = 0; a < 4; ++a) for (int b = 0; b < 2; ++b) for (int e = 0; e < 4; ++e) acc[a][b][e] = a_.v[a][b][e];
+        } else if constexpr (VAR >= 40 && VAR < 50) {
+            constexpr int K = (VAR - 40) * 4;   // live dummy registers
+            uint32_t dummy[K > 0 ? K : 1];
+#pragma unroll
+            for (int k = 0; k < K; ++k) dummy[k] = opaque_u32(it * 7 + k + lane);
+            uint32_t bfr[4][2][2];
+#pragma unroll
+            for (int tc = 0; tc < 4; ++tc) ldsm_x4_trans(xs + tc * 512, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+            uint32_t T0[8], T1[8], SS[8];
+#pragma unroll
+            for (int s8 = 0; s8 < 8; ++s8) {
+                load_E(tbl_lane + (uint32_t)s8 * 64u);
+                issue_to(T0, T1, SS);
+                assemble_from(T0, T1, SS, 2 * (s8 & 1), bfr[s8 >> 1]);
+            }
+            uint32_t x = 0;
+#pragma unroll
+            for (int k = 0; k < K; ++k) x ^= dummy[k];
+            if (x == 0x12345678u) acc[0][0][0] += 1.f;
+        } else if constexpr (VAR == 30 || VAR == 31 || VAR == 32) {
+            // explicit two-phase schedule: loads + PRMT of H BTs into afr (compiler barrier), then
+            // their MMAs. VAR 30: H = 32 (half GT), 31: H = 64, 32: H = 16
+            constexpr int SH = VAR == 31 ? 8 : VAR == 30 ? 4 : 2;   // steps per phase
+            uint32_t bfr[4][2][2];
+#pragma unroll
+            for (int tc = 0; tc < 4; ++tc) ldsm_x4_trans(xs + tc * 512, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+#pragma unroll
+            for (int ph0 = 0; ph0 < 8; ph0 += SH) {
+                uint32_t afr[SH][2][4];
+#pragma unroll
+                for (int k = 0; k < SH; ++k) {
+                    uint32_t T0[8], T1[8], SS[8];
+                    load_E(tbl_lane + (uint32_t)(ph0 + k) * 64u);
+                    issue_to(T0, T1, SS);
+#pragma unroll
+                    for (int tt = 0; tt < 2; ++tt)
+#pragma unroll
+                        for (int b = 0; b < 4; ++b) afr[k][tt][b] = prmt(T0[tt * 4 + b], T1[tt * 4 + b], SS[tt * 4 + b]);
+                }
+#pragma unroll
+                for (int k = 0; k < SH; ++k)
+#pragma unroll
+                    for (int tt = 0; tt < 2; ++tt)
+                        asm volatile("" : "+r"(afr[k][tt][0]), "+r"(afr[k][tt][1]), "+r"(afr[k][tt][2]), "+r"(afr[k][tt][3]));
+#pragma unroll
+                for (int k = 0; k < SH; ++k) {
+                    const int s8 = ph0 + k;
+#pragma unroll
+                    for (int tt = 0; tt < 2; ++tt)
+#pragma unroll
+                        for (int nt = 0; nt < 2; ++nt) mma_16816(acc[2 * (s8 & 1) + tt][nt], afr[k][tt], bfr[s8 >> 1][nt][0], bfr[s8 >> 1][nt][1]);
+                }
+            }
+        } else if constexpr (VAR == 20 || VAR == 21) {
+            // scan of the next GT (bitmaps from smem, 32-lane shuffle scan, table writes into the
+            // other buffer) in the same region as this GT's decode
+            const uint32_t tb_cur = tblbase + (warp * 2 + (it & 1)) * 1024, tb_nxt = tblbase + (warp * 2 + ((it + 1) & 1)) * 1024;
+            const uint32_t bms = sb + 59392 + (warp & 7) * 512;   // static bitmaps (any bits)
+            const uint2 ba = lds_v2(bms + 8 * lane), bb = lds_v2(bms + 256 + 8 * lane);
+            uint32_t bfr[4][2][2];
+#pragma unroll
+            for (int tc = 0; tc < 4; ++tc) ldsm_x4_trans(xs + tc * 512, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+            uint32_t T0[8], T1[8], SS[8];
+            const uint32_t tl = tb_cur + (lane >> 4) * 512;
+            uint32_t pax = __popc(ba.x), pbx = __popc(bb.x);
+            uint32_t packed = (pax + __popc(ba.y)) | ((pbx + __popc(bb.y)) << 16), incl = packed;
+#pragma unroll
+            for (int s8 = 0; s8 < 8; ++s8) {
+                load_E(tl + (uint32_t)s8 * 64u);
+                issue_to(T0, T1, SS);
+                if (VAR == 20 && s8 < 5) { const uint32_t y = __shfl_up_sync(~0u, incl, 1 << s8); incl += lane >= (1 << s8) ? y : 0u; }
+                assemble_from(T0, T1, SS, 2 * (s8 & 1), bfr[s8 >> 1]);
+            }
+            if (VAR == 21) {
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) { const uint32_t y = __shfl_up_sync(~0u, incl, o); incl += lane >= o ? y : 0u; }
+            }
+            const uint32_t tot = __shfl_sync(~0u, incl, 31), excl = incl - packed;
+            const uint32_t vsm = vals + (warp * 2048) % 16384;
+            const uint32_t Aa = vsm + 2u * (excl & 0xFFFFu) - 4u + 8, Ab = vsm + 2u * ((tot & 0xFFFF) + (excl >> 16)) - 4u + 8;
+            const uint32_t te = tb_nxt + 8 * lane;
+            sts_v2(te, ba.x, Aa); sts_v2(te + 512, ba.y, Aa + 2 * pax);
+            sts_v2(te + 256, bb.x, Ab); sts_v2(te + 768, bb.y, Ab + 2 * pbx);
+            __syncwarp();
+        } else if constexpr (VAR >= 5) {
+            // depth P = VAR - 4 steps of 8 BTs in flight, fenced so the compiler cannot hoist more
+            constexpr int P = VAR >= 5 ? VAR - 4 : 1;
+            uint32_t T0[P][8], T1[P][8], SS[P][8];
+            uint32_t bfr[4][2][2];
+#pragma unroll
+            for (int tc = 0; tc < 4; ++tc) ldsm_x4_trans(xs + tc * 512, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
+#pragma unroll
+            for (int s = 0; s < 8 + P - 1; ++s) {
+                if (s < 8) { load_E(tbl_lane + (uint32_t)s * 64u); issue_to(T0[s % P], T1[s % P], SS[s % P]); }
+                const int sa = s - (P - 1);
+                if (sa >= 0) assemble_from(T0[sa % P], T1[sa % P], SS[sa % P], 2 * (sa & 1), bfr[sa >> 1]);
+                asm volatile("" ::: "memory");
+            }
+        } else {
+            uint32_t t0_[8], t1_[8], s1_[8];
+#pragma unroll 1
+            for (int tc = 0; tc < 4; ++tc) {
+                uint32_t bfr[2][2];
+                ldsm_x4_trans(xs + tc * 512, bfr[0][0], bfr[0][1], bfr[1][0], bfr[1][1]);
+#pragma unroll
+                for (int hh = 0; hh < 2; ++hh) {
+                    load_E(tbl_lane + (uint32_t)(tc * 16 + hh * 8) * 8u);
+                    issue_to(t0_, t1_, s1_);
+                    assemble_from(t0_, t1_, s1_, 2 * hh, bfr);
+                }
+            }
+        }
+    }
+    __syncthreads();
+    const long long t1 = clock64();
+    float s = 0;
+    for (int a = 0; a < 4; ++a) for (int b = 0; b < 2; ++b) for (int e = 0; e < 4; ++e) s += acc[a][b][e];
+    if (s == 1234.5f) out[0] = s;
+    if (threadIdx.x == 0) { cyc[blockIdx.x] = t1 - t0; g_stop = 1; }
+}
+
+template <int VAR, int TB = 640>
+void run(int warps, int iters, int tma = 0) {
+    float *out; long long *cyc; cudaMalloc(&out, 4); cudaMalloc(&cyc, 8 * 148);
+    static uint8_t *src = nullptr; if (!src) { cudaMalloc(&src, 64ull << 20); cudaMemset(src, 1, 64ull << 20); }
+    const int smem = tma ? 65536 + 4 * 32768 + 64 : 64 * 1024;
+    cudaFuncSetAttribute(k_dec<VAR, TB>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    const int nt = (warps + (tma ? 1 : 0)) * 32;
+    int zero = 0;
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    float ms = 0;
+    for (int rep = 0; rep < 2; ++rep) {
+        cudaMemcpyToSymbol(g_stop, &zero, 4);
+        cudaEventRecord(e0);
+        k_dec<VAR, TB><<<148, nt, smem>>>(iters, out, cyc, src, tma);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        cudaEventElapsedTime(&ms, e0, e1);
+    }
+    printf("   wall %.1f us -> %.3f ns per BT per SM\n", ms * 1e3, ms * 1e6 / ((double)warps * iters * 64));
+    cudaDeviceSynchronize();
+    long long h[148]; cudaMemcpy(h, cyc, sizeof(h), cudaMemcpyDeviceToHost);
+    double m = 0; for (int i = 0; i < 148; ++i) m += h[i]; m /= 148;
+    printf("tma %d var %d tb %d warps %2d: %.3f SM-cycles per BitmapTile (%s)\n", tma, VAR, TB, warps, m / ((double)warps * iters * 64),
+           cudaGetErrorString(cudaGetLastError()));
+    cudaFree(out); cudaFree(cyc);
+}
+
+int main() {
+    for (int w : {16}) { run<0>(w, 200); run<5>(w, 200); }
+    return 0;
+}
