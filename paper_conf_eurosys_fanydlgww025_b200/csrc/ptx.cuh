@@ -81,6 +81,14 @@ __device__ __forceinline__ bool mbar_test_wait(uint32_t bar, uint32_t parity) {
 __device__ __forceinline__ void mbar_wait_poll(uint32_t bar, uint32_t parity, uint32_t ns) {
     while (!mbar_test_wait(bar, parity)) __nanosleep(ns);
 }
+// Exponential back-off between probes, from ns0 up to ns_max.
+__device__ __forceinline__ void mbar_wait_expo(uint32_t bar, uint32_t parity, uint32_t ns0, uint32_t ns_max) {
+    uint32_t ns = ns0;
+    while (!mbar_test_wait(bar, parity)) {
+        __nanosleep(ns);
+        ns = ns < ns_max ? 2 * ns : ns_max;
+    }
+}
 // For waiters that usually block for a long time (scan on data, producer on a free slot):
 // the hinted try_wait sleeps until ANY mbarrier event of the CTA, i.e. it wakes ~25 times
 // per stage; a timed back-off (plain nanosleep, not woken by barrier traffic) polls a few times.

@@ -41,6 +41,18 @@ constexpr int kCWd = 16;                  // consumer warps: r = w >> 3, m = w &
 constexpr int kProdWarp0 = kCWd;          // producer warps kCWd, kCWd + 2 (SMSPs 0 and 2)
 constexpr int kNProd = 2;                 // stage i is issued by producer i % 2
 constexpr int kRedWarp = kCWd + 1;        // reducer warp (SMSP 1)
+// producer back-off between probes of a slot's empty barrier (ns): first, maximum
+#ifndef SPINFER_DW_PNS0
+#define SPINFER_DW_PNS0 64u
+#endif
+#ifndef SPINFER_DW_PNS1
+#define SPINFER_DW_PNS1 1024u
+#endif
+// slot release through hardware named barriers (ids kBarIdSlot0 + slot) instead of mbarriers
+#ifndef SPINFER_DW_NBAR
+#define SPINFER_DW_NBAR 1
+#endif
+constexpr uint32_t kBarIdSlot0 = 3;   // 0: __syncthreads, 1-2: final-segment reduction
 #ifndef SPINFER_DW_VSCAN
 #define SPINFER_DW_VSCAN 0
 #endif
@@ -447,6 +459,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         it.init(u0, u1, KG, G, MG);
         int nseg = 0, i = 0;
         uint32_t pslot = 0, pph = 0;   // ring position of stage i
+        uint32_t owners_pk = 0;        // 4 bits per slot: GT owners of the stage last issued into it
         auto step = [&](Stages &s, int &ns, int &ii) {   // one stage forward (segment count, index)
             if (s.seg_last(KG)) ++ns;
             s.next(KG, G, MG);
@@ -476,12 +489,19 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             const uint32_t slot = pslot, ph = pph;
             pf.lap(1);
             if (lane == 0) pf.st(prm.prof, p, i, 3, true);
-            if (i >= S) mbar_wait_poll(bar_empty + 8 * slot, ph ^ 1u, 128u);
+#if SPINFER_DW_NBAR
+            // the slot's previous stage (i - S) released by its GT owners: hardware named barrier
+            // (the waiting warp is not woken by the CTA's mbarrier traffic, no polling)
+            if (i >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + ((owners_pk >> (4 * slot)) & 15u)));
+#else
+            if (i >= S) mbar_wait_expo(bar_empty + 8 * slot, ph ^ 1u, SPINFER_DW_PNS0, SPINFER_DW_PNS1);
+#endif
             pf.lap(0);
             if (lane == 0) pf.st(prm.prof, p, i, 0, true);
             const uint32_t st = ring + slot * prm.slot_bytes, fb = bar_full + 8 * slot;
             const uint32_t hb = sbase + kOffHdr + slot * kHdrBytes;
             const int g = it.g, rows = it.rows;
+            owners_pk = (owners_pk & ~(15u << (4 * slot))) | ((uint32_t)(rows * g) << (4 * slot));
             // validate the stage's value ranges (never trust the caller's max_gt_values)
             const int obeg = __shfl_sync(0xffffffffu, oc, lane & 8);
             const int oend = __shfl_sync(0xffffffffu, oc, (lane & 8) + g);
@@ -512,9 +532,11 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                 // one arrival with every transaction byte registered up front: the phase completes
                 // only when all copies of the stage have landed (release: the header stores above)
                 mbar_arrive_expect_tx(fb, (uint32_t)rows * bmb + xbytes + vbl + vb1);
+#if !SPINFER_DW_NBAR
                 // the empty barrier expects kRd * kMaxGd arrivals: one per GT owner of the stage, the rest now
                 const uint32_t owners = (uint32_t)(rows * g);
                 if (owners < (uint32_t)(kRd * kMaxGd)) mbar_arrive_cnt(bar_empty + 8 * slot, (uint32_t)(kRd * kMaxGd) - owners);
+#endif
             }
             pf.lap(3);
             uint32_t dst = 0, bytes = 0;
@@ -546,7 +568,11 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         {
             if ((i & 1) != q) ++i;   // the loop can stop one index short of this producer's parity
             const uint32_t slot = (uint32_t)(i % S), ph = (uint32_t)(i / S) & 1u;
+#if SPINFER_DW_NBAR
+            if (i >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + ((owners_pk >> (4 * slot)) & 15u)));
+#else
             if (i >= S) mbar_wait_poll(bar_empty + 8 * slot, ph ^ 1u, 128u);
+#endif
             if (lane == 0) {
                 sts_v4(sbase + kOffHdr + slot * kHdrBytes, make_uint4(0u, kHdrStop, (uint32_t)nseg, 0u));
                 mbar_arrive(bar_full + 8 * slot);
@@ -577,7 +603,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             const bool complete = sstart == rb * KG && send == (rb + 1) * KG;
             for (int r = 0; r < rows; ++r) {
                 pf.lap(1);
-                mbar_wait_poll(bar_sfull + 16 * k + 8 * r, par, 512u);
+                mbar_wait_expo(bar_sfull + 16 * k + 8 * r, par, 256u, 4096u);
                 pf.lap(0);
                 const uint32_t cmask = lds_u32(seg_mask + 8 * k + 4 * r);   // warps that own a GT of the segment
                 if (lane == 0) sts_u32(seg_mask + 8 * k + 4 * r, 0u);
@@ -1169,7 +1195,11 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                 atomicOr(prm.ws_err, 2);   // corrupt GT (or poisoned stage): skipped, Y is not valid
             }
             __syncwarp();
+#if SPINFER_DW_NBAR
+            named_bar_arrive(kBarIdSlot0 + slot, 32u * (1u + (uint32_t)(rows * g)));   // the slot's GT owners + its producer
+#else
             if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
+#endif
             if (lane == 0) pf.st(prm.prof, p, i, 2, true);
             if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 5);
         }
@@ -1296,7 +1326,9 @@ bool make_dplan(int M, int K, int Np, int max_gt_values, DPlan *pl) {
         const uint32_t st_bm = al((uint32_t)G * 64 * Np * 2, 128);
         const uint32_t vcap = al((uint32_t)G * maxv * 2, 128);
         const uint32_t slot = al(st_bm + kRd * G * 512 + 2 * vcap, 1024);
-        const int S = (int)std::min<long long>(smax, ((long long)smem_max - kOffRing - 1024) / slot);
+        // an even slot count: producer q always refills its own stages' slots (the slot release
+        // barrier counts the GT owners of the stage that producer issued there)
+        const int S = (int)std::min<long long>(smax, ((long long)smem_max - kOffRing - 1024) / slot) & ~1;
         if ((uint32_t)S * slot < final_scratch) continue;
         if (S >= 4) { bestG = G; bestS = S; break; }
         if (S >= 2 && S > bestS) { bestG = G; bestS = S; }
