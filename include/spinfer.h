@@ -98,13 +98,15 @@ SPINFER_API int spinfer_encode_fill(const uint16_t *W, const spinfer_tca *T, voi
 SPINFER_API int spinfer_decode(const spinfer_tca *T, uint16_t *W_out, void *stream);
 
 /* Bytes of device workspace spinfer_spmm needs for this shape: a fixed 64 KiB
- * region of split-K fix-up counters (one int32 per GT row; M <= 1,048,576)
- * followed by fp32 split-K partials and, when N is not a multiple of 8, a
- * zero-padded copy of X (K x roundup(N, 8) fp16). 0 for an invalid shape. The workspace must
- * be ZERO-FILLED before its first use; every spinfer_spmm call leaves the
- * counter region zero again, so one zeroed workspace (sized for the largest
- * shape) can be reused by successive calls of any shape on ONE stream — never
- * by two calls that may run concurrently. */
+ * region of split-K fix-up counters (one int32 per GT row; ceil(M/64) < 16383)
+ * whose last int32 (byte offset 65532) is the ERROR WORD, followed by fp32
+ * split-K partials and, when N is not a multiple of 8, a zero-padded copy of X
+ * (K x roundup(N, 8) fp16). 0 for an invalid shape. The workspace must be
+ * ZERO-FILLED before its first use; every spinfer_spmm call leaves the counter
+ * region zero again, so one zeroed workspace (sized for the largest shape) can
+ * be reused by successive calls of any shape on ONE stream — never by two calls
+ * that may run concurrently. The grid (and so the partials' size) depends on
+ * the device's SM count and SPINFER_OPT_MAX_CTAS: query after setting options. */
 SPINFER_API size_t spinfer_spmm_workspace_bytes(int M, int K, int N);
 
 /* Y = W x X with fp32 accumulation and one round-to-nearest-even to
@@ -140,6 +142,35 @@ SPINFER_API int spinfer_tp_rows(int M, int world, int rank, int *row_begin /* ho
  * (e.g. NCCL all-gather) when the next layer needs it. */
 SPINFER_API int spinfer_spmm_tp(const spinfer_tca *T_shard, const uint16_t *X, uint16_t *Y_full, int M_full,
                     int K, int N, int world, int rank, void *workspace, size_t ws_bytes, void *stream);
+
+/* Corrupt-input report. The kernels check every stage they load against the TCA-BME
+ * invariants (gtile_offset non-decreasing and <= n_values, a GroupTile's popcount equal to
+ * its padded value count rounded down by < 8, at most max_gt_values values per GroupTile):
+ * a violating stage is not copied / decoded (its rows' contribution is zero, so Y is NOT
+ * valid) and a flag is OR-ed into the workspace's error word — 1: gtile_offset out of range
+ * or larger than max_gt_values; 2: bitmaps inconsistent with gtile_offset. No out-of-bounds
+ * access happens either way. This call copies the error word to *flags (host), resets it to
+ * 0 and synchronizes `stream`. */
+SPINFER_API int spinfer_spmm_check(void *workspace, int32_t *flags /* host */, void *stream);
+
+/* Process-wide options (tests, ablation, tuning). 0 is every option's default. Not
+ * synchronized with calls running on other host threads: set them before launching work.
+ *   SPINFER_OPT_KERNEL    0 auto (N <= 16: the mma.sync decoupled-warp kernel, else tcgen05),
+ *                         1 force the decoupled-warp kernel (N <= 16 only), 2 force tcgen05;
+ *   SPINFER_OPT_MAX_CTAS  cap on the persistent grid (0: one CTA per SM);
+ *   SPINFER_OPT_STAGE_G   cap on GroupTile columns per pipeline stage (0: the kernel's max);
+ *   SPINFER_OPT_STAGE_S   cap on pipeline stages (0: as many as shared memory holds).
+ * SPINFER_EINVAL for an unknown key or an out-of-range value. */
+#define SPINFER_OPT_KERNEL 0
+#define SPINFER_OPT_MAX_CTAS 1
+#define SPINFER_OPT_STAGE_G 2
+#define SPINFER_OPT_STAGE_S 3
+#define SPINFER_OPT_COUNT 4
+#define SPINFER_KERNEL_AUTO 0
+#define SPINFER_KERNEL_DW 1
+#define SPINFER_KERNEL_TC 2
+SPINFER_API int spinfer_set_option(int key, int value);
+SPINFER_API int spinfer_get_option(int key);
 
 /* Static string for a status code. */
 SPINFER_API const char *spinfer_status_str(int status);

@@ -246,9 +246,13 @@ def tp_rows(M: int, world: int, rank: int):
 
 def shard(T: TCA, row_begin: int, row_count: int) -> TCA:
     """Row shard of an encoding as a contiguous slice of all three arrays with
-    GTileOffset rebased: GT rows [a, b) are GTs [a*KG, b*KG)."""
-    KG = T.K // GT
-    a, b = row_begin // GT, (row_begin + row_count) // GT
+    GTileOffset rebased: GT rows [a, b) are GTs [a*KG, b*KG).
+    Ragged shapes are zero-padded to whole GroupTiles (A8): KG = ceil(K / 64) and a
+    shard ending at a ragged M owns the partial last GT row, b = ceil((row_begin + row_count) / 64)."""
+    if row_begin % GT or (row_count % GT and row_begin + row_count != T.M):
+        raise ValueError("shard rows must be whole GT rows (except a ragged tail ending at M)")
+    KG = -(-T.K // GT)
+    a, b = row_begin // GT, -(-(row_begin + row_count) // GT)
     off = T.gtile_offset[a * KG: b * KG + 1].astype(np.int64)
     base = int(off[0])
     vals = T.values[base: int(off[-1])].copy()

@@ -15,7 +15,8 @@ from dataclasses import dataclass
 import torch
 
 __all__ = ["TCA", "SpinferError", "encode", "decode", "spmm", "spmm_tp", "tp_rows", "workspace",
-           "workspace_bytes", "storage_bytes", "algorithmic_bytes", "lib", "LIB_PATH"]
+           "workspace_bytes", "storage_bytes", "algorithmic_bytes", "check", "set_option", "get_option",
+           "lib", "LIB_PATH"]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("SPINFER_LIB") or os.path.join(_PKG, "libspinfer.so")   # SPINFER_LIB: experiments only
@@ -42,7 +43,12 @@ _lib = None
 
 # Exported symbols (must match include/spinfer.h; checked by tests/test_abi.py).
 SYMBOLS = ["spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spinfer_spmm_workspace_bytes",
-           "spinfer_spmm", "spinfer_spmm_ex", "spinfer_tp_rows", "spinfer_spmm_tp", "spinfer_status_str", "spinfer_version"]
+           "spinfer_spmm", "spinfer_spmm_ex", "spinfer_tp_rows", "spinfer_spmm_tp", "spinfer_spmm_check",
+           "spinfer_set_option", "spinfer_get_option", "spinfer_status_str", "spinfer_version"]
+
+# spinfer.h SPINFER_OPT_* / SPINFER_KERNEL_*
+OPTIONS = {"kernel": 0, "max_ctas": 1, "stage_g": 2, "stage_s": 3}
+KERNELS = {"auto": 0, "dw": 1, "tc": 2}
 
 
 def lib() -> ctypes.CDLL:
@@ -65,11 +71,14 @@ def lib() -> ctypes.CDLL:
     L.spinfer_spmm_ex.argtypes = [P(_Tca), vp, vp, i32, i32, i32, vp, i32, vp, sz, vp]
     L.spinfer_tp_rows.argtypes = [i32, i32, i32, P(ctypes.c_int), P(ctypes.c_int)]
     L.spinfer_spmm_tp.argtypes = [P(_Tca), vp, vp, i32, i32, i32, i32, i32, vp, sz, vp]
+    L.spinfer_spmm_check.argtypes = [vp, P(ctypes.c_int32), vp]
+    L.spinfer_set_option.argtypes = [i32, i32]
+    L.spinfer_get_option.argtypes = [i32]
     L.spinfer_status_str.argtypes = [i32]
     L.spinfer_status_str.restype = ctypes.c_char_p
     L.spinfer_version.restype = ctypes.c_char_p
-    for f in ("spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spinfer_spmm", "spinfer_tp_rows",
-              "spinfer_spmm_tp"):
+    for f in ("spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spinfer_spmm", "spinfer_spmm_ex",
+              "spinfer_tp_rows", "spinfer_spmm_tp", "spinfer_spmm_check", "spinfer_set_option", "spinfer_get_option"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -186,16 +195,45 @@ def workspace_bytes(M: int, K: int, N: int) -> int:
 _ws_cache: dict = {}
 
 
-def workspace(M: int, K: int, N: int, device=None) -> torch.Tensor:
-    """A zero-filled workspace for spinfer_spmm (cached per device; one stream at a time)."""
+def workspace(M: int, K: int, N: int, device=None, stream=None) -> torch.Tensor:
+    """A zero-filled workspace for spinfer_spmm, cached per (device, stream): calls on one stream
+    are ordered, so they may share one; two streams never do (spinfer.h)."""
     dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
     with torch.cuda.device(dev):
         need = max(int(lib().spinfer_spmm_workspace_bytes(M, K, N)), 256)
-    ws = _ws_cache.get(dev)
+        key = (dev, _stream(stream))
+    if need <= 256 and (M <= 0 or K <= 0 or not 1 <= N <= 32):
+        raise ValueError(f"no workspace for M/K/N = {M}/{K}/{N}")
+    ws = _ws_cache.get(key)
     if ws is None or ws.numel() < need:
         ws = torch.zeros(need, dtype=torch.uint8, device=dev)
-        _ws_cache[dev] = ws
+        _ws_cache[key] = ws
     return ws
+
+
+def check(ws: torch.Tensor, stream=None) -> int:
+    """The workspace's corrupt-input flags since the last check (spinfer_spmm_check; 0 = none:
+    1 = gtile_offset out of range, 2 = bitmaps inconsistent with gtile_offset), then resets them."""
+    flags = ctypes.c_int32()
+    with torch.cuda.device(ws.device):
+        _check(lib().spinfer_spmm_check(ws.data_ptr(), ctypes.byref(flags), _stream(stream)), "spinfer_spmm_check")
+    return int(flags.value)
+
+
+def set_option(name: str, value) -> None:
+    """Process-wide library option (spinfer.h spinfer_set_option): "kernel" ("auto" | "dw" | "tc"),
+    "max_ctas", "stage_g", "stage_s" (0 = default)."""
+    v = KERNELS[value] if name == "kernel" and isinstance(value, str) else int(value)
+    _check(lib().spinfer_set_option(OPTIONS[name], v), f"spinfer_set_option({name})")
+
+
+def get_option(name: str) -> int:
+    return int(lib().spinfer_get_option(OPTIONS[name]))
+
+
+def _same_device(X: torch.Tensor, name: str, t: torch.Tensor):
+    if t.device != X.device:
+        raise ValueError(f"{name} is on {t.device}, X on {X.device}")
 
 
 ACT_NONE, ACT_RELU = 0, 1   # spinfer.h SPINFER_ACT_*
@@ -206,18 +244,26 @@ def spmm(T: TCA, X: torch.Tensor, Y: torch.Tensor | None = None, ws: torch.Tenso
     """Y = act(W X + bias): X fp16 [K][N] (CUDA), 1 <= N <= 32; bias fp16 [M] or
     None; act None or "relu" (fused into the SpMM epilogue, spinfer_spmm_ex); returns fp16 [M][N]."""
     X = _dev_u16(X, "X")
+    if X.dim() != 2:
+        raise ValueError("X must be 2-D [K][N]")
     K, N = X.shape
     if K != T.K:
         raise ValueError(f"X has K={K}, W has K={T.K}")
+    _same_device(X, "W", T.bitmap)
     if Y is None:
         Y = torch.empty((T.M, N), dtype=torch.float16, device=X.device)
     Yv = _dev_u16(Y, "Y")
+    if tuple(Yv.shape) != (T.M, N):
+        raise ValueError(f"Y has shape {tuple(Yv.shape)}, expected {(T.M, N)}")
+    _same_device(X, "Y", Yv)
     if ws is None:
-        ws = workspace(T.M, T.K, N, X.device)
+        ws = workspace(T.M, T.K, N, X.device, stream)
+    _same_device(X, "workspace", ws)
     actc = {None: ACT_NONE, "none": ACT_NONE, "relu": ACT_RELU}[act]
     bptr = None
     if bias is not None:
         bv = _dev_u16(bias, "bias")
+        _same_device(X, "bias", bv)
         if bv.numel() != T.M:
             raise ValueError(f"bias has {bv.numel()} entries, W has M={T.M}")
         bptr = bv.data_ptr()
@@ -242,10 +288,17 @@ def spmm_tp(T_shard: TCA, X: torch.Tensor, Y_full: torch.Tensor, M_full: int, wo
             ws: torch.Tensor | None = None, stream=None) -> torch.Tensor:
     """Row-partitioned SpMM: writes rows tp_rows(M_full, world, rank) of Y_full [M_full][N]. No communication."""
     X = _dev_u16(X, "X")
+    if X.dim() != 2:
+        raise ValueError("X must be 2-D [K][N]")
     K, N = X.shape
     Yv = _dev_u16(Y_full, "Y_full")
+    if tuple(Yv.shape) != (M_full, N):
+        raise ValueError(f"Y_full has shape {tuple(Yv.shape)}, expected {(M_full, N)}")
+    _same_device(X, "Y_full", Yv)
+    _same_device(X, "W shard", T_shard.bitmap)
     if ws is None:
-        ws = workspace(max(T_shard.M, GT), K, N, X.device)
+        ws = workspace(max(T_shard.M, GT), K, N, X.device, stream)
+    _same_device(X, "workspace", ws)
     cs = T_shard.c_struct()
     with torch.cuda.device(X.device):
         _check(lib().spinfer_spmm_tp(ctypes.byref(cs), X.data_ptr(), Yv.data_ptr(), M_full, K, N, world, rank,

@@ -25,6 +25,7 @@ int validate_tca(const spinfer_tca *T, int M, int K) {
     if (T->M != M || T->K != K || T->gt_h != kGT || T->gt_w != kGT || !shape_ok(M, K)) return SPINFER_EINVAL;
     if (T->n_values < 0) return SPINFER_EINVAL;
     if (T->n_values >= (1LL << 31)) return SPINFER_EOVERFLOW;
+    if (T->max_gt_values > kGT * kGT) return SPINFER_EINVAL;
     if (!aligned16(T->gtile_offset) || !aligned16(T->bitmap) || !aligned16(T->values)) return SPINFER_EINVAL;
     return SPINFER_OK;
 }
@@ -124,6 +125,23 @@ int spinfer_spmm_tp(const spinfer_tca *T_shard, const uint16_t *X, uint16_t *Y_f
     return spinfer_spmm(T_shard, X, Y_full + (size_t)b * N, c, K, N, workspace, ws_bytes, stream);
 }
 
+int spinfer_spmm_check(void *workspace, int32_t *flags, void *stream) {
+    if (!workspace || !flags || !aligned16(workspace)) return SPINFER_EINVAL;
+    int rc = check_device();
+    if (rc) return rc;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    int32_t *err = reinterpret_cast<int32_t *>(workspace) + kErrWord;
+    if (cudaMemcpyAsync(flags, err, 4, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        cudaMemsetAsync(err, 0, 4, st) != cudaSuccess || cudaStreamSynchronize(st) != cudaSuccess) {
+        cudaGetLastError();
+        return SPINFER_ECUDA;
+    }
+    return SPINFER_OK;
+}
+
+int spinfer_set_option(int key, int value) { return set_option(key, value); }
+int spinfer_get_option(int key) { return option(key); }
+
 const char *spinfer_status_str(int status) {
     switch (status) {
         case SPINFER_OK: return "SPINFER_OK";
@@ -136,6 +154,6 @@ const char *spinfer_status_str(int status) {
     }
 }
 
-const char *spinfer_version(void) { return "spinfer-b200 0.1 (sm_100a; TCA-BME GT=64; mma.sync SMBD)"; }
+const char *spinfer_version(void) { return "spinfer-b200 0.2 (sm_100a; TCA-BME GT=64; SMBD: mma.sync N<=16, tcgen05 N>16)"; }
 
 }  // extern "C"

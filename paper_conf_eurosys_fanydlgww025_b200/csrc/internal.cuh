@@ -26,6 +26,8 @@ constexpr size_t kCounterRegion = 65536;
 constexpr int kErrWord = 16383;
 
 // spmm.cu
+int option(int key);                     // spinfer_set_option values (0 = default)
+int set_option(int key, int value);
 int sm_count();                          // SMs of the current device (cached per device)
 int choose_grid(long long units);        // persistent grid size: min(SMs, units)
 int make_x_tmap(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows, bool swizzle);
@@ -33,6 +35,11 @@ int launch_pad_x(const uint16_t *X, uint16_t *Xp, int K, int N, int Np, cudaStre
 size_t spmm_workspace_bytes(int M, int K, int N);
 int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias, int act, void *ws,
                 size_t ws_bytes, cudaStream_t st);
+
+// spmm_tc.cu (tcgen05 kernel, N 17..32)
+size_t spmm_tc_workspace_bytes(int M, int K, int N);
+int launch_spmm_tc(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias,
+                   int act, void *ws, size_t ws_bytes, cudaStream_t st);
 
 // spmm_dw.cu (decoupled-warp kernel, N <= 16)
 size_t spmm_dw_workspace_bytes(int M, int K, int N);

@@ -41,32 +41,12 @@ constexpr int kCWd = 16;                  // consumer warps: r = w >> 3, m = w &
 constexpr int kProdWarp0 = kCWd;          // producer warps kCWd, kCWd + 2 (SMSPs 0 and 2)
 constexpr int kNProd = 2;                 // stage i is issued by producer i % 2
 constexpr int kRedWarp = kCWd + 1;        // reducer warp (SMSP 1)
-// producer back-off between probes of a slot's empty barrier (ns): first, maximum
-#ifndef SPINFER_DW_PNS0
-#define SPINFER_DW_PNS0 64u
-#endif
-#ifndef SPINFER_DW_PNS1
-#define SPINFER_DW_PNS1 1024u
-#endif
-// slot release through hardware named barriers (ids kBarIdSlot0 + slot) instead of mbarriers
-#ifndef SPINFER_DW_NBAR
-#define SPINFER_DW_NBAR 1
-#endif
+// slot release: hardware named barriers (ids kBarIdSlot0 + slot), not mbarriers — a warp
+// suspended on an mbarrier try_wait is re-woken by every mbarrier event of the CTA
 constexpr uint32_t kBarIdSlot0 = 3;   // 0: __syncthreads, 1-2: final-segment reduction
-#ifndef SPINFER_DW_VSCAN
-#define SPINFER_DW_VSCAN 0
-#endif
-#ifndef SPINFER_DW_PIPE
-#define SPINFER_DW_PIPE 2
-#endif
-#ifndef SPINFER_DW_REG
-#define SPINFER_DW_REG 0
-#endif
-// register split (setmaxnreg, per warpgroup of 4 warps): with 20 warps each SM sub-partition
-// holds 4 consumer warps + 1 role warp; setmaxnreg.inc is served only from what the role
-// warpgroup released, so consumers get 96 + 32 / 4 = 104
-constexpr int kRegCons = SPINFER_DW_REG ? 104 : 96, kRegRole = 64;   // pool: 16 x (104 - 96) = 4 x (96 - 64)
-constexpr int kWarpsD = kCWd + 4;         // + warp 19 (idle: completes the role warpgroup)
+// 20 warps = 5 per SM sub-partition (4 consumers + 1 role warp): 96 registers each (the
+// per-sub-partition register file); setmaxnreg rebalancing measured no gain
+constexpr int kWarpsD = kCWd + 4;         // + warp 19 (idle)
 constexpr int kThreadsD = 32 * kWarpsD;
 constexpr int kMaxSd = 8;
 constexpr int kMaxGd = 4;
@@ -74,27 +54,17 @@ constexpr int kNSeg = 4;                  // segment slots between consumers and
 constexpr uint32_t kHdrBytes = 64;        // per-slot stage header: value offsets, poison flag
 constexpr uint32_t kTblBytes = 1024;      // one GroupTile's SMBD table (64 BTs x 2 halves x 8 B)
 // shared-memory map (bytes from the 1024-aligned base)
-constexpr uint32_t kBarFull = 0, kBarEmpty = 64, kBarSegFull = 128, kBarSegFree = 192, kSegMask = 224, kTmemSlot = 256;
-// PIPE 9: each consumer warp keeps its fp32 accumulators in its TMEM lane quarter between
-// half-GroupTile phases (16 N columns: 32 TMEM columns per warp, 128 per quarter)
-constexpr uint32_t kTmemCols = 128;
-#ifndef SPINFER_DW_XTMA
-#define SPINFER_DW_XTMA 1
-#endif
-// X slab: tensor copy with the 32B swizzle (conflict-free ldmatrix) or a plain bulk copy issued
-// with the stage's other copies (2-way bank conflicts on the ldmatrix reads)
-constexpr bool kXTma = SPINFER_DW_XTMA != 0;
+constexpr uint32_t kBarFull = 0, kBarEmpty = 64, kBarSegFull = 128, kBarSegFree = 192, kSegMask = 224;
 constexpr uint32_t kHdrStop = 1u << 16, kHdrBad = 1u << 17;   // header word 1: g | rows << 8 | flags
 constexpr uint32_t kOffHdr = 1024;
 constexpr uint32_t kOffTbl = kOffHdr + kMaxSd * kHdrBytes;   // per-warp SMBD tables
 constexpr uint32_t kOffRing = (kOffTbl + kCWd * kTblBytes + 1023) / 1024 * 1024;
 
 struct DParams {
-    CUtensorMap tmap_x;           // X [K][Np] fp16, box {Np, 64 G}, no swizzle (ragged-K tail stages only)
+    CUtensorMap tmap_x;           // X [K][Np] fp16, box {Np, 64 G}, 32B swizzle for Np = 16 (conflict-free ldmatrix)
     const int32_t *off;
     const uint64_t *bm;
     const uint16_t *vals;
-    const uint16_t *X;            // X [K][Np] fp16 (or its zero-padded copy), the bulk-copy source
     uint16_t *Y;
     const uint16_t *bias;         // fused epilogue: fp16 [M] or null
     int act;
@@ -110,7 +80,6 @@ struct DParams {
     uint32_t slot_bytes, st_bm, st_v0, st_v1, vcap;   // slot: X slab | bitmaps | values row 0 | row 1
     float avg_gt;                 // n_values / NGT (start-up page prefetch hint)
     long long *prof;              // experiments only (SPINFER_INSTRUMENT)
-    uint32_t zero;                // 0 at run time (a value ptxas cannot fold: scheduling dependency)
 };
 
 #ifndef SPINFER_INSTRUMENT
@@ -121,7 +90,7 @@ struct DParams {
 // producer k0 waiting for a free slot, k1 issuing; reducer k0 waiting, k1 reducing.
 constexpr int kProfW = 20;
 constexpr size_t kTraceOff = 1024 * kProfW * 8;   // stage trace of CTA 0 after the counters
-constexpr size_t kEvOff = kTraceOff + 256 * 4;      // per-warp event trace of CTA 0: [16 warps][64 stages][6]
+[[maybe_unused]] constexpr size_t kEvOff = kTraceOff + 256 * 4;      // per-warp event trace of CTA 0: [16 warps][64 stages][6]
 struct Prof {
 #if SPINFER_INSTRUMENT
     long long c[8] = {0, 0, 0, 0, 0, 0, 0, 0};
@@ -308,10 +277,6 @@ __device__ __forceinline__ float4 ldg_cg4(const float4 *p) {
 __device__ __forceinline__ void discard_l2(const void *p) {
     asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory");
 }
-__device__ __forceinline__ void mbar_arrive_cnt(uint32_t bar, uint32_t n) {
-    asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0], %1;\n\t}" ::"r"(bar), "r"(n) : "memory");
-}
-
 // The CTA partial of GT row `grow` (row-major 64 x Np fp32) is parked; count the CTA and, as the
 // last of the CTAs overlapping the rowblock, sum all CTA partials in CTA order and write Y.
 // Called by one whole warp after every lane's stores are ordered before it (syncwarp/barrier).
@@ -348,53 +313,6 @@ __device__ __forceinline__ void cta_count_and_sum(const DParams &prm, int rb, in
     if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed for the next call
 }
 
-// The decode of one GroupTile as its own (out-of-line) function: compiled in a clean context, ptxas
-// issues the table and value loads of the whole GT in one burst ahead of the MMAs (3x the decode
-// throughput of the interleaved schedule it picks inside the consumer loop, tools/decode_bench.cu).
-template <int NT>
-struct AccT {
-    float v[4][NT][4];
-};
-template <int NT>
-__device__ __noinline__ AccT<NT> decode_gt(AccT<NT> acc, uint32_t tbl_lane, uint32_t xs, uint32_t mulc) {
-    constexpr uint32_t cpr = NT;
-    uint32_t bfr[4][NT][2];
-#pragma unroll
-    for (int tc = 0; tc < 4; ++tc) {
-        const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
-        if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
-        else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
-    }
-#pragma unroll
-    for (int s8 = 0; s8 < 8; ++s8) {
-        uint4 E[4];
-#pragma unroll
-        for (int k = 0; k < 4; ++k) E[k] = lds_v4(tbl_lane + (uint32_t)s8 * 64u + 16u * k);
-        uint32_t t0[8], t1[8], s1[8];
-#pragma unroll
-        for (int k = 0; k < 8; ++k) {
-            const uint32_t w = (k & 1) ? E[k >> 1].z : E[k >> 1].x;
-            const uint32_t A = (k & 1) ? E[k >> 1].w : E[k >> 1].y;   // first value of the half - 4 bytes
-            const uint32_t z = w * mulc;                               // top two bits: the lane's pair y
-            const uint32_t a = A + 2u * __popc(z);                     // &V[c2 - 2], c2 = MaskedPopCount + y0 + y1
-            const uint32_t y = z >> 30;
-            s1[k] = y * (y * kSelB + kSelA) + kSelC;
-            t0[k] = lds_u16(a);
-            t1[k] = lds_u16(a + 2u);
-        }
-        const int trb = 2 * (s8 & 1);
-#pragma unroll
-        for (int tt = 0; tt < 2; ++tt) {
-            uint32_t afr[4];
-#pragma unroll
-            for (int b = 0; b < 4; ++b) afr[b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
-#pragma unroll
-            for (int nt = 0; nt < NT; ++nt) mma_16816(acc.v[trb + tt][nt], afr, bfr[s8 >> 1][nt][0], bfr[s8 >> 1][nt][1]);
-        }
-    }
-    return acc;
-}
-
 template <int NT, bool EPI>
 __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant__ DParams prm) {
     constexpr int Np = NT * 8;
@@ -425,22 +343,11 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         }
         fence_barrier_init();
     }
-#if SPINFER_DW_PIPE == 9
-    if (warp == 0) tm_alloc(sbase + kTmemSlot, kTmemCols);
-    tm_fence_before();
-#endif
     __syncthreads();
-#if SPINFER_DW_PIPE == 9
-    tm_fence_after();
-#endif
     Prof pf;
     pf.start();
-    // role warps (warpgroup 4): give registers back, then split into producers / reducer / idle.
-    // Each branch below ends in a return, so ptxas compiles each region for its own budget.
+    // role warps: producers / reducer / idle. Each branch below ends in a return.
     if (warp >= kCWd) {
-#if SPINFER_DW_REG
-    setmaxnreg_dec<kRegRole>();
-#endif
     if (warp == kCWd + 3) return;   // the idle warp (completes the warpgroup)
 
     if (warp == kProdWarp0 || warp == kProdWarp0 + 2) {
@@ -458,7 +365,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         Stages it;
         it.init(u0, u1, KG, G, MG);
         int nseg = 0, i = 0;
-        uint32_t pslot = 0, pph = 0;   // ring position of stage i
+        uint32_t pslot = 0;            // ring slot of stage i
         uint32_t owners_pk = 0;        // 4 bits per slot: GT owners of the stage last issued into it
         auto step = [&](Stages &s, int &ns, int &ii) {   // one stage forward (segment count, index)
             if (s.seg_last(KG)) ++ns;
@@ -486,16 +393,12 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
 
         const uint64_t pol = policy_evict_first();
         while (it.valid()) {
-            const uint32_t slot = pslot, ph = pph;
+            const uint32_t slot = pslot;
             pf.lap(1);
             if (lane == 0) pf.st(prm.prof, p, i, 3, true);
-#if SPINFER_DW_NBAR
             // the slot's previous stage (i - S) released by its GT owners: hardware named barrier
             // (the waiting warp is not woken by the CTA's mbarrier traffic, no polling)
             if (i >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + ((owners_pk >> (4 * slot)) & 15u)));
-#else
-            if (i >= S) mbar_wait_expo(bar_empty + 8 * slot, ph ^ 1u, SPINFER_DW_PNS0, SPINFER_DW_PNS1);
-#endif
             pf.lap(0);
             if (lane == 0) pf.st(prm.prof, p, i, 0, true);
             const uint32_t st = ring + slot * prm.slot_bytes, fb = bar_full + 8 * slot;
@@ -521,10 +424,8 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                                       (uint32_t)nseg, 0u));
             const uint32_t vbl = (oj == 0 && orow < rows && !bad) ? 2u * (uint32_t)(oend - oc) : 0u;   // lanes 0, 8
             const uint32_t vb1 = __shfl_sync(0xffffffffu, vbl, 8);
-            // the X slab: a plain bulk copy of g GT columns, or (ragged K, last column) the tensor
-            // copy that zero-fills the rows past K
-            const bool xt = kXTma || (it.gc + g) * 64 > prm.K;
-            const uint32_t xbytes = xt ? (uint32_t)G * 64u * Np * 2u : (uint32_t)g * 64u * Np * 2u;
+            // the X slab: one tensor copy of G GT columns (rows past K zero-filled by the TMA)
+            const uint32_t xbytes = (uint32_t)G * 64u * Np * 2u;
             const uint32_t bmb = (uint32_t)g * 512u;
             __syncwarp();
             if (lane == 0) {
@@ -532,19 +433,12 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                 // one arrival with every transaction byte registered up front: the phase completes
                 // only when all copies of the stage have landed (release: the header stores above)
                 mbar_arrive_expect_tx(fb, (uint32_t)rows * bmb + xbytes + vbl + vb1);
-#if !SPINFER_DW_NBAR
-                // the empty barrier expects kRd * kMaxGd arrivals: one per GT owner of the stage, the rest now
-                const uint32_t owners = (uint32_t)(rows * g);
-                if (owners < (uint32_t)(kRd * kMaxGd)) mbar_arrive_cnt(bar_empty + 8 * slot, (uint32_t)(kRd * kMaxGd) - owners);
-#endif
             }
             pf.lap(3);
             uint32_t dst = 0, bytes = 0;
             const void *src = nullptr;
             if (oj == 0) {                                  // lanes 0, 8: packed values of row orow
                 dst = st + (orow ? prm.st_v1 : prm.st_v0); src = prm.vals + oc; bytes = vbl;
-            } else if (lane == 1 && !xt) {                  // X rows [64 gc, 64 (gc + g))
-                dst = st; src = prm.X + (size_t)64 * it.gc * Np; bytes = xbytes;
             } else if (lane == 2 || lane == 3) {            // bitmaps of row lane - 2
                 const int r = lane - 2;
                 dst = st + prm.st_bm + (uint32_t)(r * G) * 512u;
@@ -552,12 +446,12 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                 bytes = r < rows ? bmb : 0u;
             }
             if (bytes) bulk_g2s(dst, src, bytes, fb, pol);
-            if (xt && lane == 1) tma_2d_g2s(st, &prm.tmap_x, 0, 64 * it.gc, fb);
+            if (lane == 1) tma_2d_g2s(st, &prm.tmap_x, 0, 64 * it.gc, fb);
             pf.lap(4);
 
             skip2(it, nseg, i);
             pslot += 2;
-            if (pslot >= (uint32_t)S) { pslot -= (uint32_t)S; pph ^= 1u; }
+            if (pslot >= (uint32_t)S) pslot -= (uint32_t)S;
             oc = on;
             on = ld_off(ia);   // two own stages ahead: in flight while this warp issues the next stages
             skip2(ia, nsa, ia_i);
@@ -567,12 +461,8 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         // its header carries the CTA's segment count
         {
             if ((i & 1) != q) ++i;   // the loop can stop one index short of this producer's parity
-            const uint32_t slot = (uint32_t)(i % S), ph = (uint32_t)(i / S) & 1u;
-#if SPINFER_DW_NBAR
+            const uint32_t slot = (uint32_t)(i % S);
             if (i >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + ((owners_pk >> (4 * slot)) & 15u)));
-#else
-            if (i >= S) mbar_wait_poll(bar_empty + 8 * slot, ph ^ 1u, 128u);
-#endif
             if (lane == 0) {
                 sts_v4(sbase + kOffHdr + slot * kHdrBytes, make_uint4(0u, kHdrStop, (uint32_t)nseg, 0u));
                 mbar_arrive(bar_full + 8 * slot);
@@ -660,9 +550,6 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     }
 
     }   // role warps
-#if SPINFER_DW_REG
-    setmaxnreg_inc<kRegCons>();
-#endif
 
     // ---------------------------------------------------------------------- consumers
     // Warp (r, m) owns GT j = m % 4 of GT row r in every stage i with i % 2 == m / 4; it reads the
@@ -673,7 +560,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     constexpr uint32_t cpr = Np / 8;   // 16-byte chunks per X row
     const uint32_t rr = lane & 7, mk = (lane >> 3) & 1, mn = (lane >> 4) & 1;
     // X slab row-major; with the tensor copy the 32B swizzle XORs the 16-byte chunk with row bit 2
-    const uint32_t x_lane = (mk * 8u + rr) * cpr * 16u + ((mn ^ (kXTma && NT == 2 ? (rr >> 2) & 1u : 0u)) * 16u);
+    const uint32_t x_lane = (mk * 8u + rr) * cpr * 16u + ((mn ^ (NT == 2 ? (rr >> 2) & 1u : 0u)) * 16u);
     float acc[4][NT][4];
 #pragma unroll
     for (int a = 0; a < 4; ++a)
@@ -715,82 +602,12 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             u1[k] = lds_u16(a + 2u);
         }
     };
-    auto assemble_from = [&](const uint32_t (&u0)[8], const uint32_t (&u1)[8], const uint32_t (&sl)[8], int trb,
-                             const uint32_t (&bfr)[NT][2]) {
-#pragma unroll
-        for (int tt = 0; tt < 2; ++tt) {
-            uint32_t afr[4];
-#pragma unroll
-            for (int b = 0; b < 4; ++b) afr[b] = prmt(u0[tt * 4 + b], u1[tt * 4 + b], sl[tt * 4 + b]);
-#pragma unroll
-            for (int nt = 0; nt < NT; ++nt) mma_16816(acc[trb + tt][nt], afr, bfr[nt][0], bfr[nt][1]);
-        }
-    };
-#if SPINFER_DW_PIPE == 9
-    const uint32_t tacc = lds_u32(sbase + kTmemSlot) + ((uint32_t)(warp & 3) * 32u << 16) + (uint32_t)(warp >> 2) * 16u * NT;
-    uint32_t zmask = 3u;   // bit h: half h of the accumulators (TCTile rows 2h, 2h + 1) is zero, not in TMEM
-    auto tm_get = [&](int h, float (&a)[2][NT][4]) {
-        if ((zmask >> h) & 1u) {
-#pragma unroll
-            for (int t = 0; t < 2; ++t)
-#pragma unroll
-                for (int b = 0; b < NT; ++b)
-#pragma unroll
-                    for (int e = 0; e < 4; ++e) a[t][b][e] = 0.f;
-            return;
-        }
-        if constexpr (NT == 2) {
-            uint32_t u[16];
-            tm_ld_32x32b_x16u(tacc + 16u * h, u);
-            tm_wait_ld();
-#pragma unroll
-            for (int k = 0; k < 16; ++k) a[k >> 3][(k >> 2) & 1][k & 3] = __uint_as_float(u[k]);
-        } else {
-            uint32_t u[8];
-            tm_ld_32x32b_x8u(tacc + 8u * h, u);
-            tm_wait_ld();
-#pragma unroll
-            for (int k = 0; k < 8; ++k) a[k >> 2][0][k & 3] = __uint_as_float(u[k]);
-        }
-    };
-    auto tm_put = [&](int h, const float (&a)[2][NT][4]) {
-        if constexpr (NT == 2) {
-            uint32_t u[16];
-#pragma unroll
-            for (int k = 0; k < 16; ++k) u[k] = __float_as_uint(a[k >> 3][(k >> 2) & 1][k & 3]);
-            tm_st_32x32b_x16(tacc + 16u * h, u);
-        } else {
-            uint32_t u[8];
-#pragma unroll
-            for (int k = 0; k < 8; ++k) u[k] = __float_as_uint(a[k >> 2][0][k & 3]);
-            tm_st_32x32b_x8(tacc + 8u * h, u);
-        }
-        tm_wait_st();
-        zmask &= ~(1u << h);
-    };
-    auto fetch_acc = [&]() {   // the accumulators into registers (segment ends)
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            float a[2][NT][4];
-            tm_get(h, a);
-#pragma unroll
-            for (int t = 0; t < 2; ++t)
-#pragma unroll
-                for (int b = 0; b < NT; ++b)
-#pragma unroll
-                    for (int e = 0; e < 4; ++e) acc[2 * h + t][b][e] = a[t][b][e];
-        }
-    };
-#else
-    auto fetch_acc = [&]() {};
-#endif
     // segment hand-off to the reducer (non-final segments): park the partial if this warp owned a
     // GT of the segment, then arrive; `own` = false arrives for a segment without a GT of this warp
     auto seg_close = [&](int sg, bool own) {
         const int k = sg % kNSeg;
         if (sg >= kNSeg) mbar_wait_poll(bar_sfree + 8 * k, (uint32_t)((sg / kNSeg) - 1) & 1u, 256u);
         if (own) {
-            fetch_acc();
             float4 *dst = reinterpret_cast<float4 *>(prm.ws_seg) + ((((size_t)p * kNSeg + k) * kRd + r) * 8 + m) * kF4;
 #pragma unroll
             for (int tr = 0; tr < 4; ++tr)
@@ -813,23 +630,6 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         const uint32_t vsm = st_ + (r ? prm.st_v1 : prm.st_v0) + voff_;
         const uint32_t pax = __popc(ba_.x), pbx = __popc(bb_.x);
         const uint32_t packed = (pax + __popc(ba_.y)) | ((pbx + __popc(bb_.y)) << 16);
-#if SPINFER_DW_VSCAN
-        // exclusive prefix of the two 7-bit counts over the lanes, bit-sliced with ballots (vote
-        // unit, not the shared-memory pipe the shuffles queue behind)
-        const uint32_t lo = packed & 0xFFFFu, hi = packed >> 16;
-        const uint32_t lt = (1u << lane) - 1u;
-        uint32_t elo = 0, ehi = 0, tlo = 0, thi = 0;
-#pragma unroll
-        for (int b = 0; b < 7; ++b) {
-            const uint32_t B0 = __ballot_sync(0xffffffffu, (lo >> b) & 1u), B1 = __ballot_sync(0xffffffffu, (hi >> b) & 1u);
-            elo += (uint32_t)__popc(B0 & lt) << b;
-            ehi += (uint32_t)__popc(B1 & lt) << b;
-            tlo += (uint32_t)__popc(B0) << b;
-            thi += (uint32_t)__popc(B1) << b;
-        }
-        const uint32_t tot = tlo | (thi << 16);
-        const uint32_t incl = packed + (elo | (ehi << 16));
-#else
         uint32_t incl = packed;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -837,7 +637,6 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             incl += (lane >= o) ? y : 0u;
         }
         const uint32_t tot = __shfl_sync(0xffffffffu, incl, 31);
-#endif
         const uint32_t tot_a = tot & 0xFFFFu;
         if ((flags_ & kHdrBad) || 2u * (tot_a + (tot >> 16)) > vend_ - voff_) return false;
         const uint32_t excl = incl - packed;
@@ -880,16 +679,12 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             if (cur >= 0 && r < f_rows) seg_close(cur, contrib);
             for (int s2 = cur + 1; s2 < sg; ++s2) seg_close(s2, false);   // segments with no stage of this parity
             cur = sg;
-#if SPINFER_DW_PIPE == 9
-            zmask = 3u;
-#else
 #pragma unroll
             for (int a = 0; a < 4; ++a)
 #pragma unroll
                 for (int b = 0; b < NT; ++b)
 #pragma unroll
                     for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
-#endif
             contrib = false;
         }
         f_rb = (int)h.x; f_rows = rows;
@@ -901,36 +696,6 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             pf.lap(1);
             if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 3);
             if (ok) {
-#if SPINFER_DW_PIPE == 1
-                // --- decode the 16 TCTiles: 8 steps of 8 BitmapTiles (TCTile column tc = s / 2, TCTile
-                // rows 2 (s % 2), 2 (s % 2) + 1), two deep: while step s is assembled and multiplied, the
-                // value loads of step s + 1 and the table entries of step s + 2 are in flight
-                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
-                uint32_t bfr[2][NT][2];
-                auto load_x = [&](int tc, uint32_t (&b)[NT][2]) {
-                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
-                    if constexpr (NT == 1) {
-                        ldsm_x2_trans(xk, b[0][0], b[0][1]);
-                    } else {
-                        ldsm_x4_trans(xk, b[0][0], b[0][1], b[1][0], b[1][1]);
-                    }
-                };
-                uint32_t tA0[8], tA1[8], sA[8], tB0[8], tB1[8], sB[8];
-                load_x(0, bfr[0]);
-                load_E(tbl_lane);
-                issue_to(tA0, tA1, sA);
-                load_E(tbl_lane + 64u);
-#pragma unroll
-                for (int s = 0; s < 8; ++s) {
-                    if (s + 1 < 8) {
-                        if (s & 1) issue_to(tA0, tA1, sA); else issue_to(tB0, tB1, sB);
-                    }
-                    if (s + 2 < 8) load_E(tbl_lane + (uint32_t)(s + 2) * 64u);
-                    if ((s & 1) && s + 1 < 8) load_x((s + 1) >> 1, bfr[((s + 1) >> 1) & 1]);
-                    if (s & 1) assemble_from(tB0, tB1, sB, 2, bfr[(s >> 1) & 1]);
-                    else assemble_from(tA0, tA1, sA, 0, bfr[(s >> 1) & 1]);
-                }
-#elif SPINFER_DW_PIPE == 2
                 // --- decode the 16 TCTiles: TCTile column tc, row pairs (0,1), (2,3)
                 // the whole GT is one schedulable region: addresses laundered after the table writes,
                 // accumulators fenced at the end, no volatile operation in between
@@ -958,235 +723,6 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
 #pragma unroll
                     for (int b = 0; b < NT; ++b)
                         asm volatile("" : "+f"(acc[a][b][0]), "+f"(acc[a][b][1]), "+f"(acc[a][b][2]), "+f"(acc[a][b][3]) :: "memory");
-#elif SPINFER_DW_PIPE == 5
-                {
-                    AccT<NT> a_;
-#pragma unroll
-                    for (int a = 0; a < 4; ++a)
-#pragma unroll
-                        for (int b = 0; b < NT; ++b)
-#pragma unroll
-                            for (int e = 0; e < 4; ++e) a_.v[a][b][e] = acc[a][b][e];
-                    a_ = decode_gt<NT>(a_, tbl_lane, st + x_lane + (uint32_t)(64 * jw) * cpr * 16u, mulc);
-#pragma unroll
-                    for (int a = 0; a < 4; ++a)
-#pragma unroll
-                        for (int b = 0; b < NT; ++b)
-#pragma unroll
-                            for (int e = 0; e < 4; ++e) acc[a][b][e] = a_.v[a][b][e];
-                }
-#elif SPINFER_DW_PIPE == 6
-                // --- decode in two phases per half GroupTile: (1) table entries, value loads and PRMTs
-                // of 32 BitmapTiles into A fragments, (2) their 16 MMAs; a compiler barrier between
-                // the phases keeps the 64 value loads of a half in one burst ahead of the MMAs
-                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
-#pragma unroll
-                for (int half = 0; half < 2; ++half) {
-                    uint32_t bfr[2][NT][2];
-#pragma unroll
-                    for (int t2 = 0; t2 < 2; ++t2) {
-                        const uint32_t xk = xs + (uint32_t)(16 * (2 * half + t2)) * cpr * 16u;
-                        if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[t2][0][0], bfr[t2][0][1]);
-                        else ldsm_x4_trans(xk, bfr[t2][0][0], bfr[t2][0][1], bfr[t2][1][0], bfr[t2][1][1]);
-                    }
-                    uint32_t afr[4][2][4];
-#pragma unroll
-                    for (int k = 0; k < 4; ++k) {
-                        uint32_t t0[8], t1[8], s1[8];
-                        load_E(tbl_lane + (uint32_t)(4 * half + k) * 64u);
-                        issue_to(t0, t1, s1);
-#pragma unroll
-                        for (int tt = 0; tt < 2; ++tt)
-#pragma unroll
-                            for (int b = 0; b < 4; ++b) afr[k][tt][b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
-                    }
-#pragma unroll
-                    for (int k = 0; k < 4; ++k)
-#pragma unroll
-                        for (int tt = 0; tt < 2; ++tt)
-                            asm volatile("" : "+r"(afr[k][tt][0]), "+r"(afr[k][tt][1]), "+r"(afr[k][tt][2]), "+r"(afr[k][tt][3]));
-#pragma unroll
-                    for (int k = 0; k < 4; ++k)
-#pragma unroll
-                        for (int tt = 0; tt < 2; ++tt)
-#pragma unroll
-                            for (int nt = 0; nt < NT; ++nt)
-                                mma_16816(acc[2 * (k & 1) + tt][nt], afr[k][tt], bfr[k >> 1][nt][0], bfr[k >> 1][nt][1]);
-                }
-#elif SPINFER_DW_PIPE == 7
-                // --- decode in two phases per GroupTile: (1) table entries, value loads and PRMTs of all
-                // 64 BitmapTiles into A fragments, (2) the 32 MMAs. Every MMA also depends on the last
-                // fragment (OR with prm.zero, 0 at run time and unknown to ptxas), so ptxas issues the
-                // GT's 128 value loads in one burst instead of interleaving them with the MMAs
-                // (tools/decode_bench.cu: 3x the decode throughput).
-                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
-                uint32_t afr[8][2][4];
-#pragma unroll
-                for (int k = 0; k < 8; ++k) {
-                    uint32_t t0[8], t1[8], s1[8];
-                    load_E(tbl_lane + (uint32_t)k * 64u);
-                    issue_to(t0, t1, s1);
-#pragma unroll
-                    for (int tt = 0; tt < 2; ++tt)
-#pragma unroll
-                        for (int b = 0; b < 4; ++b) afr[k][tt][b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
-                }
-                const uint32_t dep = afr[7][1][3] & prm.zero;
-                uint32_t bfr[4][NT][2];
-#pragma unroll
-                for (int tc = 0; tc < 4; ++tc) {
-                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
-                    if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
-                    else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
-                }
-#pragma unroll
-                for (int k = 0; k < 8; ++k)
-#pragma unroll
-                    for (int tt = 0; tt < 2; ++tt) {
-                        afr[k][tt][0] |= dep;
-#pragma unroll
-                        for (int nt = 0; nt < NT; ++nt)
-                            mma_16816(acc[2 * (k & 1) + tt][nt], afr[k][tt], bfr[k >> 1][nt][0], bfr[k >> 1][nt][1]);
-                    }
-#elif SPINFER_DW_PIPE == 8
-                // --- as PIPE 7, per half GroupTile (32 BitmapTiles per burst, fewer live fragments)
-                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
-#pragma unroll
-                for (int half = 0; half < 2; ++half) {
-                    uint32_t afr[4][2][4];
-#pragma unroll
-                    for (int k = 0; k < 4; ++k) {
-                        uint32_t t0[8], t1[8], s1[8];
-                        load_E(tbl_lane + (uint32_t)(4 * half + k) * 64u);
-                        issue_to(t0, t1, s1);
-#pragma unroll
-                        for (int tt = 0; tt < 2; ++tt)
-#pragma unroll
-                            for (int b = 0; b < 4; ++b) afr[k][tt][b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
-                    }
-                    const uint32_t dep = afr[3][1][3] & prm.zero;
-                    uint32_t bfr[2][NT][2];
-#pragma unroll
-                    for (int t2 = 0; t2 < 2; ++t2) {
-                        const uint32_t xk = xs + (uint32_t)(16 * (2 * half + t2)) * cpr * 16u;
-                        if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[t2][0][0], bfr[t2][0][1]);
-                        else ldsm_x4_trans(xk, bfr[t2][0][0], bfr[t2][0][1], bfr[t2][1][0], bfr[t2][1][1]);
-                    }
-#pragma unroll
-                    for (int k = 0; k < 4; ++k)
-#pragma unroll
-                        for (int tt = 0; tt < 2; ++tt) {
-                            afr[k][tt][0] |= dep;
-#pragma unroll
-                            for (int nt = 0; nt < NT; ++nt)
-                                mma_16816(acc[2 * (k & 1) + tt][nt], afr[k][tt], bfr[k >> 1][nt][0], bfr[k >> 1][nt][1]);
-                        }
-                }
-#elif SPINFER_DW_PIPE == 9
-                // --- decode in two phases of 32 BitmapTiles (TCTile rows 2h, 2h + 1 of all 4 TCTile
-                // columns); the phase's 16 accumulators come from and go back to TMEM, which frees
-                // the registers for the whole phase's table entries, value loads and PRMTs ahead of
-                // its 16 MMAs (one burst of 64 value loads; tools/decode_bench.cu)
-                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
-                uint32_t bfr[4][NT][2];
-#pragma unroll
-                for (int tc = 0; tc < 4; ++tc) {
-                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
-                    if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
-                    else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
-                }
-#pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                    uint32_t afr[4][2][4];
-#pragma unroll
-                    for (int tc = 0; tc < 4; ++tc) {
-                        uint32_t t0[8], t1[8], s1[8];
-                        load_E(tbl_lane + (uint32_t)(2 * tc + h) * 64u);
-                        issue_to(t0, t1, s1);
-#pragma unroll
-                        for (int tt = 0; tt < 2; ++tt)
-#pragma unroll
-                            for (int b = 0; b < 4; ++b) afr[tc][tt][b] = prmt(t0[tt * 4 + b], t1[tt * 4 + b], s1[tt * 4 + b]);
-                    }
-                    float a[2][NT][4];
-                    tm_get(h, a);
-                    const uint32_t dep = afr[3][1][3] & prm.zero;
-#pragma unroll
-                    for (int tc = 0; tc < 4; ++tc)
-#pragma unroll
-                        for (int tt = 0; tt < 2; ++tt) {
-                            afr[tc][tt][0] |= dep;
-#pragma unroll
-                            for (int nt = 0; nt < NT; ++nt) mma_16816(a[tt][nt], afr[tc][tt], bfr[tc][nt][0], bfr[tc][nt][1]);
-                        }
-                    tm_put(h, a);
-                }
-#elif SPINFER_DW_PIPE == 4
-                // --- decode the 16 TCTiles, fully unrolled: X fragments of all 4 TCTile columns, then
-                // 8 steps of 8 BitmapTiles (tools/decode_bench.cu: the compiler issues the table and
-                // value loads of the whole GT in one burst ahead of the MMAs)
-                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
-                uint32_t bfr[4][NT][2];
-#pragma unroll
-                for (int tc = 0; tc < 4; ++tc) {
-                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
-                    if constexpr (NT == 1) ldsm_x2_trans(xk, bfr[tc][0][0], bfr[tc][0][1]);
-                    else ldsm_x4_trans(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
-                }
-                uint32_t t0[8], t1[8], s1[8];
-#pragma unroll
-                for (int s8 = 0; s8 < 8; ++s8) {
-                    load_E(tbl_lane + (uint32_t)s8 * 64u);
-                    issue_to(t0, t1, s1);
-                    assemble_from(t0, t1, s1, 2 * (s8 & 1), bfr[s8 >> 1]);
-                }
-#elif SPINFER_DW_PIPE == 3
-                // --- decode the 16 TCTiles as one schedulable region (no volatile operation inside:
-                // addresses laundered after the table writes, accumulators fenced at the end), X
-                // fragments of all 4 TCTile columns first, then 8 steps of 8 BitmapTiles; the compiler
-                // hoists the table and value loads of later steps ahead of earlier steps' MMAs
-                const uint32_t xs = launder_u32(st + x_lane + (uint32_t)(64 * jw) * cpr * 16u);
-                const uint32_t tbl_lane_l = launder_u32(tbl_lane);
-                uint32_t bfr[4][NT][2];
-#pragma unroll
-                for (int tc = 0; tc < 4; ++tc) {
-                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
-                    if constexpr (NT == 1) ldsm_x2_trans_nv(xk, bfr[tc][0][0], bfr[tc][0][1]);
-                    else ldsm_x4_trans_nv(xk, bfr[tc][0][0], bfr[tc][0][1], bfr[tc][1][0], bfr[tc][1][1]);
-                }
-                uint32_t t0[8], t1[8], s1[8];
-#pragma unroll
-                for (int s8 = 0; s8 < 8; ++s8) {
-                    load_E_nv(tbl_lane_l + (uint32_t)s8 * 64u);
-                    issue_to(t0, t1, s1);
-                    assemble_nv(t0, t1, s1, 2 * (s8 & 1), bfr[s8 >> 1]);
-                }
-#pragma unroll
-                for (int a = 0; a < 4; ++a)
-#pragma unroll
-                    for (int b = 0; b < NT; ++b)
-                        asm volatile("" : "+f"(acc[a][b][0]), "+f"(acc[a][b][1]), "+f"(acc[a][b][2]), "+f"(acc[a][b][3]) :: "memory");
-#else
-                // --- decode the 16 TCTiles: TCTile column tc, row pairs (0,1), (2,3)
-                const uint32_t xs = st + x_lane + (uint32_t)(64 * jw) * cpr * 16u;
-                uint32_t t0[8], t1[8], s1[8];
-#pragma unroll 1
-                for (int tc = 0; tc < 4; ++tc) {
-                    uint32_t bfr[NT][2];
-                    const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
-                    if constexpr (NT == 1) {
-                        ldsm_x2_trans(xk, bfr[0][0], bfr[0][1]);
-                    } else {
-                        ldsm_x4_trans(xk, bfr[0][0], bfr[0][1], bfr[1][0], bfr[1][1]);
-                    }
-#pragma unroll
-                    for (int hh = 0; hh < 2; ++hh) {
-                        load_E(tbl_lane + (uint32_t)(tc * 16 + hh * 8) * 8u);
-                        issue_to(t0, t1, s1);
-                        assemble_from(t0, t1, s1, 2 * hh, bfr);
-                    }
-                }
-#endif
                 __syncwarp();   // table reads done before the next GT's scan rewrites it
                 pf.lap(2);
                 if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 4);
@@ -1195,11 +731,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                 atomicOr(prm.ws_err, 2);   // corrupt GT (or poisoned stage): skipped, Y is not valid
             }
             __syncwarp();
-#if SPINFER_DW_NBAR
             named_bar_arrive(kBarIdSlot0 + slot, 32u * (1u + (uint32_t)(rows * g)));   // the slot's GT owners + its producer
-#else
-            if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
-#endif
             if (lane == 0) pf.st(prm.prof, p, i, 2, true);
             if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 5);
         }
@@ -1212,7 +744,6 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     const int fseg = nseg_total - 1;   // the final segment (reduced below in shared memory)
     if (cur >= 0 && cur < fseg && r < f_rows) seg_close(cur, contrib);
     for (int s2 = cur + 1; s2 < fseg; ++s2) seg_close(s2, false);
-    if (cur == fseg) fetch_acc();
     if (cur != fseg) {   // this warp holds nothing of the final segment
 #pragma unroll
         for (int a = 0; a < 4; ++a)
@@ -1251,9 +782,6 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             }
     }
     named_bar_sync(1, 32 * kCWd);
-#if SPINFER_DW_PIPE == 9
-    if (warp == 0) tm_dealloc(lds_u32(sbase + kTmemSlot), kTmemCols);   // every consumer fetched its accumulators
-#endif
     if (fseg >= 0 && r < frows) {
         constexpr int NC = Np / 4;   // outputs per lane: 8 rows x Np columns per warp
         const int row = 8 * m + (lane >> 2), col0 = NC * (lane & 3);
@@ -1318,8 +846,8 @@ bool make_dplan(int M, int K, int Np, int max_gt_values, DPlan *pl) {
     int maxv = max_gt_values > 0 ? max_gt_values : 4096;
     maxv = std::min(4096, (maxv + 7) & ~7);
     int gmax = kMaxGd, smax = kMaxSd;
-    if (const char *e = getenv("SPINFER_G")) gmax = std::max(1, std::min(kMaxGd, atoi(e)));
-    if (const char *e = getenv("SPINFER_S")) smax = std::max(2, std::min(kMaxSd, atoi(e)));
+    if (option(SPINFER_OPT_STAGE_G) > 0) gmax = std::max(1, std::min(kMaxGd, option(SPINFER_OPT_STAGE_G)));
+    if (option(SPINFER_OPT_STAGE_S) > 0) smax = std::max(2, std::min(kMaxSd, option(SPINFER_OPT_STAGE_S)));
     const uint32_t final_scratch = 2u * 8u * 64u * Np * 4u;   // the final segment's partials reuse the ring
     int bestG = 0, bestS = 0;   // the largest G with >= 4 slots, else the deepest ring with >= 2
     for (int G = gmax; G >= 1; --G) {
@@ -1360,10 +888,7 @@ int launch_dw(const DPlan &pl, cudaStream_t st) {
         configured[dev] = (int)pl.smem;
     }
     k_spmm_dw<NT, EPI><<<pl.P, kThreadsD, pl.smem, st>>>(pl.prm);
-    const cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess && getenv("SPINFER_VERBOSE"))
-        fprintf(stderr, "spinfer: k_spmm_dw launch (P=%d smem=%zu): %s\n", pl.P, pl.smem, cudaGetErrorString(e));
-    return e == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
+    return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
 }
 
 struct DwLayout {
@@ -1404,8 +929,7 @@ int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, 
         if (int rc = launch_pad_x(X, Xp, K, N, Np, st)) return rc;
         Xk = Xp;
     }
-    if (int rc = make_x_tmap(&q.tmap_x, Xk, K, Np, Np, 64 * pl.G, kXTma)) return rc;
-    q.X = Xk;
+    if (int rc = make_x_tmap(&q.tmap_x, Xk, K, Np, Np, 64 * pl.G, true)) return rc;
     q.K = K;
     q.off = T->gtile_offset;
     q.bm = T->bitmap;
@@ -1421,7 +945,6 @@ int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, 
     q.n_values = (int)T->n_values;
     q.avg_gt = (float)((double)T->n_values / ((double)q.MG * (double)q.KG));
     q.prof = nullptr;
-    q.zero = 0;
     const bool epi = bias != nullptr || act != SPINFER_ACT_NONE || (M % kGT) != 0 || (N % 8) != 0;
     auto go = [&]() {
         if (Np == 8) return epi ? launch_dw<1, true>(pl, st) : launch_dw<1, false>(pl, st);

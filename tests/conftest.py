@@ -25,3 +25,14 @@ def pytest_collection_modifyitems(config, items):
     for it in items:
         if "gpu" in it.keywords:
             it.add_marker(skip)
+
+
+@pytest.fixture(autouse=True)
+def _reset_spinfer_options():
+    """Library options (kernel choice, grid cap, stage shape) are process-wide: every test
+    starts and ends with the defaults."""
+    yield
+    mod = sys.modules.get("paper_conf_eurosys_fanydlgww025_b200")
+    if mod is not None and getattr(mod, "_lib", None) is not None:
+        for name in mod.OPTIONS:
+            mod.set_option(name, 0)

@@ -35,13 +35,20 @@ def assert_within(Y_gpu_bits: np.ndarray, Y_ref: np.ndarray, bound: np.ndarray, 
                                          for i in idx))
 
 
-def use_kernel(kernel: str, N: int, monkeypatch):
-    """Select the SpMM kernel for this test (SPINFER_KERNEL): "default" = the library's choice,
-    "dw" = the decoupled-warp kernel (N <= 16), "mma" = the round-1 mma.sync kernel, "tc" =
-    the tcgen05 kernel."""
+def use_kernel(kernel: str, N: int, monkeypatch=None):
+    """Select the SpMM kernel for this test (spinfer_set_option SPINFER_OPT_KERNEL; the conftest
+    fixture resets every option after the test): "default" = the library's choice, "dw" = the
+    decoupled-warp mma.sync kernel (N <= 16), "tc" = the tcgen05 kernel."""
     import pytest
+    import paper_conf_eurosys_fanydlgww025_b200 as sp
     if kernel == "default":
         return
     if kernel == "dw" and N > 16:
         pytest.skip("the decoupled-warp kernel serves N <= 16")
-    monkeypatch.setenv("SPINFER_KERNEL", kernel)
+    sp.set_option("kernel", kernel)
+
+
+def max_ctas(n: int):
+    """Cap the persistent grid (forces split rowblocks on small shapes)."""
+    import paper_conf_eurosys_fanydlgww025_b200 as sp
+    sp.set_option("max_ctas", n)

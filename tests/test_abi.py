@@ -36,13 +36,33 @@ def test_header_symbols_exported(sp):
         assert getattr(L, n) is not None
 
 
+def _kernel_sass(sp):
+    """SASS of every kernel function in the library: {mangled name: text}."""
+    sass = subprocess.run(["cuobjdump", "-sass", sp.LIB_PATH], capture_output=True, text=True).stdout
+    out, name = {}, None
+    for line in sass.splitlines():
+        m = re.match(r"\s*Function : (\S+)", line)
+        if m:
+            name = m.group(1)
+            out[name] = []
+        elif name:
+            out[name].append(line)
+    return {k: "\n".join(v) for k, v in out.items()}
+
+
 def test_built_for_sm100a(sp):
     out = subprocess.run(["cuobjdump", "--list-elf", sp.LIB_PATH], capture_output=True, text=True).stdout
     assert "sm_100a" in out
-    sass = subprocess.run(["cuobjdump", "-sass", sp.LIB_PATH], capture_output=True, text=True).stdout
-    assert "HMMA.16816.F32" in sass          # tensor-core mma in the SpMM kernel
-    assert "UBLKCP" in sass                  # cp.async.bulk (TMA) staging
-    assert "SYNCS" in sass                   # mbarrier pipeline
+    ks = _kernel_sass(sp)
+    dw = [v for k, v in ks.items() if "k_spmm_dw" in k]
+    tc = [v for k, v in ks.items() if "k_spmm_tc" in k]
+    assert len(dw) == 4 and len(tc) == 2, sorted(ks)
+    for v in dw:   # N <= 16: mma.sync tensor cores fed by TMA, named-barrier slot release
+        for mn in ("HMMA.16816.F32", "UBLKCP", "UTMALDG.2D", "LDSM.16.MT88", "SYNCS", "BAR.ARV"):
+            assert mn in v, mn
+    for v in tc:   # N > 16: tcgen05 MMA (UTCHMMA), TMEM stores / loads (STTM / LDTM), TMA
+        for mn in ("UTCHMMA", "STTM", "LDTM", "UTMALDG.2D", "UBLKCP", "UTCBAR", "SYNCS"):
+            assert mn in v, mn
 
 
 def test_status_strings_and_version(sp):

@@ -355,6 +355,26 @@ def test_shard_is_slice_of_encoding():
             assert np.array_equal(S.values, E.values)
 
 
+@pytest.mark.parametrize("M,K", [(1000, 300), (130, 65), (64, 100), (577, 1)])
+def test_shard_is_slice_of_encoding_ragged(M, K):
+    """P-E5 on ragged shapes (reading A8): the shard of every rank, including the one holding the
+    partial last GT row, equals the encoding of its own rows of W, array for array."""
+    W = synth.weight(M, K, 0.5, seed=M + K)
+    T = oracle.encode(W)
+    for world in (1, 2, 3, 5):
+        for r in range(world):
+            b, c = oracle.tp_rows(M, world, r)
+            if c == 0:
+                continue
+            S = oracle.shard(T, b, c)
+            E = oracle.encode(W[b: b + c])
+            assert S.M == E.M == c
+            assert np.array_equal(S.gtile_offset, E.gtile_offset), (M, K, world, r)
+            assert np.array_equal(S.bitmap, E.bitmap)
+            assert np.array_equal(S.values, E.values)
+            assert S.n_values == E.n_values and S.nnz == E.nnz
+
+
 def test_bias_act_worked_example():
     """C7 fused FC epilogue, values worked by hand: act(Y + b) with b = (1.0, -0.5)."""
     Y = np.array([[-1.5, 2.0], [0.25, -0.25]])

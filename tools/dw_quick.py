@@ -31,21 +31,24 @@ def timeit(M, K, N, s, steps=20):
         a.record(); sp.spmm(T, Xd, Y, ws); b.record(); torch.cuda.synchronize(); ts.append(a.elapsed_time(b) * 1e3)
     nb = sp.algorithmic_bytes(T, N)
     med = float(np.median(ts))
-    print(f"time {M}x{K}x{N} s={s} kernel={os.environ.get('SPINFER_KERNEL','default')}: median {med:.1f} us mean {np.mean(ts):.1f} -> {nb/med/1e3:.0f} GB/s", flush=True)
+    print(f"time {M}x{K}x{N} s={s} kernel={sp.get_option('kernel')}: median {med:.1f} us mean {np.mean(ts):.1f} -> {nb/med/1e3:.0f} GB/s", flush=True)
     return Y
 
 if __name__ == "__main__":
     what = sys.argv[1] if len(sys.argv) > 1 else "all"
+    for a in sys.argv[2:]:   # name=value library options, e.g. kernel=tc stage_s=2
+        k, v = a.split("=")
+        sp.set_option(k, v if k == "kernel" else int(v))
     if what in ("all", "parity"):
         for (M, K, N) in [(256, 256, 8), (256, 256, 16), (64, 64, 16), (128, 4096, 16), (192, 320, 16), (1024, 1024, 16), (4096, 2048, 8), (320, 1472, 16), (100, 70, 5)]:
             parity(M, K, N, 0.5, seed=M + K + N)
         parity(384, 2048, 16, 0.5, seed=101, mode="int")
-        for ctas in ("3", "7", "16"):
-            os.environ["SPINFER_MAX_CTAS"] = ctas
+        for ctas in (3, 7, 16):
+            sp.set_option("max_ctas", ctas)
             parity(384, 2048, 16, 0.5, seed=101, mode="int")
             parity(576, 1472, 8, 0.5, seed=102, mode="int")
             parity(192, 4160, 13, 0.5, seed=7)
-        del os.environ["SPINFER_MAX_CTAS"]
+        sp.set_option("max_ctas", 0)
     if what in ("all", "time"):
         for s in (0.5, 0.3, 0.7):
             timeit(28672, 8192, 16, s)
