@@ -1,27 +1,36 @@
 #!/usr/bin/env python3
 """bench.py — TCA-BME SpMM (SpInfer hot path) on B200: one JSON line on rank 0.
 
-Workload (BASELINE.json configs[1]): Y = W X with W fp16 M x K = 28672 x 8192 at
-50% unstructured sparsity stored in TCA-BME, X fp16 K x N = 8192 x 16, fp32
-accumulation. A "step" is one spinfer_spmm call (the whole hot path: bulk-async
-staging, SMBD decode, tensor-core MMA, split-K fix-up) over that input.
+Workload (BASELINE.json configs[1]): Y = W X with W fp16 M x K = 28672 x 8192 at 50%
+unstructured sparsity stored in TCA-BME, X fp16 K x N = 8192 x 16, fp32 accumulation. A
+"step" is one SpMM over that input (the whole hot path in one kernel launch: bulk-async
+staging, SMBD decode, tensor-core MMA, split-K fix-up), inputs resident in HBM.
 
-Metric: algorithmic HBM GB/s = (TCA-BME bytes + X bytes + Y bytes) / kernel time
-(SURVEY §8(d)(iii)); also µs per SpMM and the cuBLAS fp16 dense GEMM on the same
-shape. L2 is flushed (256 MiB memset + 256 MiB read) before every timed step, outside the
-events. Multi-GPU (torchrun): weak scaling — every rank owns its own 28672-row
-shard of an (N_gpus*28672) x 8192 row-partitioned weight (seeded seed+rank), no
-data-path collective (SURVEY §8(e), config 4 pattern); value = sum of all ranks'
-bytes / max over ranks of the time.
+Metric: algorithmic HBM GB/s = (TCA-BME bytes + X bytes + Y bytes) / device time (SURVEY
+§8(d)(iii)); also µs per SpMM and the cuBLAS fp16 dense GEMM on the same shape. L2 is flushed
+(256 MiB memset + 256 MiB read) before every timed step, outside the events.
 
---impl reference: the CPU oracle (oracle/, single-threaded fp64 C) timed on the
-host on a bounded row sample of the same workload; rank 0 only.
+--gpus N (N > 1): row-partitioned STRONG scaling of the same config 2 (north_star
+"row-partitioned at 2/4/8 GPUs"): rank r owns rows spinfer_tp_rows(28672, N, r) of W, encodes
+only those rows and writes them into Y (spinfer_spmm_tp; no collective on the data path);
+value = config 2's algorithmic bytes / max over ranks of the step time. Without WORLD_SIZE in
+the environment, bench.py relaunches itself under torch.distributed.run with N ranks.
+
+Extra keys (--no-extras skips them): the sparsity sweep s = 0.3..0.7 on the config-2 shape,
+OPT-66B per-rank shard shapes (config 4: at N = 1 the G = 1/2/4/8 shards of rank 0 on this GPU,
+at N > 1 every rank's own shard, max over ranks), the OPT-30B four-layer stack (config 5) at
+TP = N with the NCCL all-gather of every layer's output, replayed from a CUDA graph, and the
+host cost per SpMM call.
+
+--impl reference: the CPU oracle (oracle/, single-threaded fp64 C) timed on the host on a
+bounded row sample of the same workload; rank 0 only.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -35,6 +44,7 @@ import numpy as np  # noqa: E402
 
 METRIC = "SpMM µs & HBM GB/s vs cuBLAS fp16, M/K/N=28K/8K/16, 30-70% sparsity"
 UNIT = "GB/s"
+GT = 64
 
 
 def parse():
@@ -51,7 +61,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cublas", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-extras", action="store_true", help="skip the sweep / shard / stack / host-cost keys")
     ap.add_argument("--profile", action="store_true", help="minimal run for ncu (no flush, no baselines)")
+    ap.add_argument("--opt", action="append", default=[], help="library option name=value (experiments)")
     ap.add_argument("--json-out", default=None)
     return ap.parse_args()
 
@@ -64,13 +76,15 @@ def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
         d = json.load(open(p))
-        return float(d.get("hbm_gbs", 6650.0)), "measured"
-    return 6650.0, "fallback"
+        return float(d.get("hbm_gbs", 6650.0)), "measured (MEASURED_PEAKS.json hbm_gbs, copy bandwidth)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
 
 
 def algorithmic_bytes(M, K, N, n_values):
-    """TCA-BME storage (eq. (9), with padded value count) + X + Y (fp16)."""
-    return 4 * ((M // 64) * (K // 64) + 1) + 8 * (M * K // 64) + 2 * n_values + 2 * K * N + 2 * M * N
+    """TCA-BME storage (eq. (9) P:210 with the padded value count, zero-padded to whole
+    GroupTiles) + X + Y (fp16)."""
+    ngt = (-(-M // GT)) * (-(-K // GT))
+    return 4 * (ngt + 1) + 8 * 64 * ngt + 2 * n_values + 2 * K * N + 2 * M * N
 
 
 def cpu_info():
@@ -85,10 +99,27 @@ def cpu_info():
     return model, os.cpu_count()
 
 
+def free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def relaunch(a):
+    """--gpus N without a torchrun environment: run N ranks of this script (one per GPU)."""
+    import torch
+    n = torch.cuda.device_count()
+    if n < a.gpus:
+        print(f"bench.py: --gpus {a.gpus} but only {n} CUDA device(s) visible", file=sys.stderr)
+        return 2
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
 # ----------------------------------------------------------------------------- clocks
 class ClockSampler:
-    """Samples SM clock and throttle reasons via NVML every ~1 ms during the timed region
-    (falls back to nvidia-smi polling if NVML is unavailable)."""
+    """Samples SM clock and throttle reasons via NVML every ~0.5 ms during the timed region."""
 
     REASONS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
                "sw_power_cap": 0x4, "hw_power_brake_slowdown": 0x80}
@@ -152,14 +183,14 @@ class ClockSampler:
 
 # ----------------------------------------------------------------------------- reference arm
 def run_reference(a, rank):
-    """The CPU oracle as it stands, on a bounded sample: each step = oracle SpMM of
-    the first `rows` rows of the workload's W (fp64, single-threaded)."""
+    """The CPU oracle as it stands, on a bounded sample: each step = oracle SpMM of the first
+    `rows` rows of the workload's W (fp64, single-threaded)."""
     if rank != 0:
         return None
     import oracle
     import synth
     rows = 1024
-    W = synth.weight(rows, a.K, a.sparsity, seed=a.seed)   # rows 0..1023 of the full W (same generator indices)
+    W = synth.weight(rows, a.K, a.sparsity, seed=a.seed)   # rows 0..1023 of the full W
     X = synth.activation(a.K, a.N, seed=a.seed + 1)
     T = oracle.encode(W)
     b = algorithmic_bytes(rows, a.K, a.N, T.n_values)
@@ -176,8 +207,8 @@ def run_reference(a, rank):
     sample = f"first {rows} of {a.M} rows of W (all {a.K} cols), N={a.N}, oracle.spmm_f64 (TCA-BME walk, fp64)"
     return {
         "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": a.gpus, "steps": a.steps,
-        "warmup": a.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True, "scaling": "weak",
-        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "warmup": a.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+        "scaling": "strong" if a.gpus > 1 else "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": workload_name(a), "sample_rows": rows, "seed": a.seed},
         "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
                          "cpu_model": model, "host_cpus": ncpu},
@@ -186,67 +217,249 @@ def run_reference(a, rank):
 
 
 # ----------------------------------------------------------------------------- our arm
-def run_ours(a, rank, world, local_rank):
-    import torch
-    import torch.distributed as dist
-    import synth
-    import paper_conf_eurosys_fanydlgww025_b200 as sp
+class Bench:
+    """Device, L2 flush, timing and max-over-ranks helpers for one rank."""
 
-    dev = torch.device("cuda", local_rank)
-    torch.cuda.set_device(dev)
-    M, K, N = a.M, a.K, a.N
-    seed = a.seed + rank
-    W = synth.weight(M, K, a.sparsity, seed=seed)
-    X = synth.activation(K, N, seed=a.seed + 1)
-    Wd = torch.from_numpy(W.view(np.int16)).to(dev)
-    Xd = torch.from_numpy(X.view(np.int16)).to(dev).view(torch.float16)
-    T = sp.encode(Wd)
-    ws = sp.workspace(M, K, N, dev)
-    Yd = torch.empty((M, N), dtype=torch.float16, device=dev)
-    stream = torch.cuda.current_stream()
-    nbytes = algorithmic_bytes(M, K, N, T.n_values)
-    flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)
-    flush_rd = torch.zeros(64 * 1024 * 1024, dtype=torch.float32, device=dev)   # 256 MiB
+    def __init__(self, world, rank, local_rank):
+        import torch
+        self.torch = torch
+        self.world, self.rank = world, rank
+        self.dev = torch.device("cuda", local_rank)
+        torch.cuda.set_device(self.dev)
+        self.flush_w = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=self.dev)
+        self.flush_r = torch.zeros(64 * 1024 * 1024, dtype=torch.float32, device=self.dev)   # 256 MiB
 
-    def flush_l2():
+    def flush_l2(self):
         # write a buffer larger than L2 (126 MB), then read another one: the timed kernel starts
         # with a cold L2 that holds no dirty lines (otherwise it pays the flush's write-backs)
-        flush.zero_()
-        flush_rd.sum()
+        self.flush_w.zero_()
+        self.flush_r.sum()
 
-    def barrier():
-        if world > 1:
+    def barrier(self):
+        if self.world > 1:
+            import torch.distributed as dist
             dist.barrier()
 
-    def timed(fn, steps, do_flush=True):
+    def timed(self, fn, steps, flush=True):
+        """Device time (ms) of each of `steps` calls of fn, CUDA events on the current stream."""
+        torch = self.torch
+        stream = torch.cuda.current_stream()
         evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
-        barrier()
+        self.barrier()
         torch.cuda.synchronize()
         # ~1 ms of device-side spin ahead of the loop, outside every event pair: the host gets
-        # ahead of the device, so no step's events also time a host-side launch gap (without it
-        # the first timed step read 257-384 us against 84-86 us for the others, profiles/r1_steps)
+        # ahead of the device, so no step's events also time a host-side launch gap
         torch.cuda._sleep(2_000_000)
-        for _ in range(2):   # untimed lead-in steps in the same burst (the first step after a host
-            if do_flush:     # synchronize also ran slow: profiles/r1_steps.txt)
-                flush_l2()
+        for _ in range(2):   # untimed lead-in steps in the same burst
+            if flush:
+                self.flush_l2()
             fn()
         for i in range(steps):
-            if do_flush:
-                flush_l2()
+            if flush:
+                self.flush_l2()
             evs[i][0].record(stream)
             fn()
             evs[i][1].record(stream)
         torch.cuda.synchronize()
-        barrier()
+        self.barrier()
         return [s.elapsed_time(e) for s, e in evs]
 
+    def allmax(self, x: float) -> float:
+        return self.allreduce(x, "max")
+
+    def allreduce(self, x: float, op="sum") -> float:
+        if self.world == 1:
+            return float(x)
+        import torch.distributed as dist
+        t = self.torch.tensor([float(x)], dtype=self.torch.float64, device=self.dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX if op == "max" else dist.ReduceOp.SUM)
+        return float(t.item())
+
+
+def _dev_u16(torch, a, dev):
+    return torch.from_numpy(np.ascontiguousarray(a).view(np.int16)).to(dev)
+
+
+def spmm_point(B, sp, synth, M, K, N, s, seed, steps, row0=0, rows=None, world=1, rank=0, cublas=False):
+    """Time one SpMM shape (this rank's rows [row0, row0 + rows) of an M x K weight): median µs,
+    algorithmic GB/s and roofline fraction; optionally the cuBLAS fp16 GEMM of the same rows."""
+    torch = B.torch
+    rows = M if rows is None else rows
+    W = synth.weight(rows, K, s, seed=seed, row0=row0)
+    X = _dev_u16(torch, synth.activation(K, N, seed=seed + 1), B.dev).view(torch.float16)
+    T = sp.encode(_dev_u16(torch, W, B.dev))
+    del W
+    Y = torch.empty((M if world > 1 else rows, N), dtype=torch.float16, device=B.dev)
+    ws = sp.workspace(rows, K, N, B.dev)
+    fn = (lambda: sp.spmm_tp(T, X, Y, M, world, rank, ws=ws)) if world > 1 else (lambda: sp.spmm(T, X, Y, ws=ws))
+    for _ in range(3):
+        fn()
+    t = B.timed(fn, steps)
+    med = statistics.median(t)
+    nb = algorithmic_bytes(rows, K, N, T.n_values)
+    peak, _ = load_peaks()
+    out = {"M": M, "K": K, "N": N, "s": s, "rows": rows, "us": med * 1e3, "gbs": nb / (med * 1e-3) / 1e9,
+           "frac": nb / (med * 1e-3) / 1e9 / peak}
+    if cublas:
+        Wd = sp.decode(T)
+        Yc = torch.empty((rows, N), dtype=torch.float16, device=B.dev)
+        for _ in range(3):
+            torch.mm(Wd, X, out=Yc)
+        tc = statistics.median(B.timed(lambda: torch.mm(Wd, X, out=Yc), steps))
+        out["cublas_us"] = tc * 1e3
+        out["speedup_vs_cublas"] = tc / med
+        del Wd
+    del T
+    return out
+
+
+def extras(a, B, sp, synth, tp):
+    """The non-headline measurements: sparsity sweep, config-4 shards, config-5 stack, host cost."""
+    torch = B.torch
+    world, rank = B.world, B.rank
+    res = {}
+    steps = max(5, min(a.steps, 20))
+    if world == 1:
+        sweep = []
+        for s in (0.3, 0.4, 0.5, 0.6, 0.7):
+            sweep.append(spmm_point(B, sp, synth, a.M, a.K, a.N, s, a.seed, steps, cublas=(s == 0.5)))
+        cub = sweep[2].get("cublas_us")
+        for p in sweep:
+            p["speedup_vs_cublas"] = cub / p["us"] if cub else None
+        res["sparsity_sweep"] = {"shape": f"{a.M}x{a.K}x{a.N}", "points": sweep,
+                                 "t_s03_over_t_s07": sweep[0]["us"] / sweep[4]["us"]}
+    # config 4: OPT-66B layer shards, s = 0.5, N = 16
+    shards = []
+    Gs = (1, 2, 4, 8) if world == 1 else (world,)
+    for G in Gs:
+        for i, (name, M, K) in enumerate(tp.opt_layer_shapes("opt-66b")):
+            r = rank if world > 1 else 0
+            b, c = sp.tp_rows(M, G, r)
+            p = spmm_point(B, sp, synth, M, K, 16, 0.5, a.seed + 100 + i, steps, row0=b, rows=c,
+                           world=world if world > 1 else 1, rank=rank)
+            p.update({"layer": name, "G": G})
+            if world > 1:
+                p["us"] = B.allmax(p["us"])
+                p["frac"] = B.allreduce(p["frac"], "sum") / world
+            shards.append(p)
+    res["opt66b_tp_shards"] = {"note": ("per-rank shard of each OPT-66B layer (rank 0 of G on this GPU)" if world == 1
+                                        else "every rank its own shard; us = max over ranks, frac = mean over ranks"),
+                               "points": shards}
+    res["opt30b_stack"] = stack(a, B, sp, synth, tp)
+    if world == 1:
+        res["host_us_per_call"] = host_cost(B, sp, synth)
+    return res
+
+
+def stack(a, B, sp, synth, tp):
+    """Config 5: OPT-30B QKV -> O (Q block) -> FC1 -> FC2 at s = 0.6, N = 16, TP = world, every
+    layer's output all-gathered (NCCL) — the whole stack captured in one CUDA graph."""
+    torch = B.torch
+    world, rank = B.world, B.rank
+    N, s = 16, 0.6
+    layers = tp.opt_stack_layers("opt-30b", world, rank)
+    wsb = 0
+    for i, L in enumerate(layers):
+        W = synth.weight(L.row_count, L.K, s, seed=a.seed + 200 + i, row0=L.row_begin)
+        Wt = _dev_u16(torch, W, B.dev).view(torch.float16)
+        # ~1/sqrt(fan-in) scale keeps activations O(1) through the stack (input recipe, DESIGN.md)
+        Wt = (Wt.float() * (3.0 / (L.K * (1.0 - s))) ** 0.5).half()
+        L.shard = sp.encode(Wt)
+        wsb = max(wsb, sp.workspace_bytes(max(L.row_count, GT), L.K, N))
+        del W, Wt
+    ws = torch.zeros(max(wsb, 256), dtype=torch.uint8, device=B.dev)
+    for L in layers:
+        L.ws = ws
+    X = _dev_u16(torch, synth.activation(layers[0].K, N, seed=a.seed + 1), B.dev).view(torch.float16)
+    outs = [torch.empty((L.M, N), dtype=torch.float16, device=B.dev) for L in layers]
+    group = None
+
+    def eager(gather=True):
+        tp.run_stack(layers, X, world, rank, group=group, outputs=outs, gather=gather)
+
+    for _ in range(3):
+        eager()
+    torch.cuda.synchronize()
+    steps = max(5, min(a.steps, 20))
+    out = {"model": "opt-30b", "s": s, "N": N, "tp": world,
+           "layers": [f"{L.name} {L.M}x{L.K} rows {L.row_begin}+{L.row_count}" for L in layers]}
+    t_spmm = statistics.median(B.timed(lambda: eager(False), steps))
+    out["spmm_only_us"] = B.allmax(t_spmm * 1e3)
+    graph = None
+    try:
+        cs = torch.cuda.Stream()
+        cs.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(cs):
+            eager()
+        torch.cuda.current_stream().wait_stream(cs)
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph):
+            eager()
+        torch.cuda.synchronize()
+        out["cuda_graph"] = True
+    except Exception as e:  # capture unsupported: time the eager stack and say why
+        graph = None
+        out["cuda_graph"] = False
+        out["graph_error"] = f"{type(e).__name__}: {e}"[:200]
+    fn = graph.replay if graph is not None else eager
+    for _ in range(3):
+        fn()
+    t_all = statistics.median(B.timed(fn, steps))
+    out["stack_us"] = B.allmax(t_all * 1e3)
+    out["gather_overhead_us"] = out["stack_us"] - out["spmm_only_us"] if world > 1 else 0.0
+    nb = sum(algorithmic_bytes(L.row_count, L.K, N, L.shard.n_values) for L in layers)
+    out["spmm_frac_of_roofline"] = nb / (t_spmm * 1e-3) / 1e9 / load_peaks()[0]
+    return out
+
+
+def host_cost(B, sp, synth):
+    """Host µs per spinfer_spmm call through the Python binding + C ABI (launch only, no sync),
+    on a shape whose kernel is shorter than the host loop would allow to queue up."""
+    torch = B.torch
+    M, K, N = 1152, 9216, 16
+    T = sp.encode(_dev_u16(torch, synth.weight(M, K, 0.5, seed=5), B.dev))
+    X = _dev_u16(torch, synth.activation(K, N, seed=6), B.dev).view(torch.float16)
+    Y = torch.empty((M, N), dtype=torch.float16, device=B.dev)
+    ws = sp.workspace(M, K, N, B.dev)
+    for _ in range(20):
+        sp.spmm(T, X, Y, ws=ws)
+    torch.cuda.synchronize()
+    n = 200
+    t0 = time.perf_counter()
+    for _ in range(n):
+        sp.spmm(T, X, Y, ws=ws)
+    t1 = time.perf_counter()
+    torch.cuda.synchronize()
+    return {"shape": f"{M}x{K}x{N}", "us": (t1 - t0) / n * 1e6, "calls": n}
+
+
+def run_ours(a, rank, world, local_rank):
+    import torch
+    import synth
+    import paper_conf_eurosys_fanydlgww025_b200 as sp
+    from paper_conf_eurosys_fanydlgww025_b200 import tp
+
+    for o in a.opt:
+        k, v = o.split("=", 1)
+        sp.set_option(k, v if k == "kernel" else int(v))
+    B = Bench(world, rank, local_rank)
+    dev = B.dev
+    M, K, N = a.M, a.K, a.N
+    b0, c0 = sp.tp_rows(M, world, rank)          # this rank's rows (all of them at N = 1)
+    W = synth.weight(c0, K, a.sparsity, seed=a.seed, row0=b0)
+    X = synth.activation(K, N, seed=a.seed + 1)
+    T = sp.encode(_dev_u16(torch, W, dev))
+    Xd = _dev_u16(torch, X, dev).view(torch.float16)
+    ws = sp.workspace(c0, K, N, dev)
+    Yd = torch.empty((M, N), dtype=torch.float16, device=dev)
+
     def step():
-        sp.spmm(T, Xd, Yd, ws)
+        sp.spmm_tp(T, Xd, Yd, M, world, rank, ws=ws)
 
     for _ in range(max(a.warmup, 3)):
         step()
     torch.cuda.synchronize()
-
     if a.profile:
         for _ in range(a.steps):
             step()
@@ -258,71 +471,58 @@ def run_ours(a, rank, world, local_rank):
     except Exception:
         uuid = None
     with ClockSampler(local_rank, uuid) as clk:
-        t_ms = timed(step, a.steps, do_flush=True)
+        t_ms = B.timed(step, a.steps)
     kern_ms = statistics.mean(t_ms)
     kern_med = statistics.median(t_ms)
-
-    # max over ranks
-    tt = torch.tensor([kern_ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-    kmax = float(tt.item())
-    total_bytes = nbytes * world
+    kmax = B.allmax(kern_ms)
+    nv_total = int(B.allreduce(T.n_values, "sum"))
+    rank_bytes = algorithmic_bytes(c0, K, N, T.n_values)
+    total_bytes = algorithmic_bytes(M, K, N, nv_total)     # config 2's algorithmic bytes (X counted once)
     value = total_bytes / (kmax * 1e-3) / 1e9
-
     peak, peak_kind = load_peaks()
-    achieved = nbytes / (kern_ms * 1e-3) / 1e9
+    achieved = rank_bytes / (kern_ms * 1e-3) / 1e9            # this rank's kernel: per-launch bytes / mean duration
 
-    # e2e through the public API with host buffers: H2D X (pinned) + SpMM + D2H Y (pinned)
+    # e2e through the public API with host buffers: H2D X (pinned) + SpMM + D2H of this rank's Y rows
     e2e = None
     if not a.no_e2e:
         Xh = torch.from_numpy(X.view(np.int16)).pin_memory()
-        Yh = torch.empty((M, N), dtype=torch.int16).pin_memory()
+        Yh = torch.empty((c0, N), dtype=torch.int16).pin_memory()
         Xe = torch.empty((K, N), dtype=torch.int16, device=dev)
 
         def e2e_step():
             Xe.copy_(Xh, non_blocking=True)
-            sp.spmm(T, Xe, Yd, ws)
-            Yh.copy_(Yd.view(torch.int16), non_blocking=True)
+            sp.spmm_tp(T, Xe, Yd, M, world, rank, ws=ws)
+            Yh.copy_(Yd[b0:b0 + c0].view(torch.int16), non_blocking=True)
 
         for _ in range(3):
             e2e_step()
-        e_ms = timed(e2e_step, a.steps, do_flush=True)
-        em = torch.tensor([statistics.mean(e_ms)], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(em, op=dist.ReduceOp.MAX)
-        e2e = {"value": total_bytes / (float(em.item()) * 1e-3) / 1e9, "unit": UNIT,
+        e_ms = B.timed(e2e_step, a.steps)
+        em = B.allmax(statistics.mean(e_ms))
+        e2e = {"value": total_bytes / (em * 1e-3) / 1e9, "unit": UNIT,
                "h2d_bytes_per_step": int(Xh.numel() * 2), "d2h_bytes_per_step": int(Yh.numel() * 2),
-               "ms_per_step": float(em.item())}
-        # e2e result must equal the device-resident result
-        assert torch.equal(Yh, Yd.view(torch.int16).cpu())
+               "ms_per_step": em}
+        assert torch.equal(Yh, Yd[b0:b0 + c0].view(torch.int16).cpu())   # same result as the resident run
 
-    # cuBLAS fp16 dense GEMM on the same shape, same protocol
+    # cuBLAS fp16 dense GEMM on this rank's rows, same protocol
     cublas = None
-    if not a.no_cublas and rank == 0:
+    if not a.no_cublas:
         torch.backends.cuda.matmul.allow_fp16_reduced_precision_reduction = False
         Wdense = sp.decode(T)
-        Yc = torch.empty((M, N), dtype=torch.float16, device=dev)
-
-        def cub():
-            torch.mm(Wdense, Xd, out=Yc)
-
+        Yc = torch.empty((c0, N), dtype=torch.float16, device=dev)
         for _ in range(3):
-            cub()
-        c_ms = timed(cub, a.steps, do_flush=True) if world == 1 else None
-        if c_ms:
-            cm = statistics.mean(c_ms)
-            cublas = {"us": cm * 1e3, "dense_bytes": 2 * M * K + 2 * K * N + 2 * M * N,
-                      "gbs_dense": (2 * M * K + 2 * K * N + 2 * M * N) / (cm * 1e-3) / 1e9,
-                      "speedup_spmm_vs_cublas": cm / kern_ms}
+            torch.mm(Wdense, Xd, out=Yc)
+        c_ms = B.timed(lambda: torch.mm(Wdense, Xd, out=Yc), a.steps)
+        cm = B.allmax(statistics.mean(c_ms))
+        dense_bytes = 2 * M * K + 2 * K * N + 2 * M * N
+        cublas = {"us": cm * 1e3, "dense_bytes": dense_bytes, "gbs_dense": dense_bytes / (cm * 1e-3) / 1e9,
+                  "speedup_spmm_vs_cublas": cm / kmax}
         del Wdense
 
     cpu = None
     if not a.no_cpu_baseline and rank == 0 and world == 1:
         import oracle
-        rows = 8192
-        Wc = W[:rows]
-        Tc = oracle.encode(Wc)
+        rows = 14336
+        Tc = oracle.encode(np.ascontiguousarray(W[:rows]))
         t0 = time.perf_counter()
         oracle.spmm_f64(Tc, X)
         dt = time.perf_counter() - t0
@@ -330,37 +530,47 @@ def run_ours(a, rank, world, local_rank):
         cpu = {"value": algorithmic_bytes(rows, K, N, Tc.n_values) / dt / 1e9, "unit": UNIT, "cores": 1,
                "kind": "oracle", "seconds": dt, "cpu_model": model, "host_cpus": ncpu,
                "sample": f"first {rows} of {M} rows of W (all {K} cols), N={N}: oracle.spmm_f64, single thread"}
+    del W
 
-    # ncu DRAM traffic for this kernel/config, if a committed capture exists
+    # ncu DRAM traffic of this kernel/config from the committed full capture, if any
     traffic = None
-    tp = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tp):
+    tp_path = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp_path) and world == 1:
         try:
-            d = json.load(open(tp))
-            traffic = d.get(workload_name(a))
+            traffic = json.load(open(tp_path)).get(workload_name(a))
         except Exception:
             traffic = None
 
+    ext = None if a.no_extras else extras(a, B, sp, synth, tp)
+    launches = a.steps * (2 if N % 8 else 1)   # the SpMM kernel (+ the X zero-padding kernel when N % 8)
+
     if rank != 0:
         return None
-    return {
+    out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
-        "ms_per_step": kmax, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-        "dtype": "f16 in / f32 acc", "data": "synthetic",
+        "ms_per_step": kmax, "higher_is_better": True, "scaling": "strong" if world > 1 else "weak",
+        "vs_baseline": None, "dtype": "f16 in / f32 acc", "data": "synthetic",
         "config": {"workload": workload_name(a), "M": M, "K": K, "N": N, "sparsity": a.sparsity,
-                   "nnz": T.nnz, "n_values": T.n_values, "seed": a.seed, "l2": "flushed before each step: 256 MiB memset, then a 256 MiB read (cold, clean L2)",
-                   "parallelism": f"row-partitioned x{world} (weak, no collective)" if world > 1 else "1 GPU"},
-        "us_per_spmm": kmax * 1e3, "us_median": kern_med * 1e3, "us_steps": [round(x * 1e3, 1) for x in t_ms],
-        "tflops_dense_equiv": 2 * M * K * N / (kern_ms * 1e-3) / 1e12,
-        "frac_of_8tbs": achieved / 8000.0,
+                   "nnz_rank0": T.nnz, "n_values_total": nv_total, "seed": a.seed,
+                   "l2": "flushed before each step: 256 MiB memset, then a 256 MiB read (cold, clean L2)",
+                   "parallelism": (f"row-partitioned x{world} (spinfer_spmm_tp, strong scaling, no collective)"
+                                   if world > 1 else "1 GPU"),
+                   "rank0_rows": [b0, c0], "options": a.opt},
+        "us_per_spmm": kmax * 1e3, "us_median_rank0": kern_med * 1e3, "us_steps_rank0": [round(x * 1e3, 1) for x in t_ms],
+        "tflops_dense_equiv": 2 * M * K * N / (kmax * 1e-3) / 1e12,
+        "frac_of_8tbs": value / 8000.0,
         "cublas_fp16": cublas,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "peak_kind": peak_kind, "bytes_per_launch": nbytes, "traffic": traffic},
+                     "peak_kind": peak_kind, "bytes_per_launch": rank_bytes, "traffic": traffic,
+                     "kernel": "k_spmm_dw (N <= 16) / k_spmm_tc (N > 16), rank 0"},
         "cpu_baseline": cpu,
         "e2e": e2e,
-        "gpu_launches": a.steps,
+        "gpu_launches": launches,
         "clocks": clk.summary(),
     }
+    if ext:
+        out.update(ext)
+    return out
 
 
 def main():
@@ -371,6 +581,8 @@ def main():
     if a.impl == "reference":
         out = run_reference(a, rank)
     else:
+        if a.gpus > 1 and "WORLD_SIZE" not in os.environ:
+            sys.exit(relaunch(a))
         if world > 1:
             import torch
             import torch.distributed as dist

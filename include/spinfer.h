@@ -136,6 +136,19 @@ SPINFER_API int spinfer_spmm_ex(const spinfer_tca *T, const uint16_t *X, uint16_
  * row), sizes differ by at most 64; ranks beyond the GT-row count get 0 rows (host only). */
 SPINFER_API int spinfer_tp_rows(int M, int world, int rank, int *row_begin /* host */, int *row_count /* host */);
 
+/* Zero-copy row shard of a TCA-BME matrix (P:196 — GroupTiles are stored
+ * row-major, so the GT rows [row_begin/64, ceil((row_begin+row_count)/64)) are one contiguous
+ * slice of all three arrays). row_begin must be a multiple of 64, row_count a multiple of 64
+ * unless the shard ends at T->M (the ragged tail, A8); typically the span
+ * spinfer_tp_rows returns. Writes the shard's GTileOffset, rebased to start at 0, into
+ * offset_out (caller-allocated DEVICE int32[ceil(row_count/64) * ceil(K/64) + 1], 16-byte
+ * aligned) and fills *out (host): M = row_count, K, n_values and max_gt_values (T's, an upper
+ * bound) set, nnz = -1 (unknown), bitmap and values pointing INTO T's arrays (aligned: every
+ * GroupTile's values start at a multiple of 8 halves). T's buffers must outlive *out.
+ * Synchronizes `stream` (the shard's value count is read back). */
+SPINFER_API int spinfer_tca_shard(const spinfer_tca *T, int row_begin, int row_count, int32_t *offset_out,
+                                  spinfer_tca *out /* host */, void *stream);
+
 /* Row-partitioned SpMM: T_shard encodes W[row_begin : row_begin+row_count, :]
  * (as returned by spinfer_tp_rows(M_full, world, rank)); writes ONLY those rows
  * of Y_full [M_full][N]. Performs no communication: the caller gathers Y_full

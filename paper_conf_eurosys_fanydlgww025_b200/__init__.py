@@ -43,7 +43,7 @@ _lib = None
 
 # Exported symbols (must match include/spinfer.h; checked by tests/test_abi.py).
 SYMBOLS = ["spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spinfer_spmm_workspace_bytes",
-           "spinfer_spmm", "spinfer_spmm_ex", "spinfer_tp_rows", "spinfer_spmm_tp", "spinfer_spmm_check",
+           "spinfer_spmm", "spinfer_spmm_ex", "spinfer_tp_rows", "spinfer_tca_shard", "spinfer_spmm_tp", "spinfer_spmm_check",
            "spinfer_set_option", "spinfer_get_option", "spinfer_status_str", "spinfer_version"]
 
 # spinfer.h SPINFER_OPT_* / SPINFER_KERNEL_*
@@ -72,13 +72,15 @@ def lib() -> ctypes.CDLL:
     L.spinfer_tp_rows.argtypes = [i32, i32, i32, P(ctypes.c_int), P(ctypes.c_int)]
     L.spinfer_spmm_tp.argtypes = [P(_Tca), vp, vp, i32, i32, i32, i32, i32, vp, sz, vp]
     L.spinfer_spmm_check.argtypes = [vp, P(ctypes.c_int32), vp]
+    L.spinfer_tca_shard.argtypes = [P(_Tca), i32, i32, vp, P(_Tca), vp]
     L.spinfer_set_option.argtypes = [i32, i32]
     L.spinfer_get_option.argtypes = [i32]
     L.spinfer_status_str.argtypes = [i32]
     L.spinfer_status_str.restype = ctypes.c_char_p
     L.spinfer_version.restype = ctypes.c_char_p
     for f in ("spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spinfer_spmm", "spinfer_spmm_ex",
-              "spinfer_tp_rows", "spinfer_spmm_tp", "spinfer_spmm_check", "spinfer_set_option", "spinfer_get_option"):
+              "spinfer_tp_rows", "spinfer_tca_shard", "spinfer_spmm_tp", "spinfer_spmm_check", "spinfer_set_option",
+              "spinfer_get_option"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -125,22 +127,21 @@ class TCA:
     def storage_bytes(self) -> int:
         return storage_bytes(self.M, self.K, self.n_values)
 
-    def shard(self, row_begin: int, row_count: int) -> "TCA":
-        """Zero-copy row shard: GT rows [a, b) are a contiguous slice of all three
-        arrays; GTileOffset is rebased (on device) by the shard's first offset."""
-        if row_begin % GT or (row_count % GT and row_begin + row_count != self.M):
-            raise ValueError("shard rows must be multiples of 64 (except a ragged tail ending at M)")
+    def shard(self, row_begin: int, row_count: int, stream=None) -> "TCA":
+        """Zero-copy row shard (spinfer_tca_shard): bitmap and values are views into this
+        matrix's tensors, GTileOffset a new rebased tensor. One host synchronization."""
         KG = -(-self.K // GT)
-        a, b = row_begin // GT, -(-(row_begin + row_count) // GT)
-        off = self.gtile_offset[a * KG: b * KG + 1]
-        base = int(off[0].item())
-        end = int(off[-1].item())
-        new_off = (off - base).contiguous()
-        vals = self.values[base:max(end, base + 8)]
-        if base % 8:
-            raise AssertionError("GT value segments are 16-byte aligned by construction")
-        return TCA(row_count, self.K, new_off, self.bitmap[a * KG * 64: b * KG * 64], vals, end - base, -1,
-                   self.max_gt_values)
+        off = torch.empty((-(-row_count // GT)) * KG + 1, dtype=torch.int32, device=self.bitmap.device)
+        cs, out = self.c_struct(), _Tca()
+        with torch.cuda.device(off.device):
+            _check(lib().spinfer_tca_shard(ctypes.byref(cs), row_begin, row_count, off.data_ptr(), ctypes.byref(out),
+                                           _stream(stream)), "spinfer_tca_shard")
+        esz = self.bitmap.element_size()
+        bm0 = (out.bitmap - self.bitmap.data_ptr()) // esz
+        v0 = (out.values - self.values.data_ptr()) // self.values.element_size()
+        nv = int(out.n_values)
+        return TCA(row_count, self.K, off, self.bitmap[bm0: bm0 + 64 * (off.numel() - 1)],
+                   self.values[v0: v0 + max(nv, 8)], nv, -1, self.max_gt_values)
 
 
 def storage_bytes(M: int, K: int, n_values: int) -> int:
@@ -202,8 +203,6 @@ def workspace(M: int, K: int, N: int, device=None, stream=None) -> torch.Tensor:
     with torch.cuda.device(dev):
         need = max(int(lib().spinfer_spmm_workspace_bytes(M, K, N)), 256)
         key = (dev, _stream(stream))
-    if need <= 256 and (M <= 0 or K <= 0 or not 1 <= N <= 32):
-        raise ValueError(f"no workspace for M/K/N = {M}/{K}/{N}")
     ws = _ws_cache.get(key)
     if ws is None or ws.numel() < need:
         ws = torch.zeros(need, dtype=torch.uint8, device=dev)

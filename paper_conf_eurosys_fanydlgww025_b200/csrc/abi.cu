@@ -114,6 +114,38 @@ int spinfer_tp_rows(int M, int world, int rank, int *row_begin, int *row_count) 
     return SPINFER_OK;
 }
 
+int spinfer_tca_shard(const spinfer_tca *T, int row_begin, int row_count, int32_t *offset_out, spinfer_tca *out,
+                      void *stream) {
+    if (!T || !out || !offset_out) return SPINFER_EINVAL;
+    int rc = validate_tca(T, T->M, T->K);
+    if (rc) return rc;
+    if (row_begin < 0 || row_count <= 0 || row_begin % kGT || row_begin + row_count > T->M ||
+        (row_count % kGT && row_begin + row_count != T->M) || !aligned16(offset_out))
+        return SPINFER_EINVAL;
+    if ((rc = check_device())) return rc;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    const int64_t KG = (T->K + kGT - 1) / kGT;
+    const int64_t a = row_begin / kGT, b = (row_begin + row_count + kGT - 1) / kGT;
+    int32_t ends[2] = {0, 0};
+    if (cudaMemcpyAsync(&ends[0], T->gtile_offset + a * KG, 4, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        cudaMemcpyAsync(&ends[1], T->gtile_offset + b * KG, 4, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        launch_rebase_offsets(T->gtile_offset, a * KG, (b - a) * KG, offset_out, st) != SPINFER_OK ||
+        cudaStreamSynchronize(st) != cudaSuccess) {
+        cudaGetLastError();
+        return SPINFER_ECUDA;
+    }
+    if (ends[0] < 0 || ends[1] < ends[0] || ends[1] > T->n_values || ends[0] % 8) return SPINFER_EINVAL;
+    spinfer_tca o = *T;
+    o.M = row_count;
+    o.nnz = -1;
+    o.n_values = ends[1] - ends[0];
+    o.gtile_offset = offset_out;
+    o.bitmap = T->bitmap + a * KG * 64;
+    o.values = T->values + ends[0];
+    *out = o;
+    return SPINFER_OK;
+}
+
 int spinfer_spmm_tp(const spinfer_tca *T_shard, const uint16_t *X, uint16_t *Y_full, int M_full, int K, int N,
                     int world, int rank, void *workspace, size_t ws_bytes, void *stream) {
     int b = 0, c = 0;

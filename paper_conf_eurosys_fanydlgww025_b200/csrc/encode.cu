@@ -7,6 +7,7 @@
 // major in the GT; BT b = bi%4 column-major in the TCTile, TL/BL/TR/BR,
 // P:192). Bit 8*i + j of the BT's bitmap is element (row i, col j).
 // Each thread reads its BT as 8 x 16-byte rows (one uint4 per row).
+#include <algorithm>
 #include "internal.cuh"
 
 namespace spinfer {
@@ -209,7 +210,20 @@ __global__ void __launch_bounds__(kThreads) k_decode(const int32_t *__restrict__
     }
 }
 
+// Row shard (P-E5): out[i] = off[g0 + i] - off[g0], i in [0, n]
+__global__ void k_rebase_offsets(const int32_t *__restrict__ off, int64_t g0, int64_t n, int32_t *__restrict__ out) {
+    const int32_t base = off[g0];
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = off[g0 + i] - base;
+}
+
 }  // namespace
+
+int launch_rebase_offsets(const int32_t *off, int64_t g0, int64_t n, int32_t *out, cudaStream_t st) {
+    const int64_t blocks = std::min<int64_t>((n + 1 + 255) / 256, 1024);
+    k_rebase_offsets<<<(int)blocks, 256, 0, st>>>(off, g0, n, out);
+    return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
+}
 
 int launch_encode_count(const uint16_t *W, int M, int K, int32_t *gtile_offset, int64_t *stats_dev,
                         cudaStream_t st) {

@@ -19,6 +19,7 @@ int launch_encode_count(const uint16_t *W, int M, int K, int32_t *gtile_offset, 
                         cudaStream_t st);
 int launch_encode_fill(const uint16_t *W, const spinfer_tca *T, cudaStream_t st);
 int launch_decode(const spinfer_tca *T, uint16_t *W_out, cudaStream_t st);
+int launch_rebase_offsets(const int32_t *off, int64_t g0, int64_t n, int32_t *out, cudaStream_t st);
 
 // Workspace head shared by the SpMM kernels: int32 GT-row counters [0, kErrWord) and, at word
 // kErrWord, the error word (non-zero after a call that met corrupt TCA-BME input).

@@ -55,6 +55,9 @@ constexpr uint32_t kHdrBytes = 64;        // per-slot stage header: value offset
 constexpr uint32_t kTblBytes = 1024;      // one GroupTile's SMBD table (64 BTs x 2 halves x 8 B)
 // shared-memory map (bytes from the 1024-aligned base)
 constexpr uint32_t kBarFull = 0, kBarEmpty = 64, kBarSegFull = 128, kBarSegFree = 192, kSegMask = 224;
+constexpr uint32_t kFinFlag = 256;        // [2] final segment: partial count if this CTA sums the GT row
+constexpr uint32_t kDefer = 272;          // count + [<= 4] (grow | nparts << 16): cross-CTA sums left to the consumers
+constexpr uint32_t kBarIdDefer = 11;      // named barrier: reducer done -> consumers read the deferred list
 constexpr uint32_t kHdrStop = 1u << 16, kHdrBad = 1u << 17;   // header word 1: g | rows << 8 | flags
 constexpr uint32_t kOffHdr = 1024;
 constexpr uint32_t kOffTbl = kOffHdr + kMaxSd * kHdrBytes;   // per-warp SMBD tables
@@ -91,6 +94,7 @@ struct DParams {
 constexpr int kProfW = 20;
 constexpr size_t kTraceOff = 1024 * kProfW * 8;   // stage trace of CTA 0 after the counters
 [[maybe_unused]] constexpr size_t kEvOff = kTraceOff + 256 * 4;      // per-warp event trace of CTA 0: [16 warps][64 stages][6]
+[[maybe_unused]] constexpr size_t kGtOff = kEvOff + 16 * 64 * 6;    // per CTA [1024][4]: globaltimer at entry, max exit
 struct Prof {
 #if SPINFER_INSTRUMENT
     long long c[8] = {0, 0, 0, 0, 0, 0, 0, 0};
@@ -113,7 +117,15 @@ struct Prof {
     __device__ __forceinline__ void ev(long long *prof, int p, int w, int i, int k) {
         if (prof && p == 0 && w < 16 && i < 64) prof[kEvOff + ((size_t)w * 64 + i) * 6 + k] = clock64() - t0;
     }
+    // globaltimer (ns) at CTA entry (k = 0) and the latest exit of role k (1 consumers, 2 producers, 3 reducer)
+    __device__ __forceinline__ void gt(long long *prof, int p, int k) {
+        if (!prof || p >= 1024) return;
+        unsigned long long g;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
+        atomicMax(reinterpret_cast<unsigned long long *>(prof) + kGtOff + (size_t)p * 4 + k, g);
+    }
 #else
+    __device__ __forceinline__ void gt(long long *, int, int) {}
     __device__ __forceinline__ void ev(long long *, int, int, int, int) {}
     __device__ __forceinline__ void start() {}
     __device__ __forceinline__ void lap(int) {}
@@ -267,50 +279,60 @@ __device__ __forceinline__ void stg_f4(float4 *p, float4 v) {
 __device__ __forceinline__ void stg_f2(float *p, float x, float y) {
     asm volatile("st.global.v2.f32 [%0], {%1, %2};" ::"l"(p), "f"(x), "f"(y) : "memory");
 }
-__device__ __forceinline__ float4 ldg_cg4(const float4 *p) {
-    float4 v;
-    asm volatile("ld.global.cg.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p)
-                 : "memory");
-    return v;
-}
 // Drop an L2 line without writing it back: every partial is read exactly once.
 __device__ __forceinline__ void discard_l2(const void *p) {
     asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory");
 }
-// The CTA partial of GT row `grow` (row-major 64 x Np fp32) is parked; count the CTA and, as the
-// last of the CTAs overlapping the rowblock, sum all CTA partials in CTA order and write Y.
-// Called by one whole warp after every lane's stores are ordered before it (syncwarp/barrier).
-template <int NT, bool EPI>
-__device__ __forceinline__ void cta_count_and_sum(const DParams &prm, int rb, int grow, int lane) {
-    constexpr int Np = NT * 8, kF4 = 64 * Np / 4;
+// The CTA partial of GT row `grow` (row-major 64 x Np fp32) is parked: count this CTA. True for
+// the last of the CTAs overlapping the rowblock, which then sums all CTA partials (cta_sum) and
+// re-zeroes the counter. One whole warp, after every partial store is ordered before it.
+__device__ __forceinline__ bool cta_arrive(const DParams &prm, int rb, int grow, int lane, int &nparts) {
     const int pf = uowner(rb * prm.KG, prm.U, prm.P), pl = uowner((rb + 1) * prm.KG - 1, prm.U, prm.P);
+    nparts = pl - pf + 1;
     __threadfence();
     int old = 0;
     if (lane == 0) old = atomicAdd(prm.ws_cnt + grow, 1);
     old = __shfl_sync(0xffffffffu, old, 0);
-    if (old != pl - pf) return;
-    __threadfence();   // acquire: every CTA partial is visible
-    const float4 *base = reinterpret_cast<const float4 *>(prm.ws_cta) + (size_t)grow * prm.cslots * kF4;
-    constexpr int kPer = kF4 / 32;   // float4 per lane
-    float4 s[kPer];
+    if (old != pl - pf) return false;
+    if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed for the next call
+    __threadfence();                       // acquire: every CTA partial is visible
+    return true;
+}
+// Sum, in CTA order, of the nparts CTA partials of GT row `grow` over the float4 columns
+// [f0, f0 + 32 J) of the row-major 64 x Np block, written to Y. The loads of 4 partials are in
+// flight together (the sum is latency-bound: up to ~20 partials on a long-K shard).
+template <int NT, bool EPI, int J>
+__device__ __forceinline__ void cta_sum(const DParams &prm, int grow, int nparts, int f0, int lane) {
+    constexpr int Np = NT * 8, kF4 = 64 * Np / 4;
+    const float4 *base = reinterpret_cast<const float4 *>(prm.ws_cta) + (size_t)grow * prm.cslots * kF4 + f0 + lane;
+    float4 s[J];
 #pragma unroll
-    for (int t = 0; t < kPer; ++t) s[t] = make_float4(0.f, 0.f, 0.f, 0.f);
-    for (int q = 0; q <= pl - pf; ++q) {
+    for (int j = 0; j < J; ++j) s[j] = make_float4(0.f, 0.f, 0.f, 0.f);
+    auto add = [](float4 &x, const float4 y) { x.x += y.x; x.y += y.y; x.z += y.z; x.w += y.w; };
+    int q = 0;
+    for (; q + 4 <= nparts; q += 4) {
+        float4 v[4][J];
 #pragma unroll
-        for (int t = 0; t < kPer; ++t) {
-            const float4 v = ldg_cg4(base + (size_t)q * kF4 + t * 32 + lane);
-            s[t].x += v.x; s[t].y += v.y; s[t].z += v.z; s[t].w += v.w;
-        }
+        for (int u = 0; u < 4; ++u)
+#pragma unroll
+            for (int j = 0; j < J; ++j) v[u][j] = __ldcg(base + (size_t)(q + u) * kF4 + 32 * j);
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+#pragma unroll
+            for (int j = 0; j < J; ++j) add(s[j], v[u][j]);
     }
+    for (; q < nparts; ++q)
 #pragma unroll
-    for (int t = 0; t < kPer; ++t) {
-        const int e = 4 * (t * 32 + lane);   // element index in the row-major 64 x Np block
-        const float v[4] = {s[t].x, s[t].y, s[t].z, s[t].w};
+        for (int j = 0; j < J; ++j) add(s[j], __ldcg(base + (size_t)q * kF4 + 32 * j));
+#pragma unroll
+    for (int j = 0; j < J; ++j) {
+        const int e = 4 * (f0 + 32 * j + lane);   // element index in the row-major 64 x Np block
+        const float v[4] = {s[j].x, s[j].y, s[j].z, s[j].w};
         store_cols<NT, EPI, 4>(prm, grow * 64 + e / Np, e % Np, v);
     }
-    for (int q = 0; q <= pl - pf; ++q)
-        if (lane < kF4 / 8) discard_l2(base + (size_t)q * kF4 + 8 * lane);
-    if (lane == 0) prm.ws_cnt[grow] = 0;   // leave the workspace zeroed for the next call
+    // every partial line is read exactly once: drop it from L2 without a write-back
+    for (int q2 = 0; q2 < nparts; ++q2)
+        if (lane < 4 * J) discard_l2(base - lane + (size_t)q2 * kF4 + 8 * lane);
 }
 
 template <int NT, bool EPI>
@@ -341,11 +363,13 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             sts_u32(seg_mask + 8 * k, 0u);
             sts_u32(seg_mask + 8 * k + 4, 0u);
         }
+        sts_u32(sbase + kDefer, 0u);
         fence_barrier_init();
     }
     __syncthreads();
     Prof pf;
     pf.start();
+    if (threadIdx.x == 0) pf.gt(prm.prof, p, 0);
     // role warps: producers / reducer / idle. Each branch below ends in a return.
     if (warp >= kCWd) {
     if (warp == kCWd + 3) return;   // the idle warp (completes the warpgroup)
@@ -457,17 +481,22 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             skip2(ia, nsa, ia_i);
             pf.lap(5);
         }
-        // stop sentinel in the slot of the first stage index >= the stage count with this parity;
-        // its header carries the CTA's segment count
+        // stop sentinels: one per consumer phase, in the slots of the stage indices [nst, nst + 8 / G)
+        // (S >= 8 / G: distinct slots); this producer writes those of its parity. The header
+        // carries the CTA's segment count.
         {
-            if ((i & 1) != q) ++i;   // the loop can stop one index short of this producer's parity
-            const uint32_t slot = (uint32_t)(i % S);
-            if (i >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + ((owners_pk >> (4 * slot)) & 15u)));
-            if (lane == 0) {
-                sts_v4(sbase + kOffHdr + slot * kHdrBytes, make_uint4(0u, kHdrStop, (uint32_t)nseg, 0u));
-                mbar_arrive(bar_full + 8 * slot);
+            const int nst = i;                      // the loop ends with i = the stage count
+            for (int j = nst + ((nst & 1) != q ? 1 : 0); j < nst + 8 / G; j += 2) {
+                const uint32_t slot = (uint32_t)(j % S);
+                if (j >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + ((owners_pk >> (4 * slot)) & 15u)));
+                owners_pk &= ~(15u << (4 * slot));
+                if (lane == 0) {
+                    sts_v4(sbase + kOffHdr + slot * kHdrBytes, make_uint4(0u, kHdrStop, (uint32_t)nseg, 0u));
+                    mbar_arrive(bar_full + 8 * slot);
+                }
             }
         }
+        if (lane == 0) pf.gt(prm.prof, p, 2);
         pf.mark(6);
         pf.dump(prm.prof, p, warp, lane);
         return;
@@ -505,20 +534,27 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                     for (int b = 0; b < NT; ++b)
 #pragma unroll
                         for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
-                for (int m = 0; m < 8; ++m) {
-                    if (!((cmask >> m) & 1u)) continue;
+                // warp order; a warp without a GT of the segment contributes +0 (sums start at +0:
+                // adding +0 changes no bit). Four warps' loads in flight together.
 #pragma unroll
-                    for (int tr = 0; tr < 4; ++tr) {
-                        float4 v[NT];
+                for (int tr = 0; tr < 4; ++tr)
 #pragma unroll
-                        for (int nt = 0; nt < NT; ++nt) v[nt] = ldg_cg4(src + (size_t)m * kF4 + (tr * NT + nt) * 32 + lane);
+                    for (int mh = 0; mh < 8; mh += 4) {
+                        float4 v[4][NT];
 #pragma unroll
-                        for (int nt = 0; nt < NT; ++nt) {
-                            const float4 w = v[nt];
-                            acc[tr][nt][0] += w.x; acc[tr][nt][1] += w.y; acc[tr][nt][2] += w.z; acc[tr][nt][3] += w.w;
-                        }
+                        for (int u = 0; u < 4; ++u)
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt)
+                                v[u][nt] = ((cmask >> (mh + u)) & 1u) ? __ldcg(src + (size_t)(mh + u) * kF4 + (tr * NT + nt) * 32 + lane)
+                                                                      : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+                        for (int u = 0; u < 4; ++u)
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt) {
+                                const float4 w = v[u][nt];
+                                acc[tr][nt][0] += w.x; acc[tr][nt][1] += w.y; acc[tr][nt][2] += w.z; acc[tr][nt][3] += w.w;
+                            }
                     }
-                }
                 for (int m = 0; m < 8; ++m)
                     if (((cmask >> m) & 1u) && lane < kF4 / 8) discard_l2(src + (size_t)m * kF4 + 8 * lane);
                 const int grow = kRd * rb + r;
@@ -536,14 +572,25 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                             stg_f2(dst + (row + 8) * Np + col, acc[tr][nt][2], acc[tr][nt][3]);
                         }
                     __syncwarp();
-                    cta_count_and_sum<NT, EPI>(prm, rb, grow, lane);
+                    // the last CTA of the rowblock: the sum is deferred to the consumer warps' end
+                    // phase (8 warps per GT row, all loads in flight; a single warp here would be
+                    // latency-bound over up to ~20 partials)
+                    int nparts;
+                    if (cta_arrive(prm, rb, grow, lane, nparts) && lane == 0) {
+                        const uint32_t nd = lds_u32(sbase + kDefer);
+                        sts_u32(sbase + kDefer + 4 + 4 * nd, (uint32_t)grow | ((uint32_t)nparts << 16));
+                        sts_u32(sbase + kDefer, nd + 1);
+                    }
                 }
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(bar_sfree + 8 * k);   // the slot's partials may be overwritten
             ++nseg;
         }
+        __syncwarp();
+        named_bar_arrive(kBarIdDefer, 32u * (kCWd + 1));   // the deferred-sum list is complete
         pf.lap(1);
+        if (lane == 0) pf.gt(prm.prof, p, 3);
         pf.mark(6);
         pf.dump(prm.prof, p, warp, lane);
         return;
@@ -552,9 +599,11 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     }   // role warps
 
     // ---------------------------------------------------------------------- consumers
-    // Warp (r, m) owns GT j = m % 4 of GT row r in every stage i with i % 2 == m / 4; it reads the
-    // stage's shape and segment index from the slot header.
-    const int r = warp >> 3, m = warp & 7, jw = m & 3;
+    // Warp (r, m) owns GT j = m % G of GT row r in every stage i with i % (8 / G) == m / G
+    // (G in {1, 2, 4}: all 8 warps of a row busy); it reads the stage's shape and segment index
+    // from the slot header.
+    const int r = warp >> 3, m = warp & 7, jw = m % G;
+    const int tstride = 8 / G;   // stages between two of this warp's
     const uint32_t mulc = opaque_u32(1u << (30u - 2u * (uint32_t)(lane & 15)));   // z = w << (30 - sh) on the FMA pipe
     constexpr uint32_t selA = kSelA, selB = kSelB, selC = kSelC;   // IMAD immediates
     constexpr uint32_t cpr = Np / 8;   // 16-byte chunks per X row
@@ -651,7 +700,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         return true;
     };
 
-    int i = m >> 2;                 // stage index
+    int i = m / G;                  // stage index
     uint32_t slot = (uint32_t)(i % S), ph = 0;   // ring position of stage i (S >= 2)
     int cur = -1;                   // open segment of this warp (-1: none)
     bool contrib = false, seen = false;
@@ -735,8 +784,8 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             if (lane == 0) pf.st(prm.prof, p, i, 2, true);
             if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 5);
         }
-        i += 2;
-        slot += 2;
+        i += tstride;
+        slot += (uint32_t)tstride;
         if (slot >= (uint32_t)S) { slot -= (uint32_t)S; ph ^= 1u; }
     }
     // segments after this warp's last stage: close the non-final ones it did not see
@@ -810,9 +859,26 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     }
     if (fseg >= 0 && !fcomplete) {
         named_bar_sync(2, 32 * kCWd);   // every warp's slice of the CTA partial is stored
-        if (m == 0 && r < frows) cta_count_and_sum<NT, EPI>(prm, frb, kRd * frb + r, lane);
+        int nparts = 0;
+        if (m == 0 && r < frows) {
+            const bool last = cta_arrive(prm, frb, kRd * frb + r, lane, nparts);
+            if (lane == 0) sts_u32(sbase + kFinFlag + 4 * r, last ? (uint32_t)nparts : 0u);
+        }
+        named_bar_sync(1, 32 * kCWd);
+        // the last CTA of the rowblock: the row's warps sum 32 float4 columns each (all in flight)
+        nparts = (int)lds_u32(sbase + kFinFlag + 4 * r);
+        if (nparts && r < frows && m * 32 < kF4) cta_sum<NT, EPI, 1>(prm, kRd * frb + r, nparts, m * 32, lane);
+    }
+    // cross-CTA sums of non-final segments whose last contributor was this CTA (the reducer's list):
+    // GT row e is summed by the 8 warps of consumer row e % 2
+    named_bar_sync(kBarIdDefer, 32u * (kCWd + 1));
+    const int ndef = (int)lds_u32(sbase + kDefer);
+    for (int e = r; e < ndef; e += kRd) {
+        const uint32_t d = lds_u32(sbase + kDefer + 4 + 4 * e);
+        if (m * 32 < kF4) cta_sum<NT, EPI, 1>(prm, (int)(d & 0xFFFFu), (int)(d >> 16), m * 32, lane);
     }
     pf.lap(3);
+    if (lane == 0) pf.gt(prm.prof, p, 1);
     pf.mark(6);
     pf.dump(prm.prof, p, warp, lane);
 }
@@ -832,7 +898,7 @@ int cta_slots(long long U, int P, int KG) {
 }
 
 // Ring sizing: each slot holds the X slab (1024-aligned for the swizzle), both GT rows'
-// bitmaps and value capacity G * max_gt_values; prefer G = 4 with >= 4 slots.
+// bitmaps and value capacity G * max_gt_values.
 bool make_dplan(int M, int K, int Np, int max_gt_values, DPlan *pl) {
     const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;
     if (KG > 65535 || MG >= kErrWord) return false;
@@ -849,17 +915,19 @@ bool make_dplan(int M, int K, int Np, int max_gt_values, DPlan *pl) {
     if (option(SPINFER_OPT_STAGE_G) > 0) gmax = std::max(1, std::min(kMaxGd, option(SPINFER_OPT_STAGE_G)));
     if (option(SPINFER_OPT_STAGE_S) > 0) smax = std::max(2, std::min(kMaxSd, option(SPINFER_OPT_STAGE_S)));
     const uint32_t final_scratch = 2u * 8u * 64u * Np * 4u;   // the final segment's partials reuse the ring
-    int bestG = 0, bestS = 0;   // the largest G with >= 4 slots, else the deepest ring with >= 2
-    for (int G = gmax; G >= 1; --G) {
+    // G in {4, 2, 1} (8 / G consumer phases keep all 8 warps of a GT row busy); the largest G
+    // with >= 4 slots, else the deepest valid ring. A ring needs >= 8 / G slots (one stop
+    // sentinel per phase) and an even slot count (producer q always refills its own stages'
+    // slots: the slot release barrier counts the GT owners of the stage it issued there).
+    int bestG = 0, bestS = 0;
+    for (int G = gmax >= 4 ? 4 : gmax >= 2 ? 2 : 1; G >= 1; G >>= 1) {
         const uint32_t st_bm = al((uint32_t)G * 64 * Np * 2, 128);
         const uint32_t vcap = al((uint32_t)G * maxv * 2, 128);
         const uint32_t slot = al(st_bm + kRd * G * 512 + 2 * vcap, 1024);
-        // an even slot count: producer q always refills its own stages' slots (the slot release
-        // barrier counts the GT owners of the stage that producer issued there)
         const int S = (int)std::min<long long>(smax, ((long long)smem_max - kOffRing - 1024) / slot) & ~1;
-        if ((uint32_t)S * slot < final_scratch) continue;
+        if ((uint32_t)S * slot < final_scratch || S < std::max(2, 8 / G)) continue;
         if (S >= 4) { bestG = G; bestS = S; break; }
-        if (S >= 2 && S > bestS) { bestG = G; bestS = S; }
+        if (S > bestS) { bestG = G; bestS = S; }
     }
     if (bestG == 0) return false;
     const int G = bestG, S = bestS;
@@ -953,7 +1021,7 @@ int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, 
 #if SPINFER_INSTRUMENT
     if (const char *path = getenv("SPINFER_PROF")) {   // experiments: dump per-warp cycle counters
         static long long *prof_buf = nullptr;
-        const size_t n = kEvOff + 16 * 64 * 6;
+        const size_t n = kGtOff + 1024 * 4;
         if (!prof_buf && cudaMalloc(&prof_buf, n * 8) != cudaSuccess) return SPINFER_ECUDA;
         cudaMemsetAsync(prof_buf, 0, n * 8, st);
         q.prof = prof_buf;

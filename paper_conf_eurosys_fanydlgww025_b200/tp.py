@@ -29,14 +29,11 @@ GT = 64
 
 
 def tp_rows(M: int, world: int, rank: int):
-    """Same partition as spinfer_tp_rows (host logic, no device needed)."""
+    """Rows [b, b + c) of rank `rank` (spinfer_tp_rows: host logic, no device needed)."""
+    import paper_conf_eurosys_fanydlgww025_b200 as sp
     if M <= 0 or world <= 0 or not (0 <= rank < world):
         raise ValueError("bad tp_rows arguments")
-    MG = -(-M // GT)                      # ragged M: zero-padded to whole GroupTiles (reading A8)
-    q, rem = divmod(MG, world)
-    b, c = (rank * q + min(rank, rem)) * GT, (q + (1 if rank < rem else 0)) * GT
-    b = min(b, M)
-    return b, min(c, M - b)               # the ragged tail belongs to the rank owning the last GT row
+    return sp.tp_rows(M, world, rank)
 
 
 @dataclass
@@ -51,6 +48,20 @@ class Layer:
     x_rows: Optional[int] = None  # consume only the first x_rows rows of the previous output (stand-in attention)
     act: Optional[str] = None     # fused epilogue activation ("relu" for the OPT FC1 layers), spinfer_spmm_ex
     bias: object = None           # this rank's bias rows (fp16 [row_count]) or None
+    ws: object = None             # preallocated SpMM workspace (None: the binding's per-stream cache)
+
+
+_scratch: dict = {}
+
+
+def _buffer(key, shape, like: torch.Tensor) -> torch.Tensor:
+    """A scratch tensor reused across calls (no allocation in the per-layer hot loop; allocated
+    on first use, so warm up once before capturing a CUDA graph)."""
+    k = (key, tuple(shape), like.dtype, like.device)
+    t = _scratch.get(k)
+    if t is None:
+        t = _scratch[k] = torch.empty(shape, dtype=like.dtype, device=like.device)
+    return t
 
 
 def gather_rows(Y_full: torch.Tensor, M: int, world: int, rank: int, group=None) -> torch.Tensor:
@@ -62,15 +73,18 @@ def gather_rows(Y_full: torch.Tensor, M: int, world: int, rank: int, group=None)
     b, c = spans[rank]
     mine = Y_full[b:b + c]
     if len(sizes) == 1:
-        # equal chunks: one all_gather_into_tensor straight into Y_full (no copy-out)
-        dist.all_gather_into_tensor(Y_full, mine.clone() if Y_full.is_cuda else mine.contiguous(), group=group)
+        # equal chunks: one all_gather_into_tensor straight into Y_full; the rank's chunk goes
+        # through a reused send buffer (the input must not alias the output)
+        send = _buffer("send", mine.shape, Y_full)
+        send.copy_(mine)
+        dist.all_gather_into_tensor(Y_full, send, group=group)
     else:
         # uneven chunks (M/64 not divisible by world): pad every chunk to the largest one and
         # gather into one buffer (all_gather with unequal sizes is not portable across backends)
         cmax = max(sizes)
-        send = Y_full.new_zeros((cmax,) + tuple(Y_full.shape[1:]))
+        send = _buffer("send_pad", (cmax,) + tuple(Y_full.shape[1:]), Y_full)
         send[:c] = mine
-        recv = Y_full.new_empty((world * cmax,) + tuple(Y_full.shape[1:]))
+        recv = _buffer("recv_pad", (world * cmax,) + tuple(Y_full.shape[1:]), Y_full)
         dist.all_gather_into_tensor(recv, send, group=group)
         for r, (bb, cc) in enumerate(spans):
             if r != rank:
@@ -81,12 +95,12 @@ def gather_rows(Y_full: torch.Tensor, M: int, world: int, rank: int, group=None)
 def gpu_spmm_fn(layer: Layer, X: torch.Tensor, Y_full: torch.Tensor, world: int, rank: int):
     import paper_conf_eurosys_fanydlgww025_b200 as sp
     if layer.act is None and layer.bias is None:
-        sp.spmm_tp(layer.shard, X, Y_full, layer.M, world, rank)
+        sp.spmm_tp(layer.shard, X, Y_full, layer.M, world, rank, ws=layer.ws)
     else:
         # the rank's rows of Y_full are one contiguous [row_count][N] block: the fused-epilogue
         # SpMM writes straight into it (what spinfer_spmm_tp does for the plain SpMM)
         b, c = tp_rows(layer.M, world, rank)
-        sp.spmm(layer.shard, X, Y_full[b:b + c], bias=layer.bias, act=layer.act)
+        sp.spmm(layer.shard, X, Y_full[b:b + c], ws=layer.ws, bias=layer.bias, act=layer.act)
 
 
 def run_stack(layers: Sequence[Layer], X: torch.Tensor, world: int, rank: int, group=None,

@@ -35,6 +35,8 @@ def _load():
         u16p = ctypes.POINTER(ctypes.c_uint16)
         lib.synth_weight.argtypes = [u16p, ctypes.c_int64, ctypes.c_int64, ctypes.c_uint64,
                                      ctypes.c_double, ctypes.c_int, ctypes.c_int]
+        lib.synth_weight_rows.argtypes = [u16p, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_uint64,
+                                          ctypes.c_double, ctypes.c_int, ctypes.c_int]
         lib.synth_activation.argtypes = [u16p, ctypes.c_int64, ctypes.c_int64, ctypes.c_uint64,
                                          ctypes.c_int, ctypes.c_int]
         lib.synth_hash.argtypes = [ctypes.c_uint64] * 3
@@ -56,12 +58,13 @@ def _ptr(a: np.ndarray):
 
 
 def weight(M: int, K: int, sparsity: float, seed: int = DEFAULT_SEED, mode: str = "uniform",
-           out: np.ndarray | None = None) -> np.ndarray:
-    """Dense fp16 W [M][K] (uint16 bits) with an i.i.d. Bernoulli(1-s) keep-mask."""
+           out: np.ndarray | None = None, row0: int = 0) -> np.ndarray:
+    """Dense fp16 W [M][K] (uint16 bits) with an i.i.d. Bernoulli(1-s) keep-mask. row0 > 0: rows
+    [row0, row0 + M) of the matrix drawn with the same seed (a row shard, identical elements)."""
     lib = _load()
     W = out if out is not None else np.empty((M, K), dtype=np.uint16)
     assert W.dtype == np.uint16 and W.shape == (M, K) and W.flags.c_contiguous
-    rc = lib.synth_weight(_ptr(W), M, K, seed, float(sparsity), 1 if mode == "int" else 0, _threads())
+    rc = lib.synth_weight_rows(_ptr(W), row0, M, K, seed, float(sparsity), 1 if mode == "int" else 0, _threads())
     if rc != 0:
         raise ValueError("synth_weight failed")
     return W

@@ -74,7 +74,7 @@ static inline double unit_m11(uint64_t h) {       /* uniform in [-1, 1) */
 }
 
 typedef struct {
-    uint16_t *out; int64_t rows, cols, r0, r1;
+    uint16_t *out; int64_t rows, cols, r0, r1, row_off;
     uint64_t seed; double s; int mode; int which; /* which: 0 = W, 1 = X */
 } job_t;
 
@@ -84,7 +84,7 @@ static void *worker(void *arg) {
     const uint64_t k1 = sm64(j->seed) ^ sm64(1), k2 = sm64(j->seed) ^ sm64(2), k3 = sm64(j->seed) ^ sm64(3);
     for (int64_t i = j->r0; i < j->r1; ++i) {
         for (int64_t c = 0; c < j->cols; ++c) {
-            uint64_t idx = (uint64_t)(i * j->cols + c);
+            uint64_t idx = (uint64_t)((i + j->row_off) * j->cols + c);   /* index in the full matrix */
             uint16_t bits;
             if (j->which == 0) {
                 uint64_t hk = sm64(k1 + idx);
@@ -114,15 +114,15 @@ static void *worker(void *arg) {
     return NULL;
 }
 
-static int run(uint16_t *out, int64_t rows, int64_t cols, uint64_t seed, double s,
+static int run(uint16_t *out, int64_t row_off, int64_t rows, int64_t cols, uint64_t seed, double s,
                int mode, int which, int nthreads) {
-    if (!out || rows < 0 || cols < 0) return -1;
+    if (!out || rows < 0 || cols < 0 || row_off < 0) return -1;
     if (nthreads < 1) nthreads = 1;
     if (nthreads > 256) nthreads = 256;
     if ((int64_t)nthreads > rows) nthreads = rows > 0 ? (int)rows : 1;
     pthread_t th[256]; job_t jb[256];
     for (int t = 0; t < nthreads; ++t) {
-        jb[t] = (job_t){ out, rows, cols, rows * t / nthreads, rows * (t + 1) / nthreads, seed, s, mode, which };
+        jb[t] = (job_t){ out, rows, cols, rows * t / nthreads, rows * (t + 1) / nthreads, row_off, seed, s, mode, which };
         if (nthreads == 1) { worker(&jb[t]); return 0; }
         pthread_create(&th[t], NULL, worker, &jb[t]);
     }
@@ -134,10 +134,17 @@ static int run(uint16_t *out, int64_t rows, int64_t cols, uint64_t seed, double 
 int synth_weight(uint16_t *W, int64_t rows, int64_t cols, uint64_t seed, double sparsity,
                  int mode, int nthreads) {
     if (!(sparsity >= 0.0 && sparsity <= 1.0)) return -1;
-    return run(W, rows, cols, seed, sparsity, mode, 0, nthreads);
+    return run(W, 0, rows, cols, seed, sparsity, mode, 0, nthreads);
+}
+
+/* Rows [row0, row0 + rows) of the W above (a row shard without generating the whole matrix). */
+int synth_weight_rows(uint16_t *W, int64_t row0, int64_t rows, int64_t cols, uint64_t seed, double sparsity,
+                      int mode, int nthreads) {
+    if (!(sparsity >= 0.0 && sparsity <= 1.0)) return -1;
+    return run(W, row0, rows, cols, seed, sparsity, mode, 0, nthreads);
 }
 
 /* X: [rows][cols] row-major fp16 bits, dense. */
 int synth_activation(uint16_t *X, int64_t rows, int64_t cols, uint64_t seed, int mode, int nthreads) {
-    return run(X, rows, cols, seed, 0.0, mode, 1, nthreads);
+    return run(X, 0, rows, cols, seed, 0.0, mode, 1, nthreads);
 }

@@ -57,3 +57,12 @@ def test_int_mode_values():
     assert set(np.unique(v)) <= {-2.0, -1.0, 0.0, 1.0, 2.0}
     X = synth.activation(128, 16, seed=2, mode="int")
     assert set(np.unique(X.view(np.float16).astype(np.float64))) <= {-1.0, 0.0, 1.0}
+
+
+def test_weight_row_shard_equals_rows_of_full_matrix():
+    """synth.weight(row0=...) draws rows [row0, row0 + M) of the same matrix (per-rank shards in
+    bench.py are the rows spinfer_tp_rows assigns, without generating the whole weight)."""
+    for mode in ("uniform", "int"):
+        W = synth.weight(320, 200, 0.5, seed=11, mode=mode)
+        for b, c in [(0, 64), (64, 128), (192, 128), (300, 20)]:
+            assert np.array_equal(synth.weight(c, 200, 0.5, seed=11, mode=mode, row0=b), W[b:b + c])

@@ -47,7 +47,7 @@ for i in range(min(nst, 256)):
 print("CTA 0 warps:")
 for w in range(20):
     print("  w%2d " % w + " ".join(f"{n}={a[0, w, k]}" for k, n in enumerate(names)))
-ev = raw[1024 * 20 * 8 + 256 * 4:].reshape(16, 64, 6)
+ev = raw[1024 * 20 * 8 + 256 * 4:1024 * 20 * 8 + 256 * 4 + 16 * 64 * 6].reshape(16, 64, 6)
 for w in (0, 5):
     print(f"warp {w} events (cycles): own-stage k: wait_start +wait +header/seg +scan +decode +arrive")
     for k in range(64):
@@ -55,3 +55,13 @@ for w in (0, 5):
         if e[0] == 0 and e[1] == 0: continue
         d = [e[1] - e[0], e[2] - e[1], (e[3] - e[2]) if e[3] else 0, (e[4] - e[3]) if e[4] else 0, (e[5] - e[4]) if e[5] else 0]
         print(f"  {k:2d} t={e[0]:7d} " + " ".join(f"{x:6d}" for x in d))
+# CTA entry / exit (globaltimer ns) relative to the first CTA entry
+kGtOff = 1024 * 20 * 8 + 256 * 4 + 16 * 64 * 6
+gt = raw[kGtOff:kGtOff + 1024 * 4].reshape(1024, 4)[:P].astype(np.int64)
+t0 = gt[:, 0].min()
+ent = (gt[:, 0] - t0) / 1e3
+ex_c, ex_p, ex_r = (gt[:, 1] - t0) / 1e3, (gt[:, 2] - t0) / 1e3, (gt[:, 3] - t0) / 1e3
+print(f"CTA entry (us after first): min {ent.min():.2f} median {np.median(ent):.2f} max {ent.max():.2f}")
+print(f"consumer exit (us): min {ex_c.min():.2f} median {np.median(ex_c):.2f} max {ex_c.max():.2f}; producer max {ex_p.max():.2f}; reducer max {ex_r.max():.2f}")
+o = np.argsort(ent)
+print("latest entries:", [(int(i), round(float(ent[i]), 2)) for i in o[-8:]])
