@@ -36,6 +36,14 @@
 namespace spinfer {
 namespace {
 
+// SPINFER_ABLATION (ablation builds only, tools/ablation.py; the product build leaves it 0):
+//   1: paper-style SMBD (Alg. 2): every lane pops the BitmapTile's bitmap itself with a
+//      serial PopCount base per BT, no warp-scan table; W staged in shared memory as usual;
+//   2: no shared-memory staging of W at all: the same per-lane decode reads bitmaps and values
+//      from global memory (only X is staged).
+#ifndef SPINFER_ABLATION
+#define SPINFER_ABLATION 0
+#endif
 constexpr int kRd = 2;                    // GT rows per rowblock (128 output rows)
 constexpr int kCWd = 16;                  // consumer warps: r = w >> 3, m = w & 7
 constexpr int kProdWarp0 = kCWd;          // producer warps kCWd, kCWd + 2 (SMSPs 0 and 2)
@@ -353,7 +361,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
-            mbar_init(bar_full + 8 * s, 1);              // the producer's arrive.expect_tx (+ TMA bytes)
+            mbar_init(bar_full + 8 * s, 32);             // the producer warp's lanes (lane 0: expect_tx) + TMA bytes
             mbar_init(bar_empty + 8 * s, kRd * kMaxGd);  // the stage's GT owners + the producer's pre-arrival
         }
         for (int k = 0; k < kNSeg; ++k) {
@@ -445,19 +453,26 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             if (orow < kRd && oj <= kMaxGd) sts_u32(hb + 16u + 20u * orow + 4u * oj, 2u * (uint32_t)(oc - obeg));
             if (lane == 31)
                 sts_v4(hb, make_uint4((uint32_t)it.rb, (uint32_t)g | ((uint32_t)rows << 8) | ((bad0 || bad1) ? kHdrBad : 0u),
-                                      (uint32_t)nseg, 0u));
+                                      (uint32_t)nseg, (uint32_t)it.gc));
+#if SPINFER_ABLATION == 2
+            if (oj == 0 && orow < kRd) sts_u32(hb + 56u + 4u * orow, (uint32_t)oc);   // the row's first value (global)
+            const uint32_t vbl = 0u;
+#else
             const uint32_t vbl = (oj == 0 && orow < rows && !bad) ? 2u * (uint32_t)(oend - oc) : 0u;   // lanes 0, 8
+#endif
             const uint32_t vb1 = __shfl_sync(0xffffffffu, vbl, 8);
             // the X slab: one tensor copy of G GT columns (rows past K zero-filled by the TMA)
             const uint32_t xbytes = (uint32_t)G * 64u * Np * 2u;
-            const uint32_t bmb = (uint32_t)g * 512u;
-            __syncwarp();
+            const uint32_t bmb = SPINFER_ABLATION == 2 ? 0u : (uint32_t)g * 512u;
             if (lane == 0) {
                 if (badm) atomicOr(prm.ws_err, 1);
-                // one arrival with every transaction byte registered up front: the phase completes
-                // only when all copies of the stage have landed (release: the header stores above)
+                // every transaction byte registered up front: the phase completes only when all
+                // copies of the stage have landed
                 mbar_arrive_expect_tx(fb, (uint32_t)rows * bmb + xbytes + vbl + vb1);
+            } else {
+                mbar_arrive(fb);   // each lane releases its own header stores
             }
+            __syncwarp();          // expect_tx before any copy is issued
             pf.lap(3);
             uint32_t dst = 0, bytes = 0;
             const void *src = nullptr;
@@ -490,10 +505,8 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                 const uint32_t slot = (uint32_t)(j % S);
                 if (j >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + ((owners_pk >> (4 * slot)) & 15u)));
                 owners_pk &= ~(15u << (4 * slot));
-                if (lane == 0) {
-                    sts_v4(sbase + kOffHdr + slot * kHdrBytes, make_uint4(0u, kHdrStop, (uint32_t)nseg, 0u));
-                    mbar_arrive(bar_full + 8 * slot);
-                }
+                if (lane == 0) sts_v4(sbase + kOffHdr + slot * kHdrBytes, make_uint4(0u, kHdrStop, (uint32_t)nseg, 0u));
+                mbar_arrive(bar_full + 8 * slot);
             }
         }
         if (lane == 0) pf.gt(prm.prof, p, 2);
@@ -525,6 +538,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                 mbar_wait_expo(bar_sfull + 16 * k + 8 * r, par, 256u, 4096u);
                 pf.lap(0);
                 const uint32_t cmask = lds_u32(seg_mask + 8 * k + 4 * r);   // warps that own a GT of the segment
+                __syncwarp();   // every lane has read the mask before it is reset
                 if (lane == 0) sts_u32(seg_mask + 8 * k + 4 * r, 0u);
                 const float4 *src = reinterpret_cast<const float4 *>(prm.ws_seg) + ((((size_t)p * kNSeg + k) * kRd + r) * 8) * kF4;
                 float acc[4][NT][4];
@@ -741,7 +755,12 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 2);
         if (r < rows && jw < g) {
             contrib = true;
+#if SPINFER_ABLATION
+            const bool ok = !(h.y & kHdrBad);
+            (void)ba; (void)bb; (void)vend;
+#else
             const bool ok = scan_gt(st, voff, vend, ba, bb, h.y, tbl);
+#endif
             pf.lap(1);
             if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 3);
             if (ok) {
@@ -751,6 +770,15 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                 const uint32_t xs = launder_u32(st + x_lane + (uint32_t)(64 * jw) * cpr * 16u);
                 const uint32_t tbl_lane_l = launder_u32(tbl_lane);
                 uint32_t t0[8], t1[8], s1[8];
+#if SPINFER_ABLATION
+                uint32_t abl_base = 0;   // values of the GT's earlier BitmapTiles
+                const uint32_t vsm_gt = st + (r ? prm.st_v1 : prm.st_v0) + voff;
+#if SPINFER_ABLATION == 2
+                const uint64_t *gbm = prm.bm + ((size_t)(kRd * (int)h.x + r) * KG + (int)h.w + jw) * 64;
+                const uint16_t *gv = prm.vals + lds_u32(hb + 56u + 4u * (uint32_t)r) + voff / 2u;
+#endif
+                (void)vsm_gt; (void)tbl_lane_l;
+#endif
 #pragma unroll
                 for (int tc = 0; tc < 4; ++tc) {
                     uint32_t bfr[NT][2];
@@ -760,12 +788,43 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                     } else {
                         ldsm_x4_trans_nv(xk, bfr[0][0], bfr[0][1], bfr[1][0], bfr[1][1]);
                     }
+#if SPINFER_ABLATION
+#pragma unroll
+                    for (int hh = 0; hh < 2; ++hh) {
+#pragma unroll
+                        for (int k = 0; k < 8; ++k) {
+                            const int b = tc * 16 + hh * 8 + k;   // BitmapTile index in the GT
+#if SPINFER_ABLATION == 1
+                            const uint2 bw = lds_v2(bms + 8u * (uint32_t)b);
+#else
+                            const uint2 bw = ldg_nc_v2(gbm + b);
+#endif
+                            const uint32_t w = (lane < 16) ? bw.x : bw.y;
+                            const uint32_t pre = abl_base + ((lane >= 16) ? (uint32_t)__popc(bw.x) : 0u);
+                            abl_base += (uint32_t)(__popc(bw.x) + __popc(bw.y));   // serial PopCount base
+                            const uint32_t z = w * mulc;
+                            const uint32_t c2 = pre + (uint32_t)__popc(z);   // values through the lane's pair
+                            const uint32_t y = z >> 30;
+                            s1[k] = y * (y * selB + selA) + selC;
+#if SPINFER_ABLATION == 1
+                            const uint32_t a = vsm_gt + 2u * c2 - 4u;
+                            t0[k] = lds_u16(a);
+                            t1[k] = lds_u16(a + 2u);
+#else
+                            t0[k] = __ldg(gv + (c2 >= 2u ? c2 - 2u : 0u));
+                            t1[k] = __ldg(gv + (c2 >= 1u ? c2 - 1u : 0u));
+#endif
+                        }
+                        assemble_nv(t0, t1, s1, 2 * hh, bfr);
+                    }
+#else
 #pragma unroll
                     for (int hh = 0; hh < 2; ++hh) {
                         load_E_nv(tbl_lane_l + (uint32_t)(tc * 16 + hh * 8) * 8u);
                         issue_to(t0, t1, s1);
                         assemble_nv(t0, t1, s1, 2 * hh, bfr);
                     }
+#endif
                 }
 #pragma unroll
                 for (int a = 0; a < 4; ++a)

@@ -242,9 +242,9 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
             mbar_init(bar_full + 8 * s, 1);
-            mbar_init(bar_empty + 8 * s, kCW);             // every decode warp
+            mbar_init(bar_empty + 8 * s, 32 * kCW);        // every lane of every decode warp (its table reads)
             mbar_init(bar_emptyx + 8 * s, 4);              // the 4 k-teams' MMA commits
-            mbar_init(bar_scan + 8 * s, 1);                // the stage's scan warp
+            mbar_init(bar_scan + 8 * s, 32);               // the stage's scan warp (every lane: its table stores)
         }
         for (int k = 0; k < 4 * ABufs; ++k) mbar_init(bar_ae + 8 * k, 1);   // [k-team][buffer]: team MMA commit
         for (int k = 0; k < 4 * ABufs; ++k) mbar_init(sbase + kTcAFull + 8 * k, 4);   // [k-team][buffer]: A written
@@ -448,7 +448,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
             // publish the table only once the slot's values and X have landed too, so the decode
             // warps wait on one barrier per stage
             mbar_wait_sleep(bar_full + 8 * slot, sg.par());
-            if (lane == 0) mbar_arrive(bar_scan + 8 * slot);
+            mbar_arrive(bar_scan + 8 * slot);
             skip2(it);
             if (it.valid()) fetch(it, cur);   // this warp's next stage
             return true;
@@ -632,7 +632,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         }
         tm_fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(bar_empty + 8 * slot);   // this warp is done with the slot's values/table
+        mbar_arrive(bar_empty + 8 * slot);   // this lane is done with the slot's values/table
         const bool mm = kt < d.g();
         // the team's 4 lane-quarter warps have written their A tiles: the team leader multiplies
         named_bar_sync(kTeamBar + (uint32_t)kt, 128);
