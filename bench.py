@@ -16,7 +16,8 @@ only those rows and writes them into Y (spinfer_spmm_tp; no collective on the da
 value = config 2's algorithmic bytes / max over ranks of the step time. Without WORLD_SIZE in
 the environment, bench.py relaunches itself under torch.distributed.run with N ranks.
 
-Extra keys (--no-extras skips them): the sparsity sweep s = 0.3..0.7 on the config-2 shape,
+Extra keys (--no-extras skips them): the sparsity sweep s = 0.3..0.7 on the config-2 shape, the
+prefill sweep N = 64..4096 (the wide-X tcgen05 kernel) against cuBLAS,
 OPT-66B per-rank shard shapes (config 4: at N = 1 the G = 1/2/4/8 shards of rank 0 on this GPU,
 at N > 1 every rank's own shard, max over ranks), the OPT-30B four-layer stack (config 5) at
 TP = N with the NCCL all-gather of every layer's output, replayed from a CUDA graph, and the
@@ -328,6 +329,14 @@ def extras(a, B, sp, synth, tp):
             p["speedup_vs_cublas"] = cub / p["us"] if cub else None
         res["sparsity_sweep"] = {"shape": f"{a.M}x{a.K}x{a.N}", "points": sweep,
                                  "t_s03_over_t_s07": sweep[0]["us"] / sweep[4]["us"]}
+    if world == 1:
+        # prefill regime: the wide-X tcgen05 kernel vs cuBLAS
+        pre = []
+        for n in (64, 256, 1024, 4096):
+            p = spmm_point(B, sp, synth, a.M, a.K, n, a.sparsity, a.seed, max(3, min(steps, 10)), cublas=True)
+            p["tflops_dense_equiv"] = 2 * a.M * a.K * n / (p["us"] * 1e-6) / 1e12
+            pre.append(p)
+        res["prefill_sweep"] = {"shape": f"{a.M}x{a.K}xN s={a.sparsity}", "kernel": "k_spmm_wide", "points": pre}
     # config 4: OPT-66B layer shards, s = 0.5, N = 16
     shards = []
     Gs = (1, 2, 4, 8) if world == 1 else (world,)

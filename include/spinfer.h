@@ -50,7 +50,7 @@ extern "C" {
 
 typedef enum {
     SPINFER_OK = 0,
-    SPINFER_EINVAL = -1,     /* null pointer, bad shape (M or K <= 0, N not in [1, 32]),
+    SPINFER_EINVAL = -1,     /* null pointer, bad shape (M or K <= 0, N not in [1, 65536]),
                                 misaligned pointer, struct/call mismatch, unknown activation */
     SPINFER_ENOSPC = -2,     /* workspace too small */
     SPINFER_EOVERFLOW = -3,  /* n_values would reach 2^31 (gtile_offset is int32) */
@@ -111,10 +111,14 @@ SPINFER_API size_t spinfer_spmm_workspace_bytes(int M, int K, int N);
 
 /* Y = W x X with fp32 accumulation and one round-to-nearest-even to
  * fp16 per output. X: device fp16 [K][N] row-major; Y: device fp16
- * [M][N] row-major (fully overwritten). 1 <= N <= 32 (decode batch; the
- * kernels compute roundup(N, 8) columns: N not a multiple of 8 costs the same as
- * the next multiple of 8 plus a zero-padded copy of X in the workspace). One persistent kernel launch (stream-K over GroupTiles with an
- * in-kernel split-K fix-up, P:216 / Alg. 1). */
+ * [M][N] row-major (fully overwritten). 1 <= N <= 65536. One persistent kernel launch:
+ *   N <= 16  (decode batch): mma.sync SMBD kernel, stream-K over GroupTiles with an
+ *            in-kernel split-K fix-up (P:216 / Alg. 1);
+ *   N 17-32: the same decomposition on tcgen05 with the accumulators in TMEM;
+ *   N > 32   (prefill): tcgen05 with W decoded into shared memory, 128-row x
+ *            (up to) 512-column output tiles, no split-K.
+ * N not a multiple of 8 costs the same as the next multiple of 8 plus a zero-padded copy of
+ * X in the workspace. */
 SPINFER_API int spinfer_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N,
                  void *workspace, size_t ws_bytes, void *stream);
 
@@ -172,13 +176,15 @@ SPINFER_API int spinfer_spmm_check(void *workspace, int32_t *flags /* host */, v
  *                         1 force the decoupled-warp kernel (N <= 16 only), 2 force tcgen05;
  *   SPINFER_OPT_MAX_CTAS  cap on the persistent grid (0: one CTA per SM);
  *   SPINFER_OPT_STAGE_G   cap on GroupTile columns per pipeline stage (0: the kernel's max);
- *   SPINFER_OPT_STAGE_S   cap on pipeline stages (0: as many as shared memory holds).
+ *   SPINFER_OPT_STAGE_S   cap on pipeline stages (0: as many as shared memory holds);
+ *   SPINFER_OPT_WIDE_BN   N > 32 kernel: cap on the MMA N of a sub-tile (multiple of 16; 0: 256).
  * SPINFER_EINVAL for an unknown key or an out-of-range value. */
 #define SPINFER_OPT_KERNEL 0
 #define SPINFER_OPT_MAX_CTAS 1
 #define SPINFER_OPT_STAGE_G 2
 #define SPINFER_OPT_STAGE_S 3
-#define SPINFER_OPT_COUNT 4
+#define SPINFER_OPT_WIDE_BN 4
+#define SPINFER_OPT_COUNT 5
 #define SPINFER_KERNEL_AUTO 0
 #define SPINFER_KERNEL_DW 1
 #define SPINFER_KERNEL_TC 2

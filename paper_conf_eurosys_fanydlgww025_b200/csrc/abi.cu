@@ -80,13 +80,13 @@ int spinfer_decode(const spinfer_tca *T, uint16_t *W_out, void *stream) {
 }
 
 size_t spinfer_spmm_workspace_bytes(int M, int K, int N) {
-    if (!shape_ok(M, K) || N < 1 || N > 32) return 0;
+    if (!shape_ok(M, K) || N < 1 || N > kMaxN) return 0;
     return spmm_workspace_bytes(M, K, N);
 }
 
 int spinfer_spmm_ex(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N,
                     const uint16_t *bias, int act, void *workspace, size_t ws_bytes, void *stream) {
-    if (!X || !Y || N < 1 || N > 32) return SPINFER_EINVAL;
+    if (!X || !Y || N < 1 || N > kMaxN) return SPINFER_EINVAL;
     if (act != SPINFER_ACT_NONE && act != SPINFER_ACT_RELU) return SPINFER_EINVAL;
     if (bias && (reinterpret_cast<uintptr_t>(bias) & 1u)) return SPINFER_EINVAL;
     if (!aligned16(X) || !aligned16(Y) || (workspace && !aligned16(workspace))) return SPINFER_EINVAL;

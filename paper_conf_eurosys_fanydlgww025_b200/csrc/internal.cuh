@@ -9,6 +9,7 @@ namespace spinfer {
 
 constexpr int kGT = 64;    // GroupTile edge (reading A1)
 constexpr int kNumSMsDefault = 148;
+constexpr int kMaxN = 65536;             // widest X (TMA coordinates and the wide kernel's tiling)
 
 int check_device();        // SPINFER_OK or SPINFER_ENODEV / SPINFER_ECUDA
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
@@ -32,10 +33,16 @@ int set_option(int key, int value);
 int sm_count();                          // SMs of the current device (cached per device)
 int choose_grid(long long units);        // persistent grid size: min(SMs, units)
 int make_x_tmap(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows, bool swizzle);
+int make_x_tmap_box(CUtensorMap *m, const uint16_t *X, int K, int N, int box_n, int box_k, CUtensorMapSwizzle sw);
 int launch_pad_x(const uint16_t *X, uint16_t *Xp, int K, int N, int Np, cudaStream_t st);
 size_t spmm_workspace_bytes(int M, int K, int N);
 int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias, int act, void *ws,
                 size_t ws_bytes, cudaStream_t st);
+
+// spmm_wide.cu (tcgen05 kernel with W decoded into shared memory, N > 32)
+size_t spmm_wide_workspace_bytes(int M, int K, int N);
+int launch_spmm_wide(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias,
+                     int act, void *ws, size_t ws_bytes, cudaStream_t st);
 
 // spmm_tc.cu (tcgen05 kernel, N 17..32)
 size_t spmm_tc_workspace_bytes(int M, int K, int N);

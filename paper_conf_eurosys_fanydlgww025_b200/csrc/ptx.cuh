@@ -96,10 +96,6 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t
         ::"r"(dst), "l"(src), "r"(bytes), "r"(bar), "l"(policy) : "memory");
 }
 
-// cp.async (LDGSTS) 16 B global -> shared, L2 only; completion tracked by an mbarrier:
-// cp.async.mbarrier.arrive.noinc makes the barrier observe one arrival when all of
-// this thread's prior cp.async operations have completed.
-// 2-D TMA tile load (tensor map in param/const space, coordinates innermost first).
 __device__ __forceinline__ void prefetch_l2(const void *p) {
     asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
@@ -108,6 +104,7 @@ __device__ __forceinline__ void prefetch_l2(const void *p) {
 __device__ __forceinline__ void prefetch_tmap(const void *tmap) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(tmap)) : "memory");
 }
+// 2-D TMA tile load (tensor map in param/const space, coordinates innermost first).
 __device__ __forceinline__ void tma_2d_g2s(uint32_t dst, const void *tmap, int c0, int c1, uint32_t bar) {
     asm volatile(
         "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
@@ -250,16 +247,20 @@ __device__ __forceinline__ void umma_f16_ts(uint32_t d_t, uint32_t a_t, uint64_t
                  "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}"
                  ::"r"(d_t), "r"(a_t), "l"(bdesc), "r"(idesc), "r"(acc) : "memory");
 }
+// D[tmem] (+)= A[smem descriptor] x B[smem descriptor]; kind::f16, cta_group::1.
+__device__ __forceinline__ void umma_f16_ss(uint32_t d_t, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}"
+                 ::"r"(d_t), "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc) : "memory");
+}
+// Generic-proxy shared-memory writes made visible to the async proxy (tensor-core operand reads).
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
 // Arrive (once) on `bar` when every tcgen05 operation issued so far by this thread has completed.
 __device__ __forceinline__ void umma_commit(uint32_t bar) {
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
 }
-}  // namespace spinfer
-
-namespace spinfer {
-}  // namespace spinfer
-
-namespace spinfer {
 __device__ __forceinline__ bool elect_one() {
     uint32_t p;
     asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\tselp.u32 %0, 1, 0, e;\n\t}" : "=r"(p));

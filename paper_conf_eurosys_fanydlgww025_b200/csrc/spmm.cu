@@ -1,7 +1,8 @@
 // spmm.cu — host side of the SpMM: kernel choice, workspace sizing, the X tensor map, the
 // zero-padded X copy, and the library options (include/spinfer.h spinfer_set_option).
 //   N <= 16: the decoupled-warp mma.sync kernel (spmm_dw.cu);
-//   N 17..32: the tcgen05 kernel (spmm_tc.cu), accumulators in TMEM.
+//   N 17..32: the tcgen05 kernel (spmm_tc.cu), accumulators in TMEM;
+//   N > 32: the wide (prefill) tcgen05 kernel (spmm_wide.cu), W decoded into shared memory.
 #include <cuda.h>   // CUtensorMap (type + enums only; the encoder comes via cudaGetDriverEntryPoint)
 #include <algorithm>
 #include <atomic>
@@ -59,9 +60,9 @@ int choose_grid(long long units) {
     return (int)std::max(1LL, std::min(cap, units));
 }
 
-// X [K][N] fp16 row-major, box {NX, box_rows}; NX > N reads past the tensor's columns, which the
-// TMA fills with zeros (X padded to the MMA's N without a copy); rows past K are zero-filled too.
-int make_x_tmap(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows, bool swizzle) {
+// X [K][N] fp16 row-major as a 2-D tensor map, box {box_n, box_k}; box columns past N and rows
+// past K are zero-filled by the TMA (X padded to the MMA's N without a copy).
+int make_x_tmap_box(CUtensorMap *m, const uint16_t *X, int K, int N, int box_n, int box_k, CUtensorMapSwizzle sw) {
     static EncodeTiledFn fn = nullptr;
     if (!fn) {
         void *f = nullptr;
@@ -75,16 +76,21 @@ int make_x_tmap(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box
     }
     const cuuint64_t dims[2] = {(cuuint64_t)N, (cuuint64_t)K};
     const cuuint64_t strides[1] = {(cuuint64_t)N * 2};
-    const cuuint32_t box[2] = {(cuuint32_t)NX, (cuuint32_t)box_rows};
+    const cuuint32_t box[2] = {(cuuint32_t)box_n, (cuuint32_t)box_k};
     const cuuint32_t estr[2] = {1u, 1u};
-    // 32B / 64B swizzle: the ldmatrix / MMA-descriptor bank-conflict-free layouts of a 16 / 32 column slab
-    const CUtensorMapSwizzle sw = !swizzle ? CU_TENSOR_MAP_SWIZZLE_NONE
-                                  : NX == 16 ? CU_TENSOR_MAP_SWIZZLE_32B : NX == 32 ? CU_TENSOR_MAP_SWIZZLE_64B
-                                                                                 : CU_TENSOR_MAP_SWIZZLE_NONE;
     CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, const_cast<uint16_t *>(X), dims, strides, box, estr,
                     CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS ? SPINFER_OK : SPINFER_EINVAL;
+}
+
+// The narrow kernels' X slab: box {NX, box_rows}; 32B / 64B swizzle = the ldmatrix / MMA-descriptor
+// bank-conflict-free layouts of a 16 / 32 column slab.
+int make_x_tmap(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows, bool swizzle) {
+    const CUtensorMapSwizzle sw = !swizzle ? CU_TENSOR_MAP_SWIZZLE_NONE
+                                  : NX == 16 ? CU_TENSOR_MAP_SWIZZLE_32B : NX == 32 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                                                 : CU_TENSOR_MAP_SWIZZLE_NONE;
+    return make_x_tmap_box(m, X, K, N, NX, box_rows, sw);
 }
 
 int launch_pad_x(const uint16_t *X, uint16_t *Xp, int K, int N, int Np, cudaStream_t st) {
@@ -93,9 +99,10 @@ int launch_pad_x(const uint16_t *X, uint16_t *Xp, int K, int N, int Np, cudaStre
     return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
 }
 
-// The workspace serves whichever kernel a call picks: the larger of the two layouts.
+// The workspace serves whichever kernel a call picks: the largest of their layouts.
 size_t spmm_workspace_bytes(int M, int K, int N) {
-    if (M <= 0 || K <= 0 || N <= 0 || N > 32 || (M + kGT - 1) / kGT >= kErrWord) return 0;
+    if (M <= 0 || K <= 0 || N <= 0 || N > kMaxN || (M + kGT - 1) / kGT >= kErrWord) return 0;
+    if (N > 32) return spmm_wide_workspace_bytes(M, K, N);
     const size_t tc = spmm_tc_workspace_bytes(M, K, N);
     const size_t dw = N <= 16 ? spmm_dw_workspace_bytes(M, K, N) : 0;
     return std::max(tc, dw);
@@ -107,6 +114,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     // kernel for N <= 16, the tcgen05 kernel for N > 16 (N not a multiple of 8 computes the next
     // multiple of 8 and stores the N real columns). SPINFER_OPT_KERNEL overrides (tests, ablation).
     const int Np = (N + 7) & ~7;
+    if (Np > 32) return launch_spmm_wide(T, X, Y, M, K, N, bias, act, ws, ws_bytes, st);
     const int ko = option(SPINFER_OPT_KERNEL);
     const bool dw = ko == SPINFER_KERNEL_DW ? true : ko == SPINFER_KERNEL_TC ? false : Np <= 16;
     if (dw && Np > 16) return SPINFER_EINVAL;

@@ -222,7 +222,7 @@ def test_spmm_errors():
     import torch
     sp = _sp()
     T = sp.encode(to_dev(synth.weight(128, 128, 0.5)))
-    X = torch.zeros((128, 33), dtype=torch.float16, device="cuda")   # N > 32
+    X = torch.zeros((128, 65537), dtype=torch.float16, device="cuda")   # N > 65536
     with pytest.raises(sp.SpinferError) as e:
         sp.spmm(T, X)
     assert e.value.status == -1

@@ -43,8 +43,8 @@ VARIANTS = [
 NCU_METRICS = ["gpu__time_duration.sum", "dram__throughput.avg.pct_of_peak_sustained_elapsed",
                "smsp__issue_active.avg.pct_of_peak_sustained_active",
                "smsp__average_warp_latency_per_inst_issued.ratio",
-               "sm__pipe_tensor_op_hmma_cycles_active.avg.pct_of_peak_sustained_active",
-               "sm__inst_executed_pipe_uma.avg.pct_of_peak_sustained_active",
+               "sm__pipe_tensor_subpipe_hmma_cycles_active.avg.pct_of_peak_sustained_active",
+               "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active",
                "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum", "smsp__inst_executed.sum"]
 
 
@@ -73,14 +73,7 @@ def run_bench(args, lib):
         return None, None
 
 
-def available_metrics():
-    q = subprocess.run(["ncu", "--query-metrics", "--chip", "gb100"], capture_output=True, text=True).stdout
-    names = {line.split()[0] for line in q.splitlines() if line.strip() and not line.startswith(("-", "Device"))}
-    return names
-
-
 def run_ncu(args, lib, metrics):
-    rep = os.path.join(ROOT, "gpurun_out", "abl_ncu")
     cmd = ["ncu", "--metrics", ",".join(metrics), "--clock-control", "none", "-k", "regex:k_spmm", "-s", "3", "-c", "1",
            "--csv", sys.executable, os.path.join(ROOT, "bench.py"), "--profile", "--steps", "1", "--warmup", "3", *args]
     try:
@@ -115,15 +108,13 @@ def main():
             res[tag].append(run_bench(args, lib))
     ncu = {}
     if not a.no_ncu:
-        have = available_metrics()
-        metrics = [m for m in NCU_METRICS if not have or m in have]
         for tag, _, args, lib in VARIANTS:
-            ncu[tag] = run_ncu(args, lib, metrics)
+            ncu[tag] = run_ncu(args, lib, NCU_METRICS)
     base = [m for m, _ in res["default"] if m]
     base = statistics.mean(base) if base else None
     rows = []
-    hdr = (f"{'variant':10s} {'us(ev)':>7s} {'rel':>6s} {'ncu dur':>7s} {'DRAM%':>6s} {'issue%':>7s} {'cyc/inst':>8s} "
-           f"{'HMMA%':>6s} {'UMMA%':>6s}  what")
+    hdr = (f"{'variant':10s} {'us(ev)':>7s} {'rel':>6s} {'ncu ns':>7s} {'DRAM%':>6s} {'issue%':>7s} {'cyc/inst':>8s} "
+           f"{'HMMA%':>6s} {'TC%':>6s}  what")
     lines = [hdr]
     for tag, what, args, lib in VARIANTS:
         ms = [m for m, _ in res[tag] if m]
@@ -134,14 +125,14 @@ def main():
         rows.append(row)
 
         def f(k):
-            return f"{n[k][0]:.1f}" if k in n else "-"
+            return f"{n[k][0]:.1f}" if k in n else "-"   # value (units in the jsonl)
         rel = row["rel_to_default"]
         lines.append(f"{tag:10s} {(f'{mean:.1f}' if mean else 'failed'):>7s} {(f'{rel:.3f}' if rel else '-'):>6s} "
                      f"{f('gpu__time_duration.sum'):>7s} {f('dram__throughput.avg.pct_of_peak_sustained_elapsed'):>6s} "
                      f"{f('smsp__issue_active.avg.pct_of_peak_sustained_active'):>7s} "
                      f"{f('smsp__average_warp_latency_per_inst_issued.ratio'):>8s} "
-                     f"{f('sm__pipe_tensor_op_hmma_cycles_active.avg.pct_of_peak_sustained_active'):>6s} "
-                     f"{f('sm__inst_executed_pipe_uma.avg.pct_of_peak_sustained_active'):>6s}  {what}")
+                     f"{f('sm__pipe_tensor_subpipe_hmma_cycles_active.avg.pct_of_peak_sustained_active'):>6s} "
+                     f"{f('sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active'):>6s}  {what}")
     print("\n".join(lines))
     if a.out:
         with open(a.out + ".txt", "w") as fh:
