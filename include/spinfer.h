@@ -160,12 +160,34 @@ SPINFER_API int spinfer_tca_shard(const spinfer_tca *T, int row_begin, int row_c
 SPINFER_API int spinfer_spmm_tp(const spinfer_tca *T_shard, const uint16_t *X, uint16_t *Y_full, int M_full,
                     int K, int N, int world, int rank, void *workspace, size_t ws_bytes, void *stream);
 
+/* Fused all-gather epilogue (the exchange the paper blames for its shrinking
+ * multi-GPU gains): spinfer_spmm_tp whose kernel also stores this rank's rows of Y
+ * directly into every rank's Y_full (peer stores over NVLink / NVSwitch, no NCCL), followed by one
+ * release increment of every rank's completion counter.
+ *   Y_full_peers: HOST array [world] of DEVICE pointers: rank r's Y_full [M_full][N] as mapped in
+ *                 this process (CUDA IPC / torch symmetric memory; on one device, plain pointers);
+ *   flag_peers:   HOST array [world] of DEVICE pointers to each rank's uint32 counter (zeroed once).
+ * world <= 8, N <= 16 (the decode regime; SPINFER_EINVAL otherwise), no bias / activation. Rank r's
+ * Y_full holds every rank's rows once its spinfer_gather_wait has returned (on its stream). */
+SPINFER_API int spinfer_spmm_tp_gather(const spinfer_tca *T_shard, const uint16_t *X, uint16_t *const *Y_full_peers,
+                                       int M_full, int K, int N, int world, int rank, uint32_t *const *flag_peers,
+                                       void *workspace, size_t ws_bytes, void *stream);
+
+/* Stream-ordered wait (one device thread) until every rank's signal of the current exchange reached
+ * this rank's counter `flag` (device). `state` (device uint32, zeroed together with the counter)
+ * holds the expected count, so a captured CUDA graph replays the exchange correctly. timeout_us > 0
+ * bounds the wait: on expiry flag 4 is OR-ed into the workspace's error word (if workspace is not
+ * NULL) and the wait returns. */
+SPINFER_API int spinfer_gather_wait(uint32_t *flag, uint32_t *state, int world, void *workspace, uint32_t timeout_us,
+                                    void *stream);
+
 /* Corrupt-input report. The kernels check every stage they load against the TCA-BME
  * invariants (gtile_offset non-decreasing and <= n_values, a GroupTile's popcount equal to
  * its padded value count rounded down by < 8, at most max_gt_values values per GroupTile):
  * a violating stage is not copied / decoded (its rows' contribution is zero, so Y is NOT
  * valid) and a flag is OR-ed into the workspace's error word — 1: gtile_offset out of range
- * or larger than max_gt_values; 2: bitmaps inconsistent with gtile_offset. No out-of-bounds
+ * or larger than max_gt_values; 2: bitmaps inconsistent with gtile_offset; 4: a
+ * spinfer_gather_wait timed out. No out-of-bounds
  * access happens either way. This call copies the error word to *flags (host), resets it to
  * 0 and synchronizes `stream`. */
 SPINFER_API int spinfer_spmm_check(void *workspace, int32_t *flags /* host */, void *stream);

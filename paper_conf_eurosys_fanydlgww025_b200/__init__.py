@@ -14,7 +14,8 @@ from dataclasses import dataclass
 
 import torch
 
-__all__ = ["TCA", "SpinferError", "encode", "decode", "spmm", "spmm_tp", "tp_rows", "workspace",
+__all__ = ["TCA", "SpinferError", "encode", "decode", "spmm", "spmm_tp", "spmm_tp_gather", "gather_wait", "tp_rows",
+           "workspace",
            "workspace_bytes", "storage_bytes", "algorithmic_bytes", "check", "set_option", "get_option",
            "lib", "LIB_PATH"]
 
@@ -43,7 +44,8 @@ _lib = None
 
 # Exported symbols (must match include/spinfer.h; checked by tests/test_abi.py).
 SYMBOLS = ["spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spinfer_spmm_workspace_bytes",
-           "spinfer_spmm", "spinfer_spmm_ex", "spinfer_tp_rows", "spinfer_tca_shard", "spinfer_spmm_tp", "spinfer_spmm_check",
+           "spinfer_spmm", "spinfer_spmm_ex", "spinfer_tp_rows", "spinfer_tca_shard", "spinfer_spmm_tp",
+           "spinfer_spmm_tp_gather", "spinfer_gather_wait", "spinfer_spmm_check",
            "spinfer_set_option", "spinfer_get_option", "spinfer_status_str", "spinfer_version"]
 
 # spinfer.h SPINFER_OPT_* / SPINFER_KERNEL_*
@@ -73,14 +75,16 @@ def lib() -> ctypes.CDLL:
     L.spinfer_spmm_tp.argtypes = [P(_Tca), vp, vp, i32, i32, i32, i32, i32, vp, sz, vp]
     L.spinfer_spmm_check.argtypes = [vp, P(ctypes.c_int32), vp]
     L.spinfer_tca_shard.argtypes = [P(_Tca), i32, i32, vp, P(_Tca), vp]
+    L.spinfer_spmm_tp_gather.argtypes = [P(_Tca), vp, P(vp), i32, i32, i32, i32, i32, P(vp), vp, sz, vp]
+    L.spinfer_gather_wait.argtypes = [vp, vp, i32, vp, ctypes.c_uint32, vp]
     L.spinfer_set_option.argtypes = [i32, i32]
     L.spinfer_get_option.argtypes = [i32]
     L.spinfer_status_str.argtypes = [i32]
     L.spinfer_status_str.restype = ctypes.c_char_p
     L.spinfer_version.restype = ctypes.c_char_p
     for f in ("spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spinfer_spmm", "spinfer_spmm_ex",
-              "spinfer_tp_rows", "spinfer_tca_shard", "spinfer_spmm_tp", "spinfer_spmm_check", "spinfer_set_option",
-              "spinfer_get_option"):
+              "spinfer_tp_rows", "spinfer_tca_shard", "spinfer_spmm_tp", "spinfer_spmm_tp_gather", "spinfer_gather_wait",
+              "spinfer_spmm_check", "spinfer_set_option", "spinfer_get_option"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -91,9 +95,33 @@ def _check(rc: int, what: str):
         raise SpinferError(rc, what)
 
 
+_raw_stream = getattr(torch._C, "_cuda_getCurrentRawStream", None)
+_cur_dev = getattr(torch._C, "_cuda_getDevice", None) or torch.cuda.current_device
+
+
 def _stream(stream=None) -> int:
+    if stream is None and _raw_stream is not None:
+        return int(_raw_stream(_cur_dev()))   # the current stream's handle without a Stream object
     s = stream if stream is not None else torch.cuda.current_stream()
     return int(s.cuda_stream)
+
+
+class _NoCtx:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        return False
+
+
+_NOCTX = _NoCtx()
+_U16 = (torch.float16, torch.int16, torch.uint16)
+
+
+def _on(dev: torch.device):
+    """torch.cuda.device(dev) only when it is not already current (the context switch costs
+    microseconds per call)."""
+    return _NOCTX if dev.index == _cur_dev() else torch.cuda.device(dev)
 
 
 def _dev_u16(t: torch.Tensor, name: str) -> torch.Tensor:
@@ -121,8 +149,14 @@ class TCA:
     max_gt_values: int
 
     def c_struct(self) -> _Tca:
-        return _Tca(self.M, self.K, GT, GT, self.nnz, self.n_values, self.max_gt_values, 0,
-                    self.gtile_offset.data_ptr(), self.bitmap.data_ptr(), self.values.data_ptr())
+        key = (self.M, self.K, self.nnz, self.n_values, self.max_gt_values, id(self.gtile_offset), id(self.bitmap),
+               id(self.values))
+        c = self.__dict__.get("_cs")
+        if c is None or c[0] != key:   # built once per matrix (the host cost of a call matters at TP sizes)
+            c = (key, _Tca(self.M, self.K, GT, GT, self.nnz, self.n_values, self.max_gt_values, 0,
+                           self.gtile_offset.data_ptr(), self.bitmap.data_ptr(), self.values.data_ptr()))
+            self.__dict__["_cs"] = c
+        return c[1]
 
     def storage_bytes(self) -> int:
         return storage_bytes(self.M, self.K, self.n_values)
@@ -196,12 +230,19 @@ def workspace_bytes(M: int, K: int, N: int) -> int:
 _ws_cache: dict = {}
 
 
+_ws_need: dict = {}
+
+
 def workspace(M: int, K: int, N: int, device=None, stream=None) -> torch.Tensor:
     """A zero-filled workspace for spinfer_spmm, cached per (device, stream): calls on one stream
     are ordered, so they may share one; two streams never do (spinfer.h)."""
     dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
-    with torch.cuda.device(dev):
-        need = max(int(lib().spinfer_spmm_workspace_bytes(M, K, N)), 256)
+    with _on(dev):
+        opts = tuple(int(lib().spinfer_get_option(i)) for i in (OPTIONS["max_ctas"],))
+        nk = (dev, M, K, N, opts)
+        need = _ws_need.get(nk)
+        if need is None:
+            need = _ws_need[nk] = max(int(lib().spinfer_spmm_workspace_bytes(M, K, N)), 256)
         key = (dev, _stream(stream))
     ws = _ws_cache.get(key)
     if ws is None or ws.numel() < need:
@@ -236,29 +277,35 @@ def _same_device(X: torch.Tensor, name: str, t: torch.Tensor):
 
 
 ACT_NONE, ACT_RELU = 0, 1   # spinfer.h SPINFER_ACT_*
+_ACTS = {None: ACT_NONE, "none": ACT_NONE, "relu": ACT_RELU}
 
 
 def spmm(T: TCA, X: torch.Tensor, Y: torch.Tensor | None = None, ws: torch.Tensor | None = None,
          stream=None, bias: torch.Tensor | None = None, act: str | None = None) -> torch.Tensor:
     """Y = act(W X + bias): X fp16 [K][N] (CUDA), 1 <= N <= 32; bias fp16 [M] or
     None; act None or "relu" (fused into the SpMM epilogue, spinfer_spmm_ex); returns fp16 [M][N]."""
-    X = _dev_u16(X, "X")
-    if X.dim() != 2:
-        raise ValueError("X must be 2-D [K][N]")
+    if not (X.is_cuda and X.dtype in _U16 and X.dim() == 2 and X.is_contiguous()):
+        X = _dev_u16(X, "X")
+        if X.dim() != 2:
+            raise ValueError("X must be 2-D [K][N]")
     K, N = X.shape
     if K != T.K:
         raise ValueError(f"X has K={K}, W has K={T.K}")
-    _same_device(X, "W", T.bitmap)
+    dev = X.device
+    if T.bitmap.device != dev:
+        _same_device(X, "W", T.bitmap)
     if Y is None:
-        Y = torch.empty((T.M, N), dtype=torch.float16, device=X.device)
-    Yv = _dev_u16(Y, "Y")
-    if tuple(Yv.shape) != (T.M, N):
+        Y = torch.empty((T.M, N), dtype=torch.float16, device=dev)
+    Yv = Y if (Y.is_cuda and Y.dtype in _U16 and Y.is_contiguous()) else _dev_u16(Y, "Y")
+    if Yv.shape != (T.M, N):
         raise ValueError(f"Y has shape {tuple(Yv.shape)}, expected {(T.M, N)}")
-    _same_device(X, "Y", Yv)
+    if Yv.device != dev:
+        _same_device(X, "Y", Yv)
     if ws is None:
-        ws = workspace(T.M, T.K, N, X.device, stream)
-    _same_device(X, "workspace", ws)
-    actc = {None: ACT_NONE, "none": ACT_NONE, "relu": ACT_RELU}[act]
+        ws = workspace(T.M, T.K, N, dev, stream)
+    if ws.device != dev:
+        _same_device(X, "workspace", ws)
+    actc = _ACTS[act]
     bptr = None
     if bias is not None:
         bv = _dev_u16(bias, "bias")
@@ -267,7 +314,7 @@ def spmm(T: TCA, X: torch.Tensor, Y: torch.Tensor | None = None, ws: torch.Tenso
             raise ValueError(f"bias has {bv.numel()} entries, W has M={T.M}")
         bptr = bv.data_ptr()
     cs = T.c_struct()
-    with torch.cuda.device(X.device):
+    with _on(dev):
         if bptr is None and actc == ACT_NONE:
             _check(lib().spinfer_spmm(ctypes.byref(cs), X.data_ptr(), Yv.data_ptr(), T.M, T.K, N, ws.data_ptr(),
                                       ws.numel(), _stream(stream)), "spinfer_spmm")
@@ -303,3 +350,36 @@ def spmm_tp(T_shard: TCA, X: torch.Tensor, Y_full: torch.Tensor, M_full: int, wo
         _check(lib().spinfer_spmm_tp(ctypes.byref(cs), X.data_ptr(), Yv.data_ptr(), M_full, K, N, world, rank,
                                      ws.data_ptr(), ws.numel(), _stream(stream)), "spinfer_spmm_tp")
     return Y_full
+
+
+def _ptr(x) -> int:
+    return x.data_ptr() if isinstance(x, torch.Tensor) else int(x)
+
+
+def spmm_tp_gather(T_shard: TCA, X: torch.Tensor, Y_peers, M_full: int, world: int, rank: int, flag_peers,
+                   ws: torch.Tensor | None = None, stream=None):
+    """Fused all-gather epilogue (spinfer_spmm_tp_gather): this rank's rows of W X are stored into every
+    rank's Y_full (Y_peers[r]: tensor or device address of rank r's [M_full][N] buffer as mapped here),
+    then every rank's counter (flag_peers[r]) is signalled. N <= 16."""
+    X = _dev_u16(X, "X")
+    if X.dim() != 2:
+        raise ValueError("X must be 2-D [K][N]")
+    K, N = X.shape
+    if len(Y_peers) != world or len(flag_peers) != world:
+        raise ValueError("one Y buffer and one counter per rank")
+    if ws is None:
+        ws = workspace(max(T_shard.M, GT), K, N, X.device, stream)
+    yp = (ctypes.c_void_p * world)(*[_ptr(y) for y in Y_peers])
+    fp = (ctypes.c_void_p * world)(*[_ptr(f) for f in flag_peers])
+    cs = T_shard.c_struct()
+    with torch.cuda.device(X.device):
+        _check(lib().spinfer_spmm_tp_gather(ctypes.byref(cs), X.data_ptr(), yp, M_full, K, N, world, rank, fp,
+                                            ws.data_ptr(), ws.numel(), _stream(stream)), "spinfer_spmm_tp_gather")
+
+
+def gather_wait(flag, state, world: int, ws: torch.Tensor | None = None, timeout_us: int = 0, stream=None):
+    """Stream-ordered wait until every rank signalled this rank's counter (spinfer_gather_wait)."""
+    dev = flag.device if isinstance(flag, torch.Tensor) else torch.device("cuda", torch.cuda.current_device())
+    with torch.cuda.device(dev):
+        _check(lib().spinfer_gather_wait(_ptr(flag), _ptr(state), world, ws.data_ptr() if ws is not None else None,
+                                         int(timeout_us), _stream(stream)), "spinfer_gather_wait")

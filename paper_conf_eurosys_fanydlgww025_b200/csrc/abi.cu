@@ -1,5 +1,6 @@
 // abi.cu — the extern "C" boundary declared in include/spinfer.h: argument
 // validation, status codes, and dispatch to the sm_100a kernels.
+#include <atomic>
 #include <cstring>
 #include "internal.cuh"
 
@@ -8,13 +9,20 @@ namespace spinfer {
 int check_device() {
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return SPINFER_ENODEV; }
+    static std::atomic<int> verdict[64];   // per device: 0 unknown, 1 sm_100, 2 other (host cost per call)
+    if (dev >= 0 && dev < 64) {
+        const int v = verdict[dev].load(std::memory_order_relaxed);
+        if (v) return v == 1 ? SPINFER_OK : SPINFER_ENODEV;
+    }
     int major = 0, minor = 0;
     if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev) != cudaSuccess ||
         cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev) != cudaSuccess) {
         cudaGetLastError();
         return SPINFER_ENODEV;
     }
-    return (major == 10 && minor == 0) ? SPINFER_OK : SPINFER_ENODEV;   // built for sm_100a only
+    const bool ok = major == 10 && minor == 0;   // built for sm_100a only
+    if (dev >= 0 && dev < 64) verdict[dev].store(ok ? 1 : 2, std::memory_order_relaxed);
+    return ok ? SPINFER_OK : SPINFER_ENODEV;
 }
 
 // any M, K > 0: shapes that are not multiples of 64 are zero-padded to whole GroupTiles (A8)
@@ -155,6 +163,38 @@ int spinfer_spmm_tp(const spinfer_tca *T_shard, const uint16_t *X, uint16_t *Y_f
     if (T_shard->M != c) return SPINFER_EINVAL;
     if (c == 0) return SPINFER_OK;   // rank owns no rows (more ranks than GT rows)
     return spinfer_spmm(T_shard, X, Y_full + (size_t)b * N, c, K, N, workspace, ws_bytes, stream);
+}
+
+int spinfer_spmm_tp_gather(const spinfer_tca *T_shard, const uint16_t *X, uint16_t *const *Y_full_peers, int M_full,
+                           int K, int N, int world, int rank, uint32_t *const *flag_peers, void *workspace,
+                           size_t ws_bytes, void *stream) {
+    int b = 0, c = 0;
+    int rc = spinfer_tp_rows(M_full, world, rank, &b, &c);
+    if (rc) return rc;
+    if (!T_shard || !X || !Y_full_peers || !flag_peers || world > kMaxPeers || N < 1 || ((N + 7) & ~7) > 16)
+        return SPINFER_EINVAL;
+    for (int r = 0; r < world; ++r)
+        if (!Y_full_peers[r] || !flag_peers[r] || !aligned16(Y_full_peers[r])) return SPINFER_EINVAL;
+    if ((rc = check_device())) return rc;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    if (c > 0) {
+        if (T_shard->M != c || !aligned16(X) || (workspace && !aligned16(workspace))) return SPINFER_EINVAL;
+        if ((rc = validate_tca(T_shard, c, K))) return rc;
+        uint16_t *ypeer[kMaxPeers];
+        for (int r = 0; r < world; ++r) ypeer[r] = Y_full_peers[r] + (size_t)b * N;
+        if ((rc = launch_spmm_dw(T_shard, X, ypeer[rank], c, K, N, nullptr, SPINFER_ACT_NONE, workspace, ws_bytes, st,
+                                 ypeer, world)))
+            return rc;
+    }
+    return launch_gather_signal(flag_peers, world, st);
+}
+
+int spinfer_gather_wait(uint32_t *flag, uint32_t *state, int world, void *workspace, uint32_t timeout_us, void *stream) {
+    if (!flag || !state || world < 1 || world > kMaxPeers) return SPINFER_EINVAL;
+    int rc = check_device();
+    if (rc) return rc;
+    int32_t *err = workspace ? reinterpret_cast<int32_t *>(workspace) + kErrWord : nullptr;
+    return launch_gather_wait(flag, state, world, err, timeout_us, reinterpret_cast<cudaStream_t>(stream));
 }
 
 int spinfer_spmm_check(void *workspace, int32_t *flags, void *stream) {

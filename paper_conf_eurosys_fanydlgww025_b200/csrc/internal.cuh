@@ -9,7 +9,8 @@ namespace spinfer {
 
 constexpr int kGT = 64;    // GroupTile edge (reading A1)
 constexpr int kNumSMsDefault = 148;
-constexpr int kMaxN = 65536;             // widest X (TMA coordinates and the wide kernel's tiling)
+constexpr int kMaxN = 65536;
+constexpr int kMaxPeers = 8;             // fused all-gather: ranks of one NVLink domain             // widest X (TMA coordinates and the wide kernel's tiling)
 
 int check_device();        // SPINFER_OK or SPINFER_ENODEV / SPINFER_ECUDA
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
@@ -31,6 +32,7 @@ constexpr int kErrWord = 16383;
 int option(int key);                     // spinfer_set_option values (0 = default)
 int set_option(int key, int value);
 int sm_count();                          // SMs of the current device (cached per device)
+int smem_optin();                        // opt-in shared memory per block of the current device (cached)
 int choose_grid(long long units);        // persistent grid size: min(SMs, units)
 int make_x_tmap(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows, bool swizzle);
 int make_x_tmap_box(CUtensorMap *m, const uint16_t *X, int K, int N, int box_n, int box_k, CUtensorMapSwizzle sw);
@@ -52,6 +54,9 @@ int launch_spmm_tc(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, 
 // spmm_dw.cu (decoupled-warp kernel, N <= 16)
 size_t spmm_dw_workspace_bytes(int M, int K, int N);
 int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias,
-                   int act, void *ws, size_t ws_bytes, cudaStream_t st);
+                   int act, void *ws, size_t ws_bytes, cudaStream_t st, uint16_t *const *ypeer = nullptr, int npeer = 0);
+// gather.cu (fused all-gather epilogue: peer signalling)
+int launch_gather_signal(uint32_t *const *flag_peers, int world, cudaStream_t st);
+int launch_gather_wait(uint32_t *flag, uint32_t *state, int world, int32_t *err, uint32_t timeout_us, cudaStream_t st);
 
 }  // namespace spinfer

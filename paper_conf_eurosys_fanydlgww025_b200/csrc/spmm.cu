@@ -63,6 +63,15 @@ int choose_grid(long long units) {
 // X [K][N] fp16 row-major as a 2-D tensor map, box {box_n, box_k}; box columns past N and rows
 // past K are zero-filled by the TMA (X padded to the MMA's N without a copy).
 int make_x_tmap_box(CUtensorMap *m, const uint16_t *X, int K, int N, int box_n, int box_k, CUtensorMapSwizzle sw) {
+    // the last few encodings per host thread (decode loops call with the same X buffers)
+    struct Entry { const uint16_t *X; int K, N, box_n, box_k, sw; CUtensorMap map; };
+    static thread_local Entry cache[8];
+    static thread_local int next = 0;
+    for (const Entry &e : cache)
+        if (e.X == X && X && e.K == K && e.N == N && e.box_n == box_n && e.box_k == box_k && e.sw == (int)sw) {
+            *m = e.map;
+            return SPINFER_OK;
+        }
     static EncodeTiledFn fn = nullptr;
     if (!fn) {
         void *f = nullptr;
@@ -81,7 +90,28 @@ int make_x_tmap_box(CUtensorMap *m, const uint16_t *X, int K, int N, int box_n, 
     CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, const_cast<uint16_t *>(X), dims, strides, box, estr,
                     CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    return r == CUDA_SUCCESS ? SPINFER_OK : SPINFER_EINVAL;
+    if (r != CUDA_SUCCESS) return SPINFER_EINVAL;
+    cache[next] = Entry{X, K, N, box_n, box_k, (int)sw, *m};
+    next = (next + 1) % 8;
+    return SPINFER_OK;
+}
+
+// Opt-in shared memory per block of the current device (cached).
+int smem_optin() {
+    static std::atomic<int> cached[64];
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev >= 0 && dev < 64) {
+        const int v = cached[dev].load(std::memory_order_relaxed);
+        if (v) return v;
+    }
+    int v = 232448;
+    if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess) {
+        cudaGetLastError();
+        v = 232448;
+    }
+    if (dev >= 0 && dev < 64) cached[dev].store(v, std::memory_order_relaxed);
+    return v;
 }
 
 // The narrow kernels' X slab: box {NX, box_rows}; 32B / 64B swizzle = the ldmatrix / MMA-descriptor

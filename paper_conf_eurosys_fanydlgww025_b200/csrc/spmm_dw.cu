@@ -90,6 +90,8 @@ struct DParams {
     int cslots;                   // CTA partial slots per GT row (max CTAs one rowblock overlaps)
     uint32_t slot_bytes, st_bm, st_v0, st_v1, vcap;   // slot: X slab | bitmaps | values row 0 | row 1
     float avg_gt;                 // n_values / NGT (start-up page prefetch hint)
+    int npeer;                    // fused all-gather (spinfer_spmm_tp_gather): Y rows also stored into
+    uint16_t *ypeer[kMaxPeers];   //   every peer's Y (ypeer[0..npeer), peer-mapped); 0: Y only
     long long *prof;              // experiments only (SPINFER_INSTRUMENT)
 };
 
@@ -209,10 +211,10 @@ __device__ __forceinline__ float epi_act(float v, float b, int act) {
 }
 
 // Y rows [row_base, row_base + 64) from accumulators in the m16n8k16 D layout. EPI: fused
-// bias/activation, padding rows of a ragged M (A8), N not a multiple of 8.
+// bias/activation, padding rows of a ragged M (A8), N not a multiple of 8. The fused all-gather
+// stores the same rows into every peer's Y as well.
 template <int NT, bool EPI>
 __device__ __forceinline__ void store_frag(const DParams &prm, int row_base, float (&acc)[4][NT][4], int lane) {
-    uint16_t *const Y = prm.Y;
     const int N = prm.N;
 #pragma unroll
     for (int tr = 0; tr < 4; ++tr) {
@@ -229,6 +231,8 @@ __device__ __forceinline__ void store_frag(const DParams &prm, int row_base, flo
                 acc[tr][nt][3] = epi_act(acc[tr][nt][3], b1, prm.act);
             }
         }
+        for (int dst = 0; dst < max(1, prm.npeer); ++dst) {
+        uint16_t *const Y = prm.npeer ? prm.ypeer[dst] : prm.Y;
 #pragma unroll
         for (int nt = 0; nt < NT; ++nt) {
             const int col = nt * 8 + 2 * (lane & 3);
@@ -251,6 +255,7 @@ __device__ __forceinline__ void store_frag(const DParams &prm, int row_base, flo
                 }
             }
         }
+        }
     }
 }
 
@@ -263,7 +268,8 @@ __device__ __forceinline__ void store_cols(const DParams &prm, int row, int col0
     const float b = (EPI && prm.bias) ? __half2float(__ushort_as_half(prm.bias[row])) : 0.f;
 #pragma unroll
     for (int c = 0; c < NC; ++c) w[c] = EPI ? epi_act(v[c], b, prm.act) : v[c];
-    __half *y = reinterpret_cast<__half *>(prm.Y + (size_t)row * N);
+    for (int dst = 0; dst < max(1, prm.npeer); ++dst) {
+    __half *y = reinterpret_cast<__half *>((prm.npeer ? prm.ypeer[dst] : prm.Y) + (size_t)row * N);
     if (!EPI || N == NT * 8) {
         if constexpr (NC == 4) {
             const __half2 a = __floats2half2_rn(w[0], w[1]), c2 = __floats2half2_rn(w[2], w[3]);
@@ -278,6 +284,7 @@ __device__ __forceinline__ void store_cols(const DParams &prm, int row, int col0
 #pragma unroll
         for (int c = 0; c < NC; ++c)
             if (col0 + c < N) y[col0 + c] = __float2half_rn(w[c]);
+    }
     }
 }
 
@@ -964,10 +971,7 @@ bool make_dplan(int M, int K, int Np, int max_gt_values, DPlan *pl) {
     const long long U = (long long)((MG + kRd - 1) / kRd) * KG;
     const int P = choose_grid(U);
     if ((unsigned long long)U * (unsigned long long)P >= (1ull << 32)) return false;
-    int dev = 0, smem_max = 232448;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    cudaGetLastError();
+    const int smem_max = smem_optin();
     int maxv = max_gt_values > 0 ? max_gt_values : 4096;
     maxv = std::min(4096, (maxv + 7) & ~7);
     int gmax = kMaxGd, smax = kMaxSd;
@@ -1041,7 +1045,7 @@ DwLayout dw_layout(int M, int K, int N) {
 size_t spmm_dw_workspace_bytes(int M, int K, int N) { return dw_layout(M, K, N).total; }
 
 int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias,
-                   int act, void *ws, size_t ws_bytes, cudaStream_t st) {
+                   int act, void *ws, size_t ws_bytes, cudaStream_t st, uint16_t *const *ypeer, int npeer) {
     const int Np = (N + 7) & ~7;
     if (Np > 16) return SPINFER_EINVAL;
     DPlan pl;
@@ -1072,6 +1076,9 @@ int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, 
     q.n_values = (int)T->n_values;
     q.avg_gt = (float)((double)T->n_values / ((double)q.MG * (double)q.KG));
     q.prof = nullptr;
+    if (npeer < 0 || npeer > kMaxPeers || (npeer && !ypeer)) return SPINFER_EINVAL;
+    q.npeer = npeer;
+    for (int d = 0; d < kMaxPeers; ++d) q.ypeer[d] = d < npeer ? ypeer[d] : nullptr;
     const bool epi = bias != nullptr || act != SPINFER_ACT_NONE || (M % kGT) != 0 || (N % 8) != 0;
     auto go = [&]() {
         if (Np == 8) return epi ? launch_dw<1, true>(pl, st) : launch_dw<1, false>(pl, st);

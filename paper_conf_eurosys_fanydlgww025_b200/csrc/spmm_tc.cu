@@ -695,10 +695,7 @@ bool make_plan(int M, int K, int NB, int max_gt_values, Plan *pl) {
     pl->P = choose_grid(U);
     if ((unsigned long long)U * (unsigned long long)pl->P >= (1ull << 32)) return false;   // 32-bit unit math
     const long long upc = (U + pl->P - 1) / pl->P;
-    int dev = 0, smem_max = 232448;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    cudaGetLastError();
+    const int smem_max = smem_optin();
     int maxv = max_gt_values > 0 ? max_gt_values : 4096;
     maxv = std::min(4096, (maxv + 7) & ~7);
     int gmax = kMaxG, smax = kMaxStages;

@@ -440,10 +440,7 @@ bool make_wplan(int M, int K, int N, int max_gt_values, WPlan *pl) {
     q.w_v1 = q.vcap;
     q.w_stage = al_w(1024u + 2u * q.vcap, 128);
     q.x_bytes = (uint32_t)(q.nsub * q.bps) * kWBox;
-    int dev = 0, smem_max = 232448;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    cudaGetLastError();
+    const int smem_max = smem_optin();
     const uint32_t fixed = 1024u /* barriers, header */ + kWDecWarps * kWTblBytes + 1024u /* base alignment */;
     // ring depths: 2 X stages, then A slots and W stages in pairs (even depths: each slot is always
     // refilled for the same decode phase), then more X stages

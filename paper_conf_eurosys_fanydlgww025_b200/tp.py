@@ -122,6 +122,26 @@ def run_stack(layers: Sequence[Layer], X: torch.Tensor, world: int, rank: int, g
     return cur
 
 
+def run_stack_fused(layers: Sequence[Layer], X: torch.Tensor, world: int, rank: int, outputs: Sequence[torch.Tensor],
+                    y_peers: Sequence[Sequence[int]], flag_peers: Sequence[int], flag, state, ws=None,
+                    timeout_us: int = 0) -> torch.Tensor:
+    """Config 5 with the fused all-gather epilogue (spinfer_spmm_tp_gather): each
+    layer's kernel stores this rank's rows into every rank's output buffer (y_peers[li][r]: rank r's
+    outputs[li] as mapped here, e.g. torch symmetric memory), then one stream-ordered wait on this
+    rank's counter. No NCCL call; N <= 16, no bias / activation."""
+    import paper_conf_eurosys_fanydlgww025_b200 as sp
+    cur = X
+    for li, L in enumerate(layers):
+        if L.x_rows is not None:
+            cur = cur[:L.x_rows]
+        if cur.shape[0] != L.K:
+            raise ValueError(f"layer {L.name}: X has {cur.shape[0]} rows, W has K={L.K}")
+        sp.spmm_tp_gather(L.shard, cur, y_peers[li], L.M, world, rank, flag_peers, ws=ws if ws is not None else L.ws)
+        sp.gather_wait(flag, state, world, ws=ws if ws is not None else L.ws, timeout_us=timeout_us)
+        cur = outputs[li]
+    return cur
+
+
 # OPT linear-layer shapes (SURVEY §8(d)(i), external: OPT configs; the paper names the models, P:309)
 OPT = {
     "opt-13b": (5120, 20480),
