@@ -9,9 +9,15 @@ want = ["Duration", "DRAM Throughput", "Memory Throughput", "SM Frequency", "Exe
         "Registers Per Thread", "Dynamic Shared Memory Per Block", "Warp Cycles Per Issued Instruction",
         "Executed Instructions", "Max Bandwidth", "Mem Busy", "Mem Pipes Busy", "L2 Cache Throughput",
         "L1/TEX Cache Throughput", "Compute (SM) Throughput"]
-for row in csv.reader(io.StringIO(det)):
-    if len(row) > 3 and row[-3] in want:
-        print(f"{row[-3]:40s} {row[-1]:>14s} {row[-2]}")
+rows_d = list(csv.reader(io.StringIO(det)))
+if rows_d:
+    hd = rows_d[0]
+    iname, iunit, ival = hd.index("Metric Name"), hd.index("Metric Unit"), hd.index("Metric Value")
+    seen = set()
+    for row in rows_d[1:]:
+        if len(row) > ival and row[iname] in want and row[iname] not in seen:
+            seen.add(row[iname])
+            print(f"{row[iname]:40s} {row[ival]:>14s} {row[iunit]}")
 raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(raw)))
 if len(rows) >= 3:
