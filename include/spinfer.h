@@ -118,7 +118,8 @@ SPINFER_API size_t spinfer_spmm_workspace_bytes(int M, int K, int N);
  *   N > 32   (prefill): tcgen05 with W decoded into shared memory, 128-row x
  *            (up to) 512-column output tiles, no split-K.
  * N not a multiple of 8 costs the same as the next multiple of 8 plus a zero-padded copy of
- * X in the workspace. */
+ * X in the workspace. For N <= 32, K <= 4,194,240 (at most 65535 GroupTile columns: the stage
+ * headers pack the column index in 16 bits) and ceil(M/64) < 16383; SPINFER_EINVAL otherwise. */
 SPINFER_API int spinfer_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N,
                  void *workspace, size_t ws_bytes, void *stream);
 

@@ -105,6 +105,7 @@ constexpr int kProfW = 20;
 constexpr size_t kTraceOff = 1024 * kProfW * 8;   // stage trace of CTA 0 after the counters
 [[maybe_unused]] constexpr size_t kEvOff = kTraceOff + 256 * 4;      // per-warp event trace of CTA 0: [16 warps][64 stages][6]
 [[maybe_unused]] constexpr size_t kGtOff = kEvOff + 16 * 64 * 6;    // per CTA [1024][4]: globaltimer at entry, max exit
+[[maybe_unused]] constexpr size_t kSmidOff = kGtOff + 1024 * 4;     // per CTA: the SM it ran on
 struct Prof {
 #if SPINFER_INSTRUMENT
     long long c[8] = {0, 0, 0, 0, 0, 0, 0, 0};
@@ -385,6 +386,13 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     Prof pf;
     pf.start();
     if (threadIdx.x == 0) pf.gt(prm.prof, p, 0);
+#if SPINFER_INSTRUMENT
+    if (threadIdx.x == 0 && prm.prof && p < 1024) {
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        prm.prof[kSmidOff + p] = smid;
+    }
+#endif
     // role warps: producers / reducer / idle. Each branch below ends in a return.
     if (warp >= kCWd) {
     if (warp == kCWd + 3) return;   // the idle warp (completes the warpgroup)
@@ -1087,7 +1095,7 @@ int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, 
 #if SPINFER_INSTRUMENT
     if (const char *path = getenv("SPINFER_PROF")) {   // experiments: dump per-warp cycle counters
         static long long *prof_buf = nullptr;
-        const size_t n = kGtOff + 1024 * 4;
+        const size_t n = kSmidOff + 1024;
         if (!prof_buf && cudaMalloc(&prof_buf, n * 8) != cudaSuccess) return SPINFER_ECUDA;
         cudaMemsetAsync(prof_buf, 0, n * 8, st);
         q.prof = prof_buf;

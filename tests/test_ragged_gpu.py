@@ -69,3 +69,25 @@ def test_ragged_tp_rows(world):
     torch.cuda.synchronize()
     assert tot == M
     assert_within(f16_bits(Y), oracle.spmm_f64(oracle.encode(W), X), north_star_bound(W, X), f"tp {world}")
+
+
+@pytest.mark.parametrize("kernel,N", [("dw", 16), ("tc", 32), ("default", 100)])
+@pytest.mark.parametrize("act", [None, "relu"])
+def test_ragged_bias_act(kernel, N, act):
+    """Fused bias / ReLU with a ragged M (rows past M are padding: they read no bias and are not
+    stored), for the three kernels (N = 100: the wide kernel)."""
+    import torch
+    import paper_conf_eurosys_fanydlgww025_b200 as sp
+    use_kernel(kernel, N)
+    M, K = 100, 70
+    W = synth.weight(M, K, 0.5, seed=77)
+    X = synth.activation(K, N, seed=78)
+    b = synth.activation(M, 1, seed=79).reshape(M)
+    T = sp.encode(to_dev(W))
+    bias = to_dev(b).view(torch.float16)
+    Y = f16_bits(sp.spmm(T, to_dev(X), bias=bias, act=act))
+    torch.cuda.synchronize()
+    Yref = oracle.spmm_f64(oracle.encode(W), X) + b.view(np.float16).astype(np.float64)[:, None]
+    if act == "relu":
+        Yref = np.maximum(Yref, 0.0)
+    assert_within(Y, Yref, north_star_bound(W, X) + 1e-3, f"ragged bias {kernel} N={N} act={act}")
