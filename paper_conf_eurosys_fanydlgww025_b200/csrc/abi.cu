@@ -226,6 +226,6 @@ const char *spinfer_status_str(int status) {
     }
 }
 
-const char *spinfer_version(void) { return "spinfer-b200 0.2 (sm_100a; TCA-BME GT=64; SMBD: mma.sync N<=16, tcgen05 N>16)"; }
+const char *spinfer_version(void) { return "spinfer-b200 0.2 (sm_100a; TCA-BME GT=64; SMBD: mma.sync N<=16, tcgen05 N 17-32, tcgen05 wide N>32)"; }
 
 }  // extern "C"

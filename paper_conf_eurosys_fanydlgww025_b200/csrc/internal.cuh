@@ -34,6 +34,7 @@ int set_option(int key, int value);
 int sm_count();                          // SMs of the current device (cached per device)
 int smem_optin();                        // opt-in shared memory per block of the current device (cached)
 int choose_grid(long long units);        // persistent grid size: min(SMs, units)
+int choose_grid_rb(long long RB, long long KG);   // stream-K grid aligned to rowblocks when that pays
 int make_x_tmap(CUtensorMap *m, const uint16_t *X, int K, int N, int NX, int box_rows, bool swizzle);
 int make_x_tmap_box(CUtensorMap *m, const uint16_t *X, int K, int N, int box_n, int box_k, CUtensorMapSwizzle sw);
 int launch_pad_x(const uint16_t *X, uint16_t *Xp, int K, int N, int Np, cudaStream_t st);

@@ -1,31 +1,31 @@
 // spmm_dw.cu — decoupled-warp TCA-BME SpMM Y = W x X for N <= 16 (sm_100a; §4.3,
 // P:214-301). The library's kernel for N <= 16 (the decode regime of the paper's Fig. 1 shape).
 //
-// Why this design: in the round-1 kernel all consumer warps walked the ring in
-// lockstep behind two scan warps and met at named barriers at every segment epilogue; the decode
-// ran only 69 % of the time. Here the warps are independent:
-//   * producer warp: per stage (up to G GroupTile columns x 2 GT rows) one warp instruction issues
-//     the bulk copies of both rows' bitmaps and packed values from different lanes (a thread's
-//     successive bulk copies serialise at ~310 ns each, tools/tma_sweep2.sh) plus the X slab's
-//     tensor copy, into an S-slot ring; a small per-slot header carries the per-GT value offsets
-//     (GTileOffset). The slot's empty barrier counts only the warps that own a GT of the
-//     stage (the producer pre-arrives for the rest).
-//   * 16 consumer warps: warp (r, m) owns GT row r of each rowblock and every unit u (a GT column
-//     of the CTA's stream-K range) with u % 8 == m. Every warp walks the stage sequence itself and
-//     waits only for the stages that hold its GTs. Per GroupTile it computes the PopCount base of
-//     every BitmapTile with a 32-lane shuffle scan into its own 1 KB table, then decodes
-//     the 16 TCTiles (MaskedPopCount, Alg. 2) into mma.m16n8k16 A fragments (X via
-//     ldmatrix.trans, fp32 accumulators in registers, Listing 1).
+// Design: one persistent CTA per SM walks its stream-K range of units (one GT
+// column of a 128-row rowblock) in stages of G GroupTile columns x 2 GT rows, through an S-slot
+// shared-memory ring; every warp role walks the stage sequence on its own (no lockstep):
+//   * 2 producer warps (stages of one parity each): one warp instruction per stage issues the
+//     bulk copies of both rows' bitmaps and packed values and the X slab's tensor copy from
+//     different lanes (a thread's successive bulk copies serialise at ~310 ns each); a per-slot
+//     header carries the stage shape, its segment index and the per-GT value offsets (GTileOffset,
+//     P:196). A slot is refilled after a hardware named barrier with exactly the stage's GT owners.
+//   * 16 consumer warps: warp (r, m) owns GT m % G of GT row r in the stages i = m / G (mod 8 / G).
+//     Per GroupTile it computes the PopCount base of every BitmapTile with a 32-lane
+//     shuffle scan into its own 1 KB table, then decodes the 16 TCTiles (MaskedPopCount, Alg. 2
+//     P:282-287) into mma.m16n8k16 A fragments (X via ldmatrix.trans, fp32 accumulators in
+//     registers, Listing 1).
 //   * segment ends (the end of the CTA's part of a rowblock, the paper's ReductionWorkspace P:231,
 //     P:263): a consumer parks its fp32 partial in the workspace and signals the reducer warp,
 //     which sums the row's partials in warp order and writes Y (complete rowblock) or the CTA's
-//     partial; the last CTA of a split rowblock sums the CTA partials in CTA order. The CTA's
-//     final segment is reduced by the 16 consumers together through shared memory. Every sum
-//     runs in a fixed order: results do not depend on timing.
+//     partial; the last CTA of a split rowblock sums the CTA partials in CTA order (8 warps per GT
+//     row, in the consumers' end phase). The CTA's final segment is reduced by the 16 consumers
+//     together through shared memory. Every sum runs in a fixed order: results do not depend on
+//     timing.
 // Corrupt or stale TCA-BME input (offsets not monotone / not 16-byte aligned / past n_values, a
 // GT with more values than a stage slot holds, bitmaps with more set bits than the GT's values)
 // never reads or writes outside the caller's buffers: the stage or GT is skipped and the
-// workspace's error word is set (include/spinfer.h).
+// workspace's error word is set (include/spinfer.h). The fused all-gather variant stores every
+// Y row into each peer's Y as well (spinfer_spmm_tp_gather).
 #include <cuda.h>
 #include <algorithm>
 #include <cstdio>
@@ -977,7 +977,7 @@ bool make_dplan(int M, int K, int Np, int max_gt_values, DPlan *pl) {
     const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;
     if (KG > 65535 || MG >= kErrWord) return false;
     const long long U = (long long)((MG + kRd - 1) / kRd) * KG;
-    const int P = choose_grid(U);
+    const int P = choose_grid_rb((MG + kRd - 1) / kRd, KG);
     if ((unsigned long long)U * (unsigned long long)P >= (1ull << 32)) return false;
     const int smem_max = smem_optin();
     int maxv = max_gt_values > 0 ? max_gt_values : 4096;
@@ -1036,7 +1036,7 @@ struct DwLayout {
 DwLayout dw_layout(int M, int K, int N) {
     const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;
     const long long U = (long long)((MG + kRd - 1) / kRd) * KG;
-    const int P = choose_grid(U);
+    const int P = choose_grid_rb((MG + kRd - 1) / kRd, KG);
     const int Np = (N + 7) & ~7;
     DwLayout l;
     l.seg = (size_t)P * kNSeg * kRd * 8 * 64 * Np * 4;

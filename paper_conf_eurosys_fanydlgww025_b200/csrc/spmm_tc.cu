@@ -692,7 +692,7 @@ bool make_plan(int M, int K, int NB, int max_gt_values, Plan *pl) {
     const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;   // zero-padded to whole GTs (A8)
     if (KG > 65535) return false;                                      // StageDesc packs gc in 16 bits
     const long long U = (long long)((MG + kR - 1) / kR) * KG;
-    pl->P = choose_grid(U);
+    pl->P = choose_grid_rb((MG + kR - 1) / kR, KG);
     if ((unsigned long long)U * (unsigned long long)pl->P >= (1ull << 32)) return false;   // 32-bit unit math
     const long long upc = (U + pl->P - 1) / pl->P;
     const int smem_max = smem_optin();
@@ -751,7 +751,7 @@ size_t spmm_tc_workspace_bytes(int M, int K, int N) {
     const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;
     const long long U = (long long)((MG + kR - 1) / kR) * KG;
     if (4LL * ((MG + kR - 1) / kR) >= kErrWord) return 0;   // one counter per rowblock and TMEM lane quarter
-    const int P = choose_grid(U);
+    const int P = choose_grid_rb((MG + kR - 1) / kR, KG);
     const int Np = (N + 7) & ~7;
     const size_t part = (size_t)P * 2 * 128 * Np * 4;
     const size_t xpad = (N % 8) ? ((size_t)K * Np * 2 + 255) / 256 * 256 : 0;
