@@ -25,6 +25,10 @@ if len(rows) >= 3:
     for k in ["dram__bytes_read.sum", "dram__bytes_write.sum", "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum",
               "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum", "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
               "smsp__inst_executed.sum", "sm__pipe_tensor_op_hmma_cycles_active.avg.pct_of_peak_sustained_active",
+              "sm__pipe_tensor_subpipe_hmma_cycles_active.avg.pct_of_peak_sustained_active",
+              "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active",
+              "sm__pipe_shared_cycles_active.avg.pct_of_peak_sustained_active",
+              "gpu__time_duration.sum", "sm__cycles_elapsed.avg", "sm__cycles_active.avg",
               "lts__t_bytes.sum", "smsp__cycles_active.avg"]:
         if k in hdr:
             v = vals[hdr.index(k)]
