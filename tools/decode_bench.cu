@@ -10,6 +10,12 @@
 #include <cuda_runtime.h>
 #include <cuda_fp16.h>
 #include "../paper_conf_eurosys_fanydlgww025_b200/csrc/ptx.cuh"
+namespace spinfer {
+__device__ __forceinline__ void mma_16816(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) { mma_16816_nv(d, a, b0, b1); }
+__device__ __forceinline__ void ldsm_x4_trans(uint32_t a, uint32_t &d0, uint32_t &d1, uint32_t &d2, uint32_t &d3) { ldsm_x4_trans_nv(a, d0, d1, d2, d3); }
+__device__ __forceinline__ void ldsm_x2_trans(uint32_t a, uint32_t &d0, uint32_t &d1) { ldsm_x2_trans_nv(a, d0, d1); }
+__device__ __forceinline__ void mbar_wait_(uint32_t b, uint32_t p) { mbar_wait(b, p); }
+}
 using namespace spinfer;
 
 constexpr uint32_t kSelA = 0x7f62u, kSelB = 0x4cbfu, kSelC = 0x2333u;
@@ -208,6 +214,9 @@ __global__ void __launch_bounds__(TB, 1) k_dec(int iters, float *out, long long 
             const uint32_t y = z >> 30;
             sl[k] = y * (y * selB + selA) + selC;
             if (VAR == 3) { u0[k] = a; u1[k] = z; }
+            else if (VAR == 100) { const uint32_t ad = (a & 2u) * 32801u + a; u0[k] = lds_u32(ad); u1[k] = 0u; }
+            else if (VAR == 101) { u0[k] = lds_u32(a & ~3u); u1[k] = 0u; }
+            else if (VAR == 102) { const uint32_t ad = (a & 2u) * 32801u + a; u0[k] = lds_u32(ad); u1[k] = z; }
             else { u0[k] = lds_u16(a); u1[k] = lds_u16(a + 2u); }
         }
     };
@@ -217,7 +226,7 @@ __global__ void __launch_bounds__(TB, 1) k_dec(int iters, float *out, long long 
         for (int tt = 0; tt < 2; ++tt) {
             uint32_t afr[4];
 #pragma unroll
-            for (int b = 0; b < 4; ++b) afr[b] = prmt(u0[tt * 4 + b], u1[tt * 4 + b], sl[tt * 4 + b]);
+            for (int b = 0; b < 4; ++b) afr[b] = (VAR == 100 || VAR == 101 || VAR == 102) ? prmt(u0[tt * 4 + b], 0u, sl[tt * 4 + b]) : prmt(u0[tt * 4 + b], u1[tt * 4 + b], sl[tt * 4 + b]);
             if (VAR == 4) { acc[trb + tt][0][0] += __uint_as_float(afr[0] ^ afr[1] ^ afr[2] ^ afr[3]); continue; }
 #pragma unroll
             for (int nt = 0; nt < 2; ++nt) mma_16816(acc[trb + tt][nt], afr, bfr[nt][0], bfr[nt][1]);
@@ -351,7 +360,7 @@ __global__ void __launch_bounds__(TB, 1) k_dec(int iters, float *out, long long 
             }
         } else {
             uint32_t t0_[8], t1_[8], s1_[8];
-#pragma unroll 1
+#pragma unroll
             for (int tc = 0; tc < 4; ++tc) {
                 uint32_t bfr[2][2];
                 ldsm_x4_trans(xs + tc * 512, bfr[0][0], bfr[0][1], bfr[1][0], bfr[1][1]);
@@ -376,7 +385,7 @@ template <int VAR, int TB = 640>
 void run(int warps, int iters, int tma = 0) {
     float *out; long long *cyc; cudaMalloc(&out, 4); cudaMalloc(&cyc, 8 * 148);
     static uint8_t *src = nullptr; if (!src) { cudaMalloc(&src, 64ull << 20); cudaMemset(src, 1, 64ull << 20); }
-    const int smem = tma ? 65536 + 4 * 32768 + 64 : 64 * 1024;
+    const int smem = tma ? 65536 + 4 * 32768 + 64 : 128 * 1024;
     cudaFuncSetAttribute(k_dec<VAR, TB>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     const int nt = (warps + (tma ? 1 : 0)) * 32;
     int zero = 0;
@@ -400,6 +409,6 @@ void run(int warps, int iters, int tma = 0) {
 }
 
 int main() {
-    for (int w : {16}) { run<0>(w, 200); run<5>(w, 200); }
+    for (int w : {16, 12, 8}) { run<0>(w, 200); run<100>(w, 200); run<101>(w, 200); run<3>(w, 200); run<4>(w, 200); }
     return 0;
 }
