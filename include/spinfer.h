@@ -196,7 +196,8 @@ SPINFER_API int spinfer_spmm_check(void *workspace, int32_t *flags /* host */, v
 /* Process-wide options (tests, ablation, tuning). 0 is every option's default. Not
  * synchronized with calls running on other host threads: set them before launching work.
  *   SPINFER_OPT_KERNEL    0 auto (N <= 16: the mma.sync decoupled-warp kernel, else tcgen05),
- *                         1 force the decoupled-warp kernel (N <= 16 only), 2 force tcgen05;
+ *                         1 force the decoupled-warp kernel (N <= 32; N 17-32 run its half-GroupTile
+ *                         mode: X padded to 32 columns, two warps per GroupTile), 2 force tcgen05;
  *   SPINFER_OPT_MAX_CTAS  cap on the persistent grid (0: one CTA per SM);
  *   SPINFER_OPT_STAGE_G   cap on GroupTile columns per pipeline stage (0: the kernel's max);
  *   SPINFER_OPT_STAGE_S   cap on pipeline stages (0: as many as shared memory holds);

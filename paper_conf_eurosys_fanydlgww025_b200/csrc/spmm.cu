@@ -148,7 +148,7 @@ size_t spmm_workspace_bytes(int M, int K, int N) {
     if (M <= 0 || K <= 0 || N <= 0 || N > kMaxN || (M + kGT - 1) / kGT >= kErrWord) return 0;
     if (N > 32) return spmm_wide_workspace_bytes(M, K, N);
     const size_t tc = spmm_tc_workspace_bytes(M, K, N);
-    const size_t dw = N <= 16 ? spmm_dw_workspace_bytes(M, K, N) : 0;
+    const size_t dw = N <= 32 ? spmm_dw_workspace_bytes(M, K, N) : 0;
     return std::max(tc, dw);
 }
 
@@ -161,7 +161,7 @@ int launch_spmm(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int
     if (Np > 32) return launch_spmm_wide(T, X, Y, M, K, N, bias, act, ws, ws_bytes, st);
     const int ko = option(SPINFER_OPT_KERNEL);
     const bool dw = ko == SPINFER_KERNEL_DW ? true : ko == SPINFER_KERNEL_TC ? false : Np <= 16;
-    if (dw && Np > 16) return SPINFER_EINVAL;
+    if (dw && Np > 32) return SPINFER_EINVAL;
     if (dw) return launch_spmm_dw(T, X, Y, M, K, N, bias, act, ws, ws_bytes, st);
     return launch_spmm_tc(T, X, Y, M, K, N, bias, act, ws, ws_bytes, st);
 }

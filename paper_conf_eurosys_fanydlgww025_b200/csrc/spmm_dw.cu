@@ -214,11 +214,11 @@ __device__ __forceinline__ float epi_act(float v, float b, int act) {
 // Y rows [row_base, row_base + 64) from accumulators in the m16n8k16 D layout. EPI: fused
 // bias/activation, padding rows of a ragged M (A8), N not a multiple of 8. The fused all-gather
 // stores the same rows into every peer's Y as well.
-template <int NT, bool EPI>
-__device__ __forceinline__ void store_frag(const DParams &prm, int row_base, float (&acc)[4][NT][4], int lane) {
+template <int NT, bool EPI, int TR = 4>
+__device__ __forceinline__ void store_frag(const DParams &prm, int row_base, float (&acc)[TR][NT][4], int lane) {
     const int N = prm.N;
 #pragma unroll
-    for (int tr = 0; tr < 4; ++tr) {
+    for (int tr = 0; tr < TR; ++tr) {
         const int r0 = row_base + tr * 16 + (lane >> 2);
         if (EPI && (prm.bias || prm.act)) {
             // rows past M (padding of a ragged M) read no bias
@@ -355,6 +355,13 @@ template <int NT, bool EPI>
 __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant__ DParams prm) {
     constexpr int Np = NT * 8;
     constexpr int kF4 = 64 * Np / 4;   // float4 per 64 x Np partial
+    // half mode (N 17-32, NT = 4): a consumer warp owns TCTile rows 2h, 2h + 1 of its GroupTile (32
+    // output rows, 32 fp32 accumulators at N = 32); the two halves of a GT are two warps
+    constexpr bool HALF = NT > 2;
+    constexpr int TRW = HALF ? 2 : 4;   // TCTile rows per consumer warp
+    constexpr int kSlotW = HALF ? 4 : 8;   // GT slots per GT row and phase set (warps per half-row)
+    constexpr int JC = (kF4 + 255) / 256;   // float4 columns of a 64 x Np block per lane (8 warps)
+    constexpr uint32_t kOwnW = HALF ? 2u : 1u;   // consumer warps per GT
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *const smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     const uint32_t sbase = smem_u32(smem);
@@ -445,7 +452,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             if (lane == 0) pf.st(prm.prof, p, i, 3, true);
             // the slot's previous stage (i - S) released by its GT owners: hardware named barrier
             // (the waiting warp is not woken by the CTA's mbarrier traffic, no polling)
-            if (i >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + ((owners_pk >> (4 * slot)) & 15u)));
+            if (i >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + kOwnW * ((owners_pk >> (4 * slot)) & 15u)));
             pf.lap(0);
             if (lane == 0) pf.st(prm.prof, p, i, 0, true);
             const uint32_t st = ring + slot * prm.slot_bytes, fb = bar_full + 8 * slot;
@@ -511,14 +518,14 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             skip2(ia, nsa, ia_i);
             pf.lap(5);
         }
-        // stop sentinels: one per consumer phase, in the slots of the stage indices [nst, nst + 8 / G)
-        // (S >= 8 / G: distinct slots); this producer writes those of its parity. The header
-        // carries the CTA's segment count.
+        // stop sentinels: one per consumer phase, in the slots of the stage indices [nst, nst + phases)
+        // (phases = 8 / G, 4 / G in half mode; S >= phases: distinct slots); this producer writes
+        // those of its parity. The header carries the CTA's segment count.
         {
             const int nst = i;                      // the loop ends with i = the stage count
-            for (int j = nst + ((nst & 1) != q ? 1 : 0); j < nst + 8 / G; j += 2) {
+            for (int j = nst + ((nst & 1) != q ? 1 : 0); j < nst + (HALF ? 4 : 8) / G; j += 2) {
                 const uint32_t slot = (uint32_t)(j % S);
-                if (j >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + ((owners_pk >> (4 * slot)) & 15u)));
+                if (j >= S) named_bar_sync(kBarIdSlot0 + slot, 32u * (1u + kOwnW * ((owners_pk >> (4 * slot)) & 15u)));
                 owners_pk &= ~(15u << (4 * slot));
                 if (lane == 0) sts_v4(sbase + kOffHdr + slot * kHdrBytes, make_uint4(0u, kHdrStop, (uint32_t)nseg, 0u));
                 mbar_arrive(bar_full + 8 * slot);
@@ -556,59 +563,108 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                 __syncwarp();   // every lane has read the mask before it is reset
                 if (lane == 0) sts_u32(seg_mask + 8 * k + 4 * r, 0u);
                 const float4 *src = reinterpret_cast<const float4 *>(prm.ws_seg) + ((((size_t)p * kNSeg + k) * kRd + r) * 8) * kF4;
-                float acc[4][NT][4];
+                const int grow = kRd * rb + r;
+                if constexpr (HALF) {
+                    // rows 32 hh .. 32 hh + 31 are the sum over jm = 0..3 (warp order) of warps 2 jm + hh
+#pragma unroll 1
+                    for (int hh = 0; hh < 2; ++hh) {
+                        float acc[2][NT][4];
 #pragma unroll
-                for (int a = 0; a < 4; ++a)
-#pragma unroll
-                    for (int b = 0; b < NT; ++b)
-#pragma unroll
-                        for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
-                // warp order; a warp without a GT of the segment contributes +0 (sums start at +0:
-                // adding +0 changes no bit). Four warps' loads in flight together.
-#pragma unroll
-                for (int tr = 0; tr < 4; ++tr)
-#pragma unroll
-                    for (int mh = 0; mh < 8; mh += 4) {
-                        float4 v[4][NT];
-#pragma unroll
-                        for (int u = 0; u < 4; ++u)
-#pragma unroll
-                            for (int nt = 0; nt < NT; ++nt)
-                                v[u][nt] = ((cmask >> (mh + u)) & 1u) ? __ldcg(src + (size_t)(mh + u) * kF4 + (tr * NT + nt) * 32 + lane)
-                                                                      : make_float4(0.f, 0.f, 0.f, 0.f);
-#pragma unroll
-                        for (int u = 0; u < 4; ++u)
+                        for (int tr = 0; tr < 2; ++tr)
 #pragma unroll
                             for (int nt = 0; nt < NT; ++nt) {
-                                const float4 w = v[u][nt];
-                                acc[tr][nt][0] += w.x; acc[tr][nt][1] += w.y; acc[tr][nt][2] += w.z; acc[tr][nt][3] += w.w;
+                                float4 v[4];
+#pragma unroll
+                                for (int u = 0; u < 4; ++u) {
+                                    const int mw = 2 * u + hh;
+                                    v[u] = ((cmask >> mw) & 1u) ? __ldcg(src + (size_t)mw * kF4 + (tr * NT + nt) * 32 + lane)
+                                                                : make_float4(0.f, 0.f, 0.f, 0.f);
+                                }
+                                float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+                                for (int u = 0; u < 4; ++u) { t.x += v[u].x; t.y += v[u].y; t.z += v[u].z; t.w += v[u].w; }
+                                acc[tr][nt][0] = t.x; acc[tr][nt][1] = t.y; acc[tr][nt][2] = t.z; acc[tr][nt][3] = t.w;
                             }
+                        if (complete) {
+                            store_frag<NT, EPI, 2>(prm, grow * 64 + 32 * hh, acc, lane);
+                        } else {
+                            const int pfirst = uowner(rb * KG, prm.U, prm.P);
+                            float *const cdst = prm.ws_cta + ((size_t)grow * prm.cslots + (p - pfirst)) * (64 * Np);
+#pragma unroll
+                            for (int tr = 0; tr < 2; ++tr)
+#pragma unroll
+                                for (int nt = 0; nt < NT; ++nt) {
+                                    const int row = 32 * hh + tr * 16 + (lane >> 2), col = nt * 8 + 2 * (lane & 3);
+                                    stg_f2(cdst + row * Np + col, acc[tr][nt][0], acc[tr][nt][1]);
+                                    stg_f2(cdst + (row + 8) * Np + col, acc[tr][nt][2], acc[tr][nt][3]);
+                                }
+                        }
                     }
-                for (int m = 0; m < 8; ++m)
-                    if (((cmask >> m) & 1u) && lane < kF4 / 8) discard_l2(src + (size_t)m * kF4 + 8 * lane);
-                const int grow = kRd * rb + r;
-                if (complete) {
-                    store_frag<NT, EPI>(prm, grow * 64, acc, lane);
+                    for (int mw = 0; mw < 8; ++mw)   // each warp's partial: 2 x NT x 32 float4 = 32 lines
+                        if ((cmask >> mw) & 1u) discard_l2(src + (size_t)mw * kF4 + 8 * lane);
+                    if (!complete) {
+                        __syncwarp();
+                        int nparts;
+                        if (cta_arrive(prm, rb, grow, lane, nparts) && lane == 0) {
+                            const uint32_t nd = lds_u32(sbase + kDefer);
+                            sts_u32(sbase + kDefer + 4 + 4 * nd, (uint32_t)grow | ((uint32_t)nparts << 16));
+                            sts_u32(sbase + kDefer, nd + 1);
+                        }
+                    }
                 } else {
-                    const int pfirst = uowner(rb * KG, prm.U, prm.P);
-                    float *dst = prm.ws_cta + ((size_t)grow * prm.cslots + (p - pfirst)) * (64 * Np);
+                    float acc[4][NT][4];
+#pragma unroll
+                    for (int a = 0; a < 4; ++a)
+#pragma unroll
+                        for (int b = 0; b < NT; ++b)
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
+                    // warp order; a warp without a GT of the segment contributes +0 (sums start at +0:
+                    // adding +0 changes no bit). Four warps' loads in flight together.
 #pragma unroll
                     for (int tr = 0; tr < 4; ++tr)
 #pragma unroll
-                        for (int nt = 0; nt < NT; ++nt) {
-                            const int row = tr * 16 + (lane >> 2), col = nt * 8 + 2 * (lane & 3);
-                            stg_f2(dst + row * Np + col, acc[tr][nt][0], acc[tr][nt][1]);
-                            stg_f2(dst + (row + 8) * Np + col, acc[tr][nt][2], acc[tr][nt][3]);
+                        for (int mh = 0; mh < 8; mh += 4) {
+                            float4 v[4][NT];
+#pragma unroll
+                            for (int u = 0; u < 4; ++u)
+#pragma unroll
+                                for (int nt = 0; nt < NT; ++nt)
+                                    v[u][nt] = ((cmask >> (mh + u)) & 1u) ? __ldcg(src + (size_t)(mh + u) * kF4 + (tr * NT + nt) * 32 + lane)
+                                                                          : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+                            for (int u = 0; u < 4; ++u)
+#pragma unroll
+                                for (int nt = 0; nt < NT; ++nt) {
+                                    const float4 w = v[u][nt];
+                                    acc[tr][nt][0] += w.x; acc[tr][nt][1] += w.y; acc[tr][nt][2] += w.z; acc[tr][nt][3] += w.w;
+                                }
                         }
-                    __syncwarp();
-                    // the last CTA of the rowblock: the sum is deferred to the consumer warps' end
-                    // phase (8 warps per GT row, all loads in flight; a single warp here would be
-                    // latency-bound over up to ~20 partials)
-                    int nparts;
-                    if (cta_arrive(prm, rb, grow, lane, nparts) && lane == 0) {
-                        const uint32_t nd = lds_u32(sbase + kDefer);
-                        sts_u32(sbase + kDefer + 4 + 4 * nd, (uint32_t)grow | ((uint32_t)nparts << 16));
-                        sts_u32(sbase + kDefer, nd + 1);
+                    for (int m = 0; m < 8; ++m)
+                        if (((cmask >> m) & 1u) && lane < kF4 / 8) discard_l2(src + (size_t)m * kF4 + 8 * lane);
+                    if (complete) {
+                        store_frag<NT, EPI>(prm, grow * 64, acc, lane);
+                    } else {
+                        const int pfirst = uowner(rb * KG, prm.U, prm.P);
+                        float *dst = prm.ws_cta + ((size_t)grow * prm.cslots + (p - pfirst)) * (64 * Np);
+#pragma unroll
+                        for (int tr = 0; tr < 4; ++tr)
+#pragma unroll
+                            for (int nt = 0; nt < NT; ++nt) {
+                                const int row = tr * 16 + (lane >> 2), col = nt * 8 + 2 * (lane & 3);
+                                stg_f2(dst + row * Np + col, acc[tr][nt][0], acc[tr][nt][1]);
+                                stg_f2(dst + (row + 8) * Np + col, acc[tr][nt][2], acc[tr][nt][3]);
+                            }
+                        __syncwarp();
+                        // the last CTA of the rowblock: the sum is deferred to the consumer warps' end
+                        // phase (8 warps per GT row, all loads in flight; a single warp here would be
+                        // latency-bound over up to ~20 partials)
+                        int nparts;
+                        if (cta_arrive(prm, rb, grow, lane, nparts) && lane == 0) {
+                            const uint32_t nd = lds_u32(sbase + kDefer);
+                            sts_u32(sbase + kDefer + 4 + 4 * nd, (uint32_t)grow | ((uint32_t)nparts << 16));
+                            sts_u32(sbase + kDefer, nd + 1);
+                        }
                     }
                 }
             }
@@ -630,18 +686,24 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     // ---------------------------------------------------------------------- consumers
     // Warp (r, m) owns GT j = m % G of GT row r in every stage i with i % (8 / G) == m / G
     // (G in {1, 2, 4}: all 8 warps of a row busy); it reads the stage's shape and segment index
-    // from the slot header.
-    const int r = warp >> 3, m = warp & 7, jw = m % G;
-    const int tstride = 8 / G;   // stages between two of this warp's
+    // from the slot header. Half mode: warp (r, m) owns TCTile rows 2 hw, 2 hw + 1 (hw = m & 1) of
+    // GT j = jm % G, jm = m >> 1, in the stages i % (4 / G) == jm / G.
+    const int r = warp >> 3, m = warp & 7;
+    const int hw = HALF ? (m & 1) : 0, jm = HALF ? (m >> 1) : m;
+    const int jw = jm % G;
+    const int tstride = (HALF ? 4 : 8) / G;   // stages between two of this warp's
     const uint32_t mulc = opaque_u32(1u << (30u - 2u * (uint32_t)(lane & 15)));   // z = w << (30 - sh) on the FMA pipe
     constexpr uint32_t selA = kSelA, selB = kSelB, selC = kSelC;   // IMAD immediates
     constexpr uint32_t cpr = Np / 8;   // 16-byte chunks per X row
     const uint32_t rr = lane & 7, mk = (lane >> 3) & 1, mn = (lane >> 4) & 1;
     // X slab row-major; with the tensor copy the 32B swizzle XORs the 16-byte chunk with row bit 2
-    const uint32_t x_lane = (mk * 8u + rr) * cpr * 16u + ((mn ^ (NT == 2 ? (rr >> 2) & 1u : 0u)) * 16u);
-    float acc[4][NT][4];
+    // (Np = 16), the 64B swizzle with row bits 1-2 (Np = 32: a second ldmatrix for columns 16-31)
+    const uint32_t x_lane = (mk * 8u + rr) * cpr * 16u +
+                            ((HALF ? (mn ^ ((rr >> 1) & 3u)) : (mn ^ (NT == 2 ? (rr >> 2) & 1u : 0u))) * 16u);
+    [[maybe_unused]] const uint32_t x_lane2 = (mk * 8u + rr) * cpr * 16u + (((2u + mn) ^ ((rr >> 1) & 3u)) * 16u);
+    float acc[TRW][NT][4];
 #pragma unroll
-    for (int a = 0; a < 4; ++a)
+    for (int a = 0; a < TRW; ++a)
 #pragma unroll
         for (int b = 0; b < NT; ++b)
 #pragma unroll
@@ -688,7 +750,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         if (own) {
             float4 *dst = reinterpret_cast<float4 *>(prm.ws_seg) + ((((size_t)p * kNSeg + k) * kRd + r) * 8 + m) * kF4;
 #pragma unroll
-            for (int tr = 0; tr < 4; ++tr)
+            for (int tr = 0; tr < TRW; ++tr)
 #pragma unroll
                 for (int nt = 0; nt < NT; ++nt)
                     stg_f4(dst + (tr * NT + nt) * 32 + lane, make_float4(acc[tr][nt][0], acc[tr][nt][1], acc[tr][nt][2], acc[tr][nt][3]));
@@ -729,7 +791,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         return true;
     };
 
-    int i = m / G;                  // stage index
+    int i = jm / G;                 // stage index
     uint32_t slot = (uint32_t)(i % S), ph = 0;   // ring position of stage i (S >= 2)
     int cur = -1;                   // open segment of this warp (-1: none)
     bool contrib = false, seen = false;
@@ -758,7 +820,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
             for (int s2 = cur + 1; s2 < sg; ++s2) seg_close(s2, false);   // segments with no stage of this parity
             cur = sg;
 #pragma unroll
-            for (int a = 0; a < 4; ++a)
+            for (int a = 0; a < TRW; ++a)
 #pragma unroll
                 for (int b = 0; b < NT; ++b)
 #pragma unroll
@@ -800,8 +862,11 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                     const uint32_t xk = xs + (uint32_t)(16 * tc) * cpr * 16u;
                     if constexpr (NT == 1) {
                         ldsm_x2_trans_nv(xk, bfr[0][0], bfr[0][1]);
-                    } else {
+                    } else if constexpr (NT == 2) {
                         ldsm_x4_trans_nv(xk, bfr[0][0], bfr[0][1], bfr[1][0], bfr[1][1]);
+                    } else {   // Np = 32: columns 0-15 and 16-31
+                        ldsm_x4_trans_nv(xk, bfr[0][0], bfr[0][1], bfr[1][0], bfr[1][1]);
+                        ldsm_x4_trans_nv(xk + (x_lane2 - x_lane), bfr[2][0], bfr[2][1], bfr[3][0], bfr[3][1]);
                     }
 #if SPINFER_ABLATION
 #pragma unroll
@@ -834,15 +899,16 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                     }
 #else
 #pragma unroll
-                    for (int hh = 0; hh < 2; ++hh) {
-                        load_E_nv(tbl_lane_l + (uint32_t)(tc * 16 + hh * 8) * 8u);
+                    for (int hh = 0; hh < (HALF ? 1 : 2); ++hh) {   // TCTile row pairs (2 hh', 2 hh' + 1)
+                        const int hq = HALF ? hw : hh;
+                        load_E_nv(tbl_lane_l + (uint32_t)(tc * 16 + hq * 8) * 8u);
                         issue_to(t0, t1, s1);
-                        assemble_nv(t0, t1, s1, 2 * hh, bfr);
+                        assemble_nv(t0, t1, s1, HALF ? 0 : 2 * hh, bfr);
                     }
 #endif
                 }
 #pragma unroll
-                for (int a = 0; a < 4; ++a)
+                for (int a = 0; a < TRW; ++a)
 #pragma unroll
                     for (int b = 0; b < NT; ++b)
                         asm volatile("" : "+f"(acc[a][b][0]), "+f"(acc[a][b][1]), "+f"(acc[a][b][2]), "+f"(acc[a][b][3]) :: "memory");
@@ -854,7 +920,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
                 atomicOr(prm.ws_err, 2);   // corrupt GT (or poisoned stage): skipped, Y is not valid
             }
             __syncwarp();
-            named_bar_arrive(kBarIdSlot0 + slot, 32u * (1u + (uint32_t)(rows * g)));   // the slot's GT owners + its producer
+            named_bar_arrive(kBarIdSlot0 + slot, 32u * (1u + kOwnW * (uint32_t)(rows * g)));   // the slot's GT owner warps + its producer
             if (lane == 0) pf.st(prm.prof, p, i, 2, true);
             if (lane == 0) pf.ev(prm.prof, p, warp, i >> 1, 5);
         }
@@ -869,7 +935,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     for (int s2 = cur + 1; s2 < fseg; ++s2) seg_close(s2, false);
     if (cur != fseg) {   // this warp holds nothing of the final segment
 #pragma unroll
-        for (int a = 0; a < 4; ++a)
+        for (int a = 0; a < TRW; ++a)
 #pragma unroll
             for (int b = 0; b < NT; ++b)
 #pragma unroll
@@ -894,9 +960,10 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         fcomplete = max(ps, frb * KG) == frb * KG && pe == (frb + 1) * KG;
     }
     if (fseg >= 0 && r < frows) {
-        const uint32_t mine = ring + (uint32_t)(r * 8 + m) * (64u * Np * 4u);
+        // half mode: the two halves of GT slot jm share one 64 x Np buffer (rows 32 hw ..)
+        const uint32_t mine = ring + (uint32_t)(r * kSlotW + jm) * (64u * Np * 4u) + (uint32_t)(32 * hw * Np * 4);
 #pragma unroll
-        for (int tr = 0; tr < 4; ++tr)
+        for (int tr = 0; tr < TRW; ++tr)
 #pragma unroll
             for (int nt = 0; nt < NT; ++nt) {
                 const uint32_t row = tr * 16 + (lane >> 2), col = nt * 8 + 2 * (lane & 3);
@@ -907,15 +974,19 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     named_bar_sync(1, 32 * kCWd);
     if (fseg >= 0 && r < frows) {
         constexpr int NC = Np / 4;   // outputs per lane: 8 rows x Np columns per warp
+        constexpr int NC4 = NC > 4 ? 4 : NC;   // per store
         const int row = 8 * m + (lane >> 2), col0 = NC * (lane & 3);
         float v[NC];
 #pragma unroll
         for (int c = 0; c < NC; ++c) v[c] = 0.f;
-        for (int m2 = 0; m2 < 8; ++m2) {   // warp order; warps without a GT of the segment hold +0
-            const uint32_t a = ring + (uint32_t)(r * 8 + m2) * (64u * Np * 4u) + (uint32_t)(row * Np + col0) * 4u;
-            if constexpr (NC == 4) {
-                const float4 w = lds_f4(a);
-                v[0] += w.x; v[1] += w.y; v[2] += w.z; v[3] += w.w;
+        for (int m2 = 0; m2 < kSlotW; ++m2) {   // warp order; warps without a GT of the segment hold +0
+            const uint32_t a = ring + (uint32_t)(r * kSlotW + m2) * (64u * Np * 4u) + (uint32_t)(row * Np + col0) * 4u;
+            if constexpr (NC >= 4) {
+#pragma unroll
+                for (int q = 0; q < NC / 4; ++q) {
+                    const float4 w = lds_f4(a + 16u * q);
+                    v[4 * q] += w.x; v[4 * q + 1] += w.y; v[4 * q + 2] += w.z; v[4 * q + 3] += w.w;
+                }
             } else {
                 const uint2 w = lds_v2(a);
                 v[0] += __uint_as_float(w.x); v[1] += __uint_as_float(w.y);
@@ -923,12 +994,23 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         }
         const int grow = kRd * frb + r;
         if (fcomplete) {
-            store_cols<NT, EPI, NC>(prm, grow * 64 + row, col0, v);
+#pragma unroll
+            for (int q = 0; q < NC / NC4; ++q) {
+                float vq[NC4];
+#pragma unroll
+                for (int c = 0; c < NC4; ++c) vq[c] = v[NC4 * q + c];
+                store_cols<NT, EPI, NC4>(prm, grow * 64 + row, col0 + NC4 * q, vq);
+            }
         } else {
             const int pfirst = uowner(frb * KG, prm.U, prm.P);
             float *dst = prm.ws_cta + ((size_t)grow * prm.cslots + (p - pfirst)) * (64 * Np) + row * Np + col0;
-            if constexpr (NC == 4) stg_f4(reinterpret_cast<float4 *>(dst), make_float4(v[0], v[1], v[2], v[3]));
-            else stg_f2(dst, v[0], v[1]);
+            if constexpr (NC >= 4) {
+#pragma unroll
+                for (int q = 0; q < NC / 4; ++q)
+                    stg_f4(reinterpret_cast<float4 *>(dst) + q, make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]));
+            } else {
+                stg_f2(dst, v[0], v[1]);
+            }
         }
     }
     if (fseg >= 0 && !fcomplete) {
@@ -941,7 +1023,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
         named_bar_sync(1, 32 * kCWd);
         // the last CTA of the rowblock: the row's warps sum 32 float4 columns each (all in flight)
         nparts = (int)lds_u32(sbase + kFinFlag + 4 * r);
-        if (nparts && r < frows && m * 32 < kF4) cta_sum<NT, EPI, 1>(prm, kRd * frb + r, nparts, m * 32, lane);
+        if (nparts && r < frows && m * 32 * JC < kF4) cta_sum<NT, EPI, JC>(prm, kRd * frb + r, nparts, m * 32 * JC, lane);
     }
     // cross-CTA sums of non-final segments whose last contributor was this CTA (the reducer's list):
     // GT row e is summed by the 8 warps of consumer row e % 2
@@ -949,7 +1031,7 @@ __global__ void __launch_bounds__(kThreadsD, 1) k_spmm_dw(const __grid_constant_
     const int ndef = (int)lds_u32(sbase + kDefer);
     for (int e = r; e < ndef; e += kRd) {
         const uint32_t d = lds_u32(sbase + kDefer + 4 + 4 * e);
-        if (m * 32 < kF4) cta_sum<NT, EPI, 1>(prm, (int)(d & 0xFFFFu), (int)(d >> 16), m * 32, lane);
+        if (m * 32 * JC < kF4) cta_sum<NT, EPI, JC>(prm, (int)(d & 0xFFFFu), (int)(d >> 16), m * 32 * JC, lane);
     }
     pf.lap(3);
     if (lane == 0) pf.gt(prm.prof, p, 1);
@@ -985,9 +1067,10 @@ bool make_dplan(int M, int K, int Np, int max_gt_values, DPlan *pl) {
     int gmax = kMaxGd, smax = kMaxSd;
     if (option(SPINFER_OPT_STAGE_G) > 0) gmax = std::max(1, std::min(kMaxGd, option(SPINFER_OPT_STAGE_G)));
     if (option(SPINFER_OPT_STAGE_S) > 0) smax = std::max(2, std::min(kMaxSd, option(SPINFER_OPT_STAGE_S)));
-    const uint32_t final_scratch = 2u * 8u * 64u * Np * 4u;   // the final segment's partials reuse the ring
-    // G in {4, 2, 1} (8 / G consumer phases keep all 8 warps of a GT row busy); the largest G
-    // with >= 4 slots, else the deepest valid ring. A ring needs >= 8 / G slots (one stop
+    const int wslots = Np > 16 ? 4 : 8;   // GT slots per GT row (half mode, Np = 32: two warps per GT)
+    const uint32_t final_scratch = 2u * wslots * 64u * Np * 4u;   // the final segment's partials reuse the ring
+    // G in {4, 2, 1} (wslots / G consumer phases keep all 8 warps of a GT row busy); the largest
+    // G with >= 4 slots, else the deepest valid ring. A ring needs >= wslots / G slots (one stop
     // sentinel per phase) and an even slot count (producer q always refills its own stages'
     // slots: the slot release barrier counts the GT owners of the stage it issued there).
     int bestG = 0, bestS = 0;
@@ -996,7 +1079,7 @@ bool make_dplan(int M, int K, int Np, int max_gt_values, DPlan *pl) {
         const uint32_t vcap = al((uint32_t)G * maxv * 2, 128);
         const uint32_t slot = al(st_bm + kRd * G * 512 + 2 * vcap, 1024);
         const int S = (int)std::min<long long>(smax, ((long long)smem_max - kOffRing - 1024) / slot) & ~1;
-        if ((uint32_t)S * slot < final_scratch || S < std::max(2, 8 / G)) continue;
+        if ((uint32_t)S * slot < final_scratch || S < std::max(2, wslots / G)) continue;
         if (S >= 4) { bestG = G; bestS = S; break; }
         if (S > bestS) { bestG = G; bestS = S; }
     }
@@ -1030,6 +1113,9 @@ int launch_dw(const DPlan &pl, cudaStream_t st) {
     return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
 }
 
+// Padded X width of the decoupled-warp kernel: 8, 16, or 32 (half mode, N 17-32)
+inline int dw_np(int N) { return N > 16 ? 32 : (N + 7) & ~7; }
+
 struct DwLayout {
     size_t seg, cta, xpad, total;
 };
@@ -1037,11 +1123,11 @@ DwLayout dw_layout(int M, int K, int N) {
     const int MG = (M + kGT - 1) / kGT, KG = (K + kGT - 1) / kGT;
     const long long U = (long long)((MG + kRd - 1) / kRd) * KG;
     const int P = choose_grid_rb((MG + kRd - 1) / kRd, KG);
-    const int Np = (N + 7) & ~7;
+    const int Np = dw_np(N);
     DwLayout l;
     l.seg = (size_t)P * kNSeg * kRd * 8 * 64 * Np * 4;
     l.cta = (size_t)MG * cta_slots(U, P, KG) * 64 * Np * 4;
-    l.xpad = (N % 8) ? ((size_t)K * Np * 2 + 255) / 256 * 256 : 0;
+    l.xpad = (N != Np) ? ((size_t)K * Np * 2 + 255) / 256 * 256 : 0;
     l.total = kCounterRegion + l.seg + l.cta + l.xpad;
     return l;
 }
@@ -1054,8 +1140,8 @@ size_t spmm_dw_workspace_bytes(int M, int K, int N) { return dw_layout(M, K, N).
 
 int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, int K, int N, const uint16_t *bias,
                    int act, void *ws, size_t ws_bytes, cudaStream_t st, uint16_t *const *ypeer, int npeer) {
-    const int Np = (N + 7) & ~7;
-    if (Np > 16) return SPINFER_EINVAL;
+    if (N < 1 || N > 32) return SPINFER_EINVAL;
+    const int Np = dw_np(N);
     DPlan pl;
     if (!make_dplan(M, K, Np, T->max_gt_values, &pl)) return SPINFER_EINVAL;
     const DwLayout lay = dw_layout(M, K, N);
@@ -1063,7 +1149,7 @@ int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, 
     DParams &q = pl.prm;
     uint8_t *w8 = reinterpret_cast<uint8_t *>(ws);
     const uint16_t *Xk = X;
-    if (N % 8) {
+    if (N != Np) {
         uint16_t *Xp = reinterpret_cast<uint16_t *>(w8 + kCounterRegion + lay.seg + lay.cta);
         if (int rc = launch_pad_x(X, Xp, K, N, Np, st)) return rc;
         Xk = Xp;
@@ -1087,9 +1173,10 @@ int launch_spmm_dw(const spinfer_tca *T, const uint16_t *X, uint16_t *Y, int M, 
     if (npeer < 0 || npeer > kMaxPeers || (npeer && !ypeer)) return SPINFER_EINVAL;
     q.npeer = npeer;
     for (int d = 0; d < kMaxPeers; ++d) q.ypeer[d] = d < npeer ? ypeer[d] : nullptr;
-    const bool epi = bias != nullptr || act != SPINFER_ACT_NONE || (M % kGT) != 0 || (N % 8) != 0;
+    const bool epi = bias != nullptr || act != SPINFER_ACT_NONE || (M % kGT) != 0 || N != Np;
     auto go = [&]() {
         if (Np == 8) return epi ? launch_dw<1, true>(pl, st) : launch_dw<1, false>(pl, st);
+        if (Np == 32) return epi ? launch_dw<4, true>(pl, st) : launch_dw<4, false>(pl, st);
         return epi ? launch_dw<2, true>(pl, st) : launch_dw<2, false>(pl, st);
     };
 #if SPINFER_INSTRUMENT

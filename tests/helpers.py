@@ -38,13 +38,14 @@ def assert_within(Y_gpu_bits: np.ndarray, Y_ref: np.ndarray, bound: np.ndarray, 
 def use_kernel(kernel: str, N: int, monkeypatch=None):
     """Select the SpMM kernel for this test (spinfer_set_option SPINFER_OPT_KERNEL; the conftest
     fixture resets every option after the test): "default" = the library's choice, "dw" = the
-    decoupled-warp mma.sync kernel (N <= 16), "tc" = the tcgen05 kernel."""
+    decoupled-warp mma.sync kernel (N <= 32; half-GroupTile mode above 16), "tc" = the tcgen05
+    kernel."""
     import pytest
     import paper_conf_eurosys_fanydlgww025_b200 as sp
     if kernel == "default":
         return
-    if kernel == "dw" and N > 16:
-        pytest.skip("the decoupled-warp kernel serves N <= 16")
+    if kernel == "dw" and N > 32:
+        pytest.skip("the decoupled-warp kernel serves N <= 32")
     sp.set_option("kernel", kernel)
 
 

@@ -56,8 +56,8 @@ def test_built_for_sm100a(sp):
     ks = _kernel_sass(sp)
     dw = [v for k, v in ks.items() if "k_spmm_dw" in k]
     tc = [v for k, v in ks.items() if "k_spmm_tc" in k]
-    assert len(dw) == 4 and len(tc) == 2, sorted(ks)
-    for v in dw:   # N <= 16: mma.sync tensor cores fed by TMA, named-barrier slot release
+    assert len(dw) == 6 and len(tc) == 2, sorted(ks)   # dw: N = 8, 16, 32 (half mode) x {plain, epilogue}
+    for v in dw:   # N <= 32: mma.sync tensor cores fed by TMA, named-barrier slot release
         for mn in ("HMMA.16816.F32", "UBLKCP", "UTMALDG.2D", "LDSM.16.MT88", "SYNCS", "BAR.ARV"):
             assert mn in v, mn
     for v in tc:   # N > 16: tcgen05 MMA (UTCHMMA), TMEM stores / loads (STTM / LDTM), TMA

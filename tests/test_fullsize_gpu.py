@@ -58,7 +58,8 @@ def _run(W, X, N, kernel, ctas):
 
 @pytest.mark.parametrize("kernel,N,ctas", [
     ("default", 16, 0), ("default", 32, 0), ("dw", 8, 0), ("tc", 16, 0), ("default", 24, 0),
-    ("dw", 16, 8), ("tc", 32, 8), ("dw", 16, 147), ("tc", 32, 147), ("dw", 13, 0), ("tc", 27, 0)])
+    ("dw", 16, 8), ("tc", 32, 8), ("dw", 16, 147), ("tc", 32, 147), ("dw", 13, 0), ("tc", 27, 0),
+    ("dw", 32, 0), ("dw", 24, 147), ("dw", 32, 8)])
 def test_config2_bit_exact(config2, kernel, N, ctas):
     W, X, exp = config2
     Y = _run(W, X, N, kernel, ctas)
@@ -66,7 +67,7 @@ def test_config2_bit_exact(config2, kernel, N, ctas):
     assert bad == 0, f"{kernel} N={N} ctas={ctas}: {bad} of {Y.size} outputs differ"
 
 
-@pytest.mark.parametrize("kernel,N", [("dw", 16), ("tc", 16), ("tc", 32)])
+@pytest.mark.parametrize("kernel,N", [("dw", 16), ("tc", 16), ("tc", 32), ("dw", 32)])
 def test_opt66_fc2_bit_exact(opt66_fc2, kernel, N):
     W, X, exp = opt66_fc2
     Y = _run(W, X, N, kernel, 0)
