@@ -417,6 +417,22 @@ def stack(a, B, sp, synth, tp):
     t_all = statistics.median(B.timed(fn, steps))
     out["stack_us"] = B.allmax(t_all * 1e3)
     out["gather_overhead_us"] = out["stack_us"] - out["spmm_only_us"] if world > 1 else 0.0
+    # the same stack with programmatic dependent launch (SPINFER_OPT_PDL): each SpMM's CTAs start as
+    # the previous kernel's retire and stream their first weights while it finishes
+    sp.set_option("pdl", 1)
+    try:
+        t_spmm_pdl = statistics.median(B.timed(lambda: eager(False), steps))
+        out["spmm_only_us_pdl"] = B.allmax(t_spmm_pdl * 1e3)
+        if graph is not None:
+            graph_pdl = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(graph_pdl):
+                eager()
+            torch.cuda.synchronize()
+            for _ in range(3):
+                graph_pdl.replay()
+            out["stack_us_pdl"] = B.allmax(statistics.median(B.timed(graph_pdl.replay, steps)) * 1e3)
+    finally:
+        sp.set_option("pdl", 0)
     out["fused_allgather"] = stack_fused(B, sp, tp, layers, X, N, ws, steps, outs_ref=outs)
     nb = sum(algorithmic_bytes(L.row_count, L.K, N, L.shard.n_values) for L in layers)
     out["spmm_frac_of_roofline"] = nb / (t_spmm * 1e-3) / 1e9 / load_peaks()[0]

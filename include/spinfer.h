@@ -201,14 +201,23 @@ SPINFER_API int spinfer_spmm_check(void *workspace, int32_t *flags /* host */, v
  *   SPINFER_OPT_MAX_CTAS  cap on the persistent grid (0: one CTA per SM);
  *   SPINFER_OPT_STAGE_G   cap on GroupTile columns per pipeline stage (0: the kernel's max);
  *   SPINFER_OPT_STAGE_S   cap on pipeline stages (0: as many as shared memory holds);
- *   SPINFER_OPT_WIDE_BN   N > 32 kernel: cap on the MMA N of a sub-tile (multiple of 16; 0: 256).
+ *   SPINFER_OPT_WIDE_BN   N > 32 kernel: cap on the MMA N of a sub-tile (multiple of 16; 0: 256);
+ *   SPINFER_OPT_PDL       1: launch the N <= 32 decoupled-warp kernel with programmatic dependent
+ *                         launch (cudaLaunchAttributeProgrammaticStreamSerialization): its CTAs start
+ *                         as the previous kernel's CTAs retire and stream the first stages' weights
+ *                         (GTileOffset, bitmaps, values) while that kernel finishes; X, the workspace
+ *                         and Y are touched only after griddepcontrol.wait, i.e. after the previous
+ *                         grid completed. For chains of SpMMs on one stream (a layer stack). The
+ *                         weights must not be written by the immediately preceding kernel unless that
+ *                         kernel is one of this library's encoders (they never trigger early).
  * SPINFER_EINVAL for an unknown key or an out-of-range value. */
 #define SPINFER_OPT_KERNEL 0
 #define SPINFER_OPT_MAX_CTAS 1
 #define SPINFER_OPT_STAGE_G 2
 #define SPINFER_OPT_STAGE_S 3
 #define SPINFER_OPT_WIDE_BN 4
-#define SPINFER_OPT_COUNT 5
+#define SPINFER_OPT_PDL 5
+#define SPINFER_OPT_COUNT 6
 #define SPINFER_KERNEL_AUTO 0
 #define SPINFER_KERNEL_DW 1
 #define SPINFER_KERNEL_TC 2

@@ -49,7 +49,7 @@ SYMBOLS = ["spinfer_encode_count", "spinfer_encode_fill", "spinfer_decode", "spi
            "spinfer_set_option", "spinfer_get_option", "spinfer_status_str", "spinfer_version"]
 
 # spinfer.h SPINFER_OPT_* / SPINFER_KERNEL_*
-OPTIONS = {"kernel": 0, "max_ctas": 1, "stage_g": 2, "stage_s": 3, "wide_bn": 4}
+OPTIONS = {"kernel": 0, "max_ctas": 1, "stage_g": 2, "stage_s": 3, "wide_bn": 4, "pdl": 5}
 KERNELS = {"auto": 0, "dw": 1, "tc": 2}
 
 
