@@ -202,7 +202,7 @@ SPINFER_API int spinfer_spmm_check(void *workspace, int32_t *flags /* host */, v
  *   SPINFER_OPT_STAGE_G   cap on GroupTile columns per pipeline stage (0: the kernel's max);
  *   SPINFER_OPT_STAGE_S   cap on pipeline stages (0: as many as shared memory holds);
  *   SPINFER_OPT_WIDE_BN   N > 32 kernel: cap on the MMA N of a sub-tile (multiple of 16; 0: 256);
- *   SPINFER_OPT_PDL       1: launch the N <= 32 decoupled-warp kernel with programmatic dependent
+ *   SPINFER_OPT_PDL       1: launch the N <= 32 kernels (decoupled-warp and tcgen05) with programmatic dependent
  *                         launch (cudaLaunchAttributeProgrammaticStreamSerialization): its CTAs start
  *                         as the previous kernel's CTAs retire and stream the first stages' weights
  *                         (GTileOffset, bitmaps, values) while that kernel finishes; X, the workspace

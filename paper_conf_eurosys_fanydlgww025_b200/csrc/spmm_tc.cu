@@ -264,6 +264,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
     tm_fence_before();
     __syncthreads();
     tm_fence_after();
+    if (threadIdx.x == 0) grid_dep_launch();   // SPINFER_OPT_PDL: the next kernel may be scheduled
     const uint32_t tmem = *reinterpret_cast<volatile uint32_t *>(smem + kTcTmemSlot);
     if (u0 >= u1) {   // no work (more CTAs than units)
         if (warp == 0) tm_dealloc(tmem, CfgTC::TmemCols);
@@ -308,6 +309,9 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
                 bulk_g2s(st + (lane ? prm.st_v1 : prm.st_v0), prm.vals + poff.x, vb, bar_full + 8 * slot, pol_w);
             // the X slab region is free once the MMA of stage i - S has completed
             if (i >= S) mbar_wait(bar_emptyx + 8 * slot, sg.par() ^ 1u);
+            // X may be the previous kernel's output (SPINFER_OPT_PDL): the first stage waits for that
+            // grid with its weight copies in flight; everything else follows from this stage's data
+            if (i == 0) grid_dep_wait();
             if (lane == 0) tma_2d_g2s(st, &prm.tmap_x, 0, 64 * sg.gc, bar_full + 8 * slot);   // box {NB, 64 G}
             pit.next(prm);
             if (pit.valid()) poff = load_off(pit);
@@ -738,6 +742,19 @@ int launch_tc(const Plan &pl, cudaStream_t st) {
         if (cudaFuncSetAttribute(k_spmm_tc<NB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem) != cudaSuccess)
             return SPINFER_ECUDA;
         configured_smem[dev] = (int)pl.smem;
+    }
+    if (option(SPINFER_OPT_PDL)) {   // programmatic dependent launch (layer stacks), see spmm_dw.cu
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3((unsigned)pl.P);
+        cfg.blockDim = dim3((unsigned)CfgTC::Threads);
+        cfg.dynamicSmemBytes = pl.smem;
+        cfg.stream = st;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        return cudaLaunchKernelEx(&cfg, k_spmm_tc<NB>, pl.prm) == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;
     }
     k_spmm_tc<NB><<<pl.P, CfgTC::Threads, pl.smem, st>>>(pl.prm);
     return cudaGetLastError() == cudaSuccess ? SPINFER_OK : SPINFER_ECUDA;

@@ -73,15 +73,16 @@ def test_run_stack_world1_real_kernels():
         cur = Y
 
 
+@pytest.mark.parametrize("N", [16, 32])
 @pytest.mark.parametrize("graph", [False, True])
-def test_stack_pdl_matches_serial(graph):
+def test_stack_pdl_matches_serial(graph, N):
     """SPINFER_OPT_PDL: the layer stack's SpMMs (one shared workspace, each layer's X the previous
     layer's Y) launched with programmatic dependent launch give the same bits as serial launches,
     eagerly and replayed from a CUDA graph; the first layer also matches the oracle."""
     import torch
     import paper_conf_eurosys_fanydlgww025_b200 as sp
     from paper_conf_eurosys_fanydlgww025_b200 import tp
-    h, f, N, s = 256, 1024, 16, 0.6
+    h, f, s = 256, 1024, 0.6
     shapes = [("qkv", 3 * h, h), ("o", h, h), ("fc1", f, h), ("fc2", h, f)] * 2
     ws = torch.zeros(max(sp.workspace_bytes(M, K, N) for _, M, K in shapes), dtype=torch.uint8, device="cuda")
     layers, Ws = [], []
