@@ -23,6 +23,9 @@ __global__ void k_gather_signal(uint32_t *f0, uint32_t *f1, uint32_t *f2, uint32
 }
 
 __global__ void k_gather_wait(const uint32_t *flag, uint32_t *state, int world, int32_t *err, uint32_t timeout_us) {
+    // a PDL-launched SpMM of the next layer (SPINFER_OPT_PDL) may start streaming its weights now; it
+    // reads X (this gather's output) only after griddepcontrol.wait, i.e. after this kernel completed
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     const uint32_t target = *state + (uint32_t)world;
     *state = target;
     uint64_t t0;
