@@ -490,6 +490,23 @@ def stack_fused(B, sp, tp, layers, X, N, ws, steps, outs_ref=None):
         except Exception as e:
             fn, res["cuda_graph"], res["graph_error"] = run, False, f"{type(e).__name__}: {e}"[:200]
         res["stack_us"] = B.allmax(statistics.median(B.timed(fn, steps)) * 1e3)
+        # with programmatic dependent launch: each SpMM starts streaming its weights while the
+        # previous layer's gather wait spins (the wait kernel triggers its dependents)
+        sp.set_option("pdl", 1)
+        try:
+            for _ in range(3):
+                run()
+            torch.cuda.synchronize()
+            fn_pdl = run
+            if res["cuda_graph"]:
+                g2 = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g2):
+                    run()
+                torch.cuda.synchronize()
+                fn_pdl = g2.replay
+            res["stack_us_pdl"] = B.allmax(statistics.median(B.timed(fn_pdl, steps)) * 1e3)
+        finally:
+            sp.set_option("pdl", 0)
         res["errors"] = sp.check(ws)
         ref = outs_ref[-1] if outs_ref is not None else None
         if ref is not None:   # same final output as the NCCL path (same kernels, same summation order)
