@@ -73,7 +73,7 @@ def test_run_stack_world1_real_kernels():
         cur = Y
 
 
-@pytest.mark.parametrize("N", [16, 32])
+@pytest.mark.parametrize("N", [13, 16, 32])
 @pytest.mark.parametrize("graph", [False, True])
 def test_stack_pdl_matches_serial(graph, N):
     """SPINFER_OPT_PDL: the layer stack's SpMMs (one shared workspace, each layer's X the previous
@@ -89,7 +89,9 @@ def test_stack_pdl_matches_serial(graph, N):
     for i, (name, M, K) in enumerate(shapes):
         W = synth.weight(M, K, s, seed=60 + i)
         Ws.append(W)
-        layers.append(tp.Layer(name, M, K, 0, M, shard=sp.encode(to_dev(W)), x_rows=h if name == "o" else None, ws=ws))
+        # FC1 with the fused ReLU epilogue (spinfer_spmm_ex); N = 13 adds the X padding kernel in between
+        layers.append(tp.Layer(name, M, K, 0, M, shard=sp.encode(to_dev(W)), x_rows=h if name == "o" else None, ws=ws,
+                               act="relu" if name == "fc1" else None))
     X = to_dev(synth.activation(h, N, seed=5)).view(torch.float16)
 
     def run(pdl):
