@@ -164,8 +164,9 @@ __device__ __forceinline__ float epi_act(float v, float b, int act) {
 struct CfgTC {
     static constexpr int CW = 16;
     static constexpr int ProducerWarp = 16;
-    static constexpr int ScanWarp = 17;      // 17, 18: SMBD tables of even / odd stages
-    static constexpr int Threads = 19 * 32;  // <= 5 warps per SM sub-partition: 96 registers each
+    static constexpr int ScanWarp = 17;      // 17, 18, 19: SMBD tables of the stages i % 3 == 0, 1, 2
+    static constexpr int NScan = 3;          // (the scan warps bound the kernel: their throughput, not latency)
+    static constexpr int Threads = 20 * 32;  // 5 warps per SM sub-partition: 96 registers each
     static constexpr uint32_t TmemCols = 512;
 };
 // TMEM columns: A buffers [k-team][ABufs] x 32 columns, then D [k-team][segment parity] x NB
@@ -328,7 +329,7 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         // memory straight into registers, prefetched two stages ahead (no TMA copy: a bulk copy
         // costs the SM's TMA unit >= ~310 ns however small, tools/tma_sweep.sh). A table waits
         // only for its slot to be free, so its latency (shuffle round trips through the loaded
-        // MIO queue) is hidden; two warps double the throughput.
+        // MIO queue) is hidden; three warps (stages i % 3) share the throughput the kernel is bound by.
         constexpr int Q = 2 * kMaxG;
         const int sw = warp - CfgTC::ScanWarp;
         struct Bm { uint2 a[Q], b[Q]; int o; };   // o: lane 8 rr + j holds gtile_offset of GT j of row rr
@@ -372,8 +373,10 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
         }
         StageIter it;
         it.init(u0, u1, prm);
-        if (sw == 1) it.next(prm);
-        auto skip2 = [&](StageIter &x) { x.next(prm); if (x.valid()) x.next(prm); };
+        for (int k = 0; k < sw && it.valid(); ++k) it.next(prm);
+        auto skip2 = [&](StageIter &x) {   // this warp's next stage: NScan stages on
+            for (int k = 0; k < CfgTC::NScan && x.valid(); ++k) x.next(prm);
+        };
         Bm F;   // one register set: the next stage's loads are issued right after a table is
                 // published and complete while the warp waits for that stage's slot
         if (it.valid()) fetch(it, F);
@@ -405,9 +408,6 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
             for (int qq = 0; qq < Q; ++qq) {
                 const int rr = qq / kMaxG, j = qq % kMaxG;
                 const uint32_t t = __shfl_sync(0xffffffffu, incl[qq], 31);
-                // every GT's value count (gtile_offset difference) must be its popcount padded to 8
-                const int ob = __shfl_sync(0xffffffffu, cur.o, 8 * rr + j), oe = __shfl_sync(0xffffffffu, cur.o, 8 * rr + j + 1);
-                if (rr < sg.rows && j < sg.g) bad |= oe - ob != (int)(((t & 0xFFFFu) + (t >> 16) + 7u) & ~7u);
                 if (rr < sg.rows && j < sg.g) {
                     const uint32_t vsm = st + (rr ? prm.st_v1 : prm.st_v0);
                     const uint32_t excl = incl[qq] - packed[qq];
@@ -424,15 +424,12 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
                 // a multiple of 8 values (the GTileOffset rule, encode.cu)
                 rel[rr] += (int)(((t & 0xFFFFu) + (t >> 16) + 7u) & ~7u);
             }
-            // the bitmaps must account for exactly the row's staged values (the GTileOffset rule) and
-            // the row's range must be one the producer copied: otherwise (corrupt input) the stage
-            // decodes as zeros, reading only inside its slot
+            // memory safety first: the tables address the row's values by popcount (rel), so a row
+            // whose bitmaps claim more values than a slot holds (corrupt input) decodes as zeros,
+            // reading only inside its slot
 #pragma unroll
             for (int rr = 0; rr < kR; ++rr)
-                if (rr < sg.rows) {
-                    const int ob = __shfl_sync(0xffffffffu, cur.o, 8 * rr), oe = __shfl_sync(0xffffffffu, cur.o, 8 * rr + sg.g);
-                    bad |= ob < 0 || oe > prm.n_values || 2u * (uint32_t)(oe - ob) > prm.vcap;
-                }
+                if (rr < sg.rows) bad |= 2u * (uint32_t)rel[rr] > prm.vcap;
             if (bad) {
 #pragma unroll
                 for (int qq = 0; qq < Q; ++qq) {
@@ -453,6 +450,18 @@ __global__ void __launch_bounds__(CfgTC::Threads, 1) k_spmm_tc(const __grid_cons
             // warps wait on one barrier per stage
             mbar_wait_sleep(bar_full + 8 * slot, sg.par());
             mbar_arrive(bar_scan + 8 * slot);
+            // a GT row's GTileOffset range must equal its padded popcounts (the encoding rule): a
+            // mismatch (corrupt input) is reported after the tables are published, off the decode's
+            // critical path (the range checks of the copies are the producer's). Lane 8 rr + g holds
+            // the row's end offset and receives its start from lane 8 rr: one shuffle per stage (the
+            // scan warps bound this kernel: a per-GT check before the publish cost 6 % at N = 32)
+            {
+                const int ob = __shfl_up_sync(0xffffffffu, cur.o, (unsigned)sg.g);
+                const int rr_l = lane >> 3;
+                const bool chk = lane < 16 && rr_l < sg.rows && (lane & 7) == sg.g;
+                if (__any_sync(0xffffffffu, chk && cur.o - ob != (rr_l ? rel[1] : rel[0])) && lane == 0)
+                    atomicOr(prm.ws_err, 2);
+            }
             skip2(it);
             if (it.valid()) fetch(it, cur);   // this warp's next stage
             return true;
