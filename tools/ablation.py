@@ -38,6 +38,7 @@ VARIANTS = [
     ("tc16", "tcgen05 kernel at N=16 (A fragments -> TMEM, kind::f16 MMA, D in TMEM)", ["--opt", "kernel=tc"], None),
     ("N8", "N=8 (decoupled-warp kernel, one n8 MMA per TCTile)", ["--N", "8"], None),
     ("tc32", "N=32, tcgen05 kernel (library default for N > 16)", ["--N", "32"], None),
+    ("dw32", "N=32, decoupled-warp kernel in half-GroupTile mode (two warps per GT, mma.sync)", ["--N", "32", "--opt", "kernel=dw"], None),
 ]
 
 NCU_METRICS = ["gpu__time_duration.sum", "dram__throughput.avg.pct_of_peak_sustained_elapsed",
